@@ -1,0 +1,366 @@
+#!/usr/bin/env python
+"""Benchmark of the mini-batch preparation hot path (BASELINE.json metric: seed
+nodes/s sampled+gathered per box; gather GB/s vs the HBM/NVLink roofline).
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--config products]
+    torchrun --nproc-per-node N bench.py --gpus N ...       (one rank per GPU)
+    python bench.py --impl reference ...                    (the CPU oracle arm)
+
+A step = one mini-batch of `seeds_per_batch` seeds per GPU through every hop of
+sampling + append-unique and the final feature gather.  The
+whole step is captured as two CUDA graphs (prep, gather) and replayed; each rank
+runs its own batches (b = r mod W) against the shared DSM (weak scaling).
+"""
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--config", default="products", choices=["tiny", "products", "papers100m", "mag240m"])
+    ap.add_argument("--impl", default="wg", choices=["wg", "reference"])
+    ap.add_argument("--no-flush", action="store_true", help="do not flush L2 between steps")
+    ap.add_argument("--no-graph", action="store_true", help="launch ops eagerly instead of graph replay")
+    ap.add_argument("--cpu-sample-s", type=float, default=12.0, help="target seconds of oracle work (cpu_baseline)")
+    ap.add_argument("--e2e-steps", type=int, default=20)
+    ap.add_argument("--out", default=None, help="also append the JSON line to this file")
+    return ap.parse_args()
+
+
+METRIC = "seed nodes/sec sampled+gathered per box"
+UNIT = "seeds/s"
+
+
+# ----------------------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled DURING the timed region."""
+
+    Q = ("index,clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+         "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu_index):
+        self.gpu = gpu_index
+        self.rows = []
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.25)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm = [float(r[1]) for r in self.rows if len(r) >= 9 and r[1].replace(".", "").isdigit()]
+        mx = [float(r[2]) for r in self.rows if len(r) >= 9 and r[2].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = set()
+        for r in self.rows:
+            if len(r) >= 9:
+                for k, nm in enumerate(names):
+                    if r[5 + k].lower() == "active":
+                        reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    return 6650.0, "fallback (B200_PROFILING.md)"
+
+
+# ----------------------------------------------------------------------------- oracle arm
+def run_oracle(preset, batches, sample_s, rank=0, world=1):
+    """Time the CPU oracle (as it stands, single-threaded) on whole batches of the
+    same workload; returns (seeds/s, seconds of oracle work, batches done, cores)."""
+    import contextlib
+
+    import oracle
+    from paper_conf_sc_yanglql22_b200 import loader
+    from synth import presets, seeds
+    os.sched_setaffinity(0, {sorted(os.sched_getaffinity(0))[0]})
+    rows = loader.host_row_provider(preset.graph())
+    feats = loader.host_feat_provider(preset)
+    spent = [0.0]
+
+    @contextlib.contextmanager
+    def timer():
+        t = time.perf_counter()
+        yield
+        spent[0] += time.perf_counter() - t
+    done = 0
+    for b in batches:
+        S = seeds.seed_nodes(preset.n, preset.seeds_per_batch, presets.SEED_BASE, b)
+        oracle.minibatch(rows, feats, S, preset.fanouts, seeds.rng_seed(presets.RNG_BASE, b), timer=timer)
+        done += 1
+        if spent[0] >= sample_s:
+            break
+    return done * preset.seeds_per_batch / spent[0], spent[0], done, len(os.sched_getaffinity(0))
+
+
+def bench_reference(args):
+    from synth import presets
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    p = presets.get(args.config)
+    per_step = []
+    total_s = 0.0
+    for k in range(args.warmup + args.steps):
+        v, s, done, cores = run_oracle(p, [k], 0.0)
+        if k >= args.warmup:
+            per_step.append(s)
+            total_s += s
+    value = args.steps * p.seeds_per_batch / total_s
+    line = {"impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * total_s / args.steps,
+            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "int64+fp32-bytes",
+            "data": "synthetic", "config": workload_config(p, 1),
+            "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle",
+                             "sample": f"{args.steps} whole batches of {p.seeds_per_batch} seeds "
+                                       f"(fanout {p.fanouts} + gather), rows regenerated per hop (untimed)"},
+            "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    emit(line, args)
+
+
+def workload_config(p, W, flushed=True):
+    return {"workload": p.name, "nodes": p.n, "csr_entries_target": p.target_e, "fanouts": p.fanouts,
+            "seeds_per_gpu": p.seeds_per_batch, "features": f"{p.feat_dim}x{p.feat_dtype}",
+            "parallelism": f"dsm-w{W} (row-sharded CSR+features, P2P loads, no hot-path collective)",
+            "l2": "flushed between steps (512 MB write outside the events)" if flushed else "not flushed",
+            "note": p.note}
+
+
+def emit(line, args):
+    s = json.dumps(line)
+    print(s, flush=True)
+    if args.out:
+        with open(args.out, "a") as f:
+            f.write(s + "\n")
+
+
+# ----------------------------------------------------------------------------- GPU arm
+def bench_wg(args):
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_sc_yanglql22_b200 as pkg
+    from paper_conf_sc_yanglql22_b200 import loader
+    from synth import presets, seeds
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    ag = None
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+        ag = pkg.TorchDistAllgather(device=dev)
+    p = presets.get(args.config)
+    S = p.seeds_per_batch
+    t0 = time.perf_counter()
+    dsm, info = loader.build_dsm(p, rank=rank, world=world, device=local, allgather=ag)
+    setup_s = time.perf_counter() - t0
+    pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, S)
+    nsteps = args.warmup + args.steps
+    my_batches = [k * world + rank for k in range(nsteps)]
+    seeds_dev = [torch.from_numpy(seeds.seed_nodes(p.n, S, presets.SEED_BASE, b)).to(dev) for b in my_batches]
+    rngs = [seeds.rng_seed(presets.RNG_BASE, b) for b in my_batches]
+    flush = None if args.no_flush else torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+
+    # warm-up (eager), then capture prep and gather as two graphs
+    for k in range(args.warmup):
+        pipe.run(seeds_dev[k], rngs[k])
+    torch.cuda.synchronize()
+    g_prep = g_gather = None
+    if not args.no_graph:
+        s = torch.cuda.Stream(device=dev)
+        s.wait_stream(torch.cuda.current_stream())
+        g_prep, g_gather = torch.cuda.CUDAGraph(), torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g_prep, stream=s):
+            pipe.enqueue(gather=False)
+        with torch.cuda.graph(g_gather, stream=s):
+            pipe.enqueue_gather()
+        torch.cuda.current_stream().wait_stream(s)
+        torch.cuda.synchronize()
+        for k in range(args.warmup):     # warm the graphs too
+            pipe.set_inputs(seeds_dev[k], rngs[k])
+            g_prep.replay()
+            g_gather.replay()
+        torch.cuda.synchronize()
+    err = dsm.device_error()
+    assert err == 0, f"device error {err:#x} during warm-up"
+
+    stream = torch.cuda.current_stream()
+    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
+    rows_gathered = torch.zeros(args.steps, dtype=torch.int64, device=dev)
+    hop_counts = torch.zeros((args.steps, len(p.fanouts), 2), dtype=torch.int64, device=dev)
+    clocks = ClockSampler(local)
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    clocks.start()
+    wall0 = time.perf_counter()
+    for i in range(args.steps):
+        k = args.warmup + i
+        if flush is not None:
+            flush.fill_(i & 0xFF)
+        ev[i][0].record(stream)
+        pipe.set_inputs(seeds_dev[k], rngs[k])
+        if g_prep is not None:
+            g_prep.replay()
+        else:
+            pipe.enqueue(gather=False)
+        ev[i][1].record(stream)
+        if g_gather is not None:
+            g_gather.replay()
+        else:
+            pipe.enqueue_gather()
+        ev[i][2].record(stream)
+        rows_gathered[i:i + 1].copy_(pipe.hops[-1]["num_unique"])
+        for h, b in enumerate(pipe.hops):
+            hop_counts[i, h, 0:1].copy_(b["num_edges"])
+            hop_counts[i, h, 1:2].copy_(b["num_unique"])
+    torch.cuda.synchronize()
+    if world > 1:
+        dist.barrier()
+    wall = time.perf_counter() - wall0
+    clk = clocks.stop()
+    step_ms = [ev[i][0].elapsed_time(ev[i][2]) for i in range(args.steps)]
+    gather_ms = [ev[i][1].elapsed_time(ev[i][2]) for i in range(args.steps)]
+    dev_s = sum(step_ms) / 1e3
+    err = dsm.device_error()
+    assert err == 0, f"device error {err:#x} in the timed region"
+    if world > 1:
+        t = torch.tensor([dev_s], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dev_s = float(t.item())
+    value = world * S * args.steps / dev_s
+    rb = dsm.row_bytes
+    rows = rows_gathered.cpu().numpy()
+    hc = hop_counts.cpu().numpy()
+    gather_s = sum(gather_ms) / 1e3
+    alg_bytes = float(2 * rows.sum() * rb)           # read + write per gathered row (W=1: all local HBM)
+    peak, peak_src = peaks()
+    achieved = alg_bytes / gather_s / 1e9
+    if world > 1:
+        remote = (world - 1) / world
+        bound = "nvlink" if remote * rows.mean() * rb / 770e9 > 2 * rows.mean() * rb / (peak * 1e9) else "hbm"
+    else:
+        bound = "hbm"
+
+    # ---- e2e through the public API with pinned host buffers (H2D seeds, D2H counts)
+    e2e_times = []
+    d2h = torch.empty((len(p.fanouts), 2), dtype=torch.int64, pin_memory=True)
+    host_seeds = [seeds_dev[k % nsteps].cpu().pin_memory() for k in range(args.e2e_steps)]
+    for i in range(args.e2e_steps + 2):
+        hs = host_seeds[i % len(host_seeds)]
+        torch.cuda.synchronize()
+        t = time.perf_counter()
+        pipe.set_inputs(hs, rngs[i % nsteps])
+        if g_prep is not None:
+            g_prep.replay()
+            g_gather.replay()
+        else:
+            pipe.enqueue()
+        for h, b in enumerate(pipe.hops):
+            d2h[h, 0:1].copy_(b["num_edges"], non_blocking=True)
+            d2h[h, 1:2].copy_(b["num_unique"], non_blocking=True)
+        torch.cuda.current_stream().synchronize()
+        if i >= 2:
+            e2e_times.append(time.perf_counter() - t)
+    e2e_val = S / statistics.mean(e2e_times)
+    if world > 1:
+        t = torch.tensor([statistics.mean(e2e_times)], dtype=torch.float64, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        e2e_val = world * S / float(t.item())
+
+    line = None
+    if rank == 0:
+        cpu = None
+        if world == 1 and args.cpu_sample_s > 0:
+            v, s_spent, done, cores = run_oracle(p, range(10_000, 10_100), args.cpu_sample_s)
+            cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
+                   "sample": f"{done} whole batches of {S} seeds (fanout {p.fanouts} + gather) of the same workload, "
+                             f"{s_spent:.1f} s of single-threaded oracle work (row regeneration untimed)"}
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 1e3 * dev_s / args.steps, "higher_is_better": True,
+            "scaling": "weak", "vs_baseline": None, "dtype": "int64 ids + fp32 feature bytes",
+            "data": "synthetic (seeded power-law graph + procedural features, see DESIGN.md)",
+            "config": workload_config(p, world, flush is not None),
+            "roofline": {"kernel": "wg::gather_kernel", "bound": bound, "achieved": achieved, "peak": peak,
+                         "unit": "GB/s", "frac": achieved / peak, "traffic": None,
+                         "peak_source": peak_src,
+                         "algorithmic_bytes_per_launch": alg_bytes / args.steps,
+                         "gather_ms_per_step": 1e3 * gather_s / args.steps,
+                         "gather_share_of_step": gather_s / dev_s},
+            "cpu_baseline": cpu,
+            "e2e": {"value": e2e_val, "unit": UNIT, "h2d_bytes_per_step": S * 8,
+                    "d2h_bytes_per_step": int(d2h.numel() * 8),
+                    "note": "public API (MiniBatchPipeline.run): pinned-host seeds H2D, per-hop counts D2H, "
+                            "host-timed incl. sync"},
+            "gpu_launches": args.steps * (4 * len(p.fanouts) + 1),
+            "clocks": clk,
+            "wall_s_timed_region": wall,
+            "workload_stats": {"edges_per_hop_mean": hc[:, :, 0].mean(0).tolist(),
+                               "unique_per_hop_mean": hc[:, :, 1].mean(0).tolist(),
+                               "unique_bound_per_hop": pipe.U_cap, "rows_gathered_mean": float(rows.mean()),
+                               "row_bytes": rb},
+            "setup": {"total_s": setup_s, **info},
+            "step_ms_median": statistics.median(step_ms),
+        }
+        emit(line, args)
+    torch.cuda.synchronize()
+    dsm.destroy()
+    if world > 1:
+        dist.destroy_process_group()
+    return line
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        bench_reference(args)
+    else:
+        bench_wg(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,185 @@
+/*
+ * wg.h -- C ABI of the B200-native WholeGraph mini-batch preparation path.
+ *
+ * WholeGraph (Yang, Liu, Qi, Lai, SC'22; /root/reference/PAPER.md) prepares a
+ * GNN mini-batch on every GPU from a graph and a feature table held in a
+ * multi-GPU distributed shared memory (DSM).  Citations "L<n>" are PAPER.md
+ * lines; "A<n>" are the readings of ambiguous passages listed in DESIGN.md
+ * (section "Readings") and SURVEY.md 8(c).
+ *
+ * Conventions for every call below
+ *  - Pointers prefixed d_ are DEVICE pointers on the handle's device; the caller
+ *    owns them (e.g. torch tensors).  The handle owns the shards, the peer
+ *    mappings and an internal workspace (hash table, scan state, error word).
+ *  - Every op is stream-ordered and asynchronous: it enqueues kernels on
+ *    `stream` (a cudaStream_t; NULL = legacy default stream) and returns without
+ *    synchronising the host.  Calls on one handle must be issued on one stream
+ *    at a time (they share the workspace).  All ops are CUDA-graph capturable.
+ *  - Sizes n_* are HOST capacities (upper bounds, used to size launches and to
+ *    bound writes).  The optional d_n_* are DEVICE int64 scalars holding the
+ *    actual count produced by a previous call (e.g. d_out_num_edges), so hops
+ *    chain without a host sync; NULL means "use n_* exactly".  An actual count
+ *    larger than its capacity is clamped to the capacity and latches
+ *    WG_DEVERR_CAPACITY.
+ *  - Global node ids are int64 in [0, num_nodes) ("8 bytes to store each edge",
+ *    L236; A12).  Sub-graph (local) ids are int32.
+ *  - Argument errors are detected on the host and returned immediately
+ *    (nothing is enqueued).  Data errors found by kernels (an id out of range, a
+ *    duplicate target, a capacity overflow) are OR-ed into a device error word
+ *    read by wg_device_error(); the op still writes defined outputs.
+ *  - There is no CPU fallback: every op runs in the library's sm_100a kernels,
+ *    and wg_dsm_create returns WG_ERR_UNSUPPORTED on devices below sm_100.
+ */
+#ifndef WG_H_
+#define WG_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define WG_MAX_WORLD 8          /* ranks (GPUs) per DSM: one HGX B200 box */
+
+typedef struct wg_dsm* wg_dsm_t; /* opaque host handle, one per rank process */
+typedef void* wg_stream_t;       /* a cudaStream_t */
+
+typedef enum {
+  WG_OK = 0,
+  WG_ERR_INVALID_ARG = 1,  /* bad pointer / size / fanout; nothing enqueued */
+  WG_ERR_CUDA = 2,         /* a CUDA runtime call failed; see wg_last_error() */
+  WG_ERR_OOM = 3,          /* device allocation failed */
+  WG_ERR_PEER_ACCESS = 4,  /* IPC export/import of a peer shard failed */
+  WG_ERR_CAPACITY = 5,     /* request exceeds the workspace sized at create */
+  WG_ERR_UNSUPPORTED = 6,  /* device below sm_100, or fanout > 32 */
+  WG_ERR_COLLECTIVE = 7    /* the allgather callback returned non-zero */
+} wg_status;
+
+typedef enum { WG_F32 = 0, WG_F16 = 1, WG_BF16 = 2 } wg_dtype;
+
+/* Bits of the latched device error word (wg_device_error). */
+#define WG_DEVERR_ID_RANGE   0x1u  /* a node id outside [0, num_nodes): treated as degree 0 / skipped */
+#define WG_DEVERR_DUP_TARGET 0x2u  /* wg_append_unique: duplicate target (A8) */
+#define WG_DEVERR_CAPACITY   0x4u  /* a device count exceeded its host capacity, or the hash table filled */
+#define WG_DEVERR_DEGREE     0x8u  /* a degree >= 2^32 (A3 requires N < 2^32) */
+#define WG_DEVERR_EPOCH      0x10u /* hash-table epoch space exhausted: call wg_dsm_reset_workspace */
+
+/* Allgather of host bytes across the W ranks of the DSM ("an
+ * AllGather pattern communication is performed so that each process can get all
+ * the CUDA IPC handles").  recv receives world_size * bytes_per_rank bytes in
+ * rank order.  bytes_per_rank == 0 must act as a barrier.  Return 0 on success.
+ * Used only inside wg_dsm_create / wg_dsm_destroy (setup), never on the hot path. */
+typedef int (*wg_allgather_fn)(const void* send, void* recv, size_t bytes_per_rank, void* ctx);
+
+typedef struct {
+  int32_t rank;             /* this process's rank in [0, world_size) */
+  int32_t world_size;       /* W, 1 <= W <= WG_MAX_WORLD */
+  int32_t device;           /* CUDA device ordinal this rank drives ("one process
+                               usually controls one single GPU", L98) */
+  int32_t feat_dtype;       /* wg_dtype; only sets the element size (rows move as bytes, A14) */
+  int64_t num_nodes;        /* n; node v lives on rank o(v) = v mod W at local row
+                               l(v) = v div W (hash partition, L110; A11) */
+  int64_t local_num_edges;  /* CSR entries of the rows THIS rank owns ("edges are
+                               stored together with the source node", L110) */
+  int64_t feat_dim;         /* feature columns per node (0 = no feature table) */
+  int64_t max_batch_keys;   /* workspace sizing: the largest n_targets + n_nbrs
+                               passed to wg_append_unique and the largest
+                               n_targets passed to wg_sample_neighbors */
+  wg_allgather_fn allgather;
+  void* ctx;                /* passed through to allgather */
+} wg_dsm_desc;
+
+/* Create the DSM (section III-B).  COLLECTIVE over the W ranks.
+ * Each rank allocates its shard slab on its device -- row_ptr int64[n_local+1],
+ * col_idx int64[local_num_edges], features [n_local][row stride] with the row
+ * stride rounded up to 16 bytes -- exports a CUDA IPC handle, allgathers the
+ * handles (L100), opens every peer's handle (L100-106; same-process peers are used
+ * directly) and keeps the W base pointers as the "memory pointer table" (L106),
+ * passed by value to every kernel.  n_local = number of v in [0,n) with v mod W == rank.
+ * The shard contents are undefined until the caller fills them through
+ * wg_dsm_local_view and all ranks pass a barrier.
+ * Errors: WG_ERR_INVALID_ARG, WG_ERR_UNSUPPORTED, WG_ERR_OOM, WG_ERR_PEER_ACCESS,
+ * WG_ERR_COLLECTIVE, WG_ERR_CUDA.  On error *out is NULL and nothing leaks. */
+wg_status wg_dsm_create(const wg_dsm_desc* desc, wg_dsm_t* out);
+
+/* Device pointers of THIS rank's shard, for filling it (any stream; the caller
+ * synchronises and barriers before other ranks read).  Any output may be NULL.
+ * feat_row_stride_bytes is the padded row pitch of the feature shard. */
+wg_status wg_dsm_local_view(wg_dsm_t h, int64_t** d_row_ptr, int64_t** d_col_idx, void** d_feat,
+                            int64_t* n_local_rows, int64_t* feat_row_stride_bytes);
+
+/* Geometry of rank r's shard (any r): local rows and local CSR entries. */
+wg_status wg_dsm_shard_info(wg_dsm_t h, int32_t r, int64_t* n_local_rows, int64_t* local_num_edges);
+
+/* Destroy (COLLECTIVE): barrier (no rank still reads a peer), close the peer
+ * mappings, barrier (no peer still maps ours), free the shard and workspace.
+ * The caller must have synchronised every stream that used the handle. */
+wg_status wg_dsm_destroy(wg_dsm_t h);
+
+/* Multi-GPU sampling op, one hop (Algorithm 1).
+ * For target k (in input order) with N = deg(d_targets[k]) read from the owner's
+ * row_ptr (local HBM or a peer's over NVLink):
+ *   - if fanout >= N: all N neighbours, in CSR order ("all of N neighbors are
+ *     sampled", L118; A5);
+ *   - else: fanout neighbours drawn without replacement by Algorithm 1 with draw
+ *     r_i = floor(x_i * (N-i) / 2^32), x_i = word (i & 3) of Philox4x32-10 at
+ *     counter (i>>2, hop, lo32(node), hi32(node)) under key (lo32(seed),
+ *     hi32(seed)) (A2, A3), output in draw order i = 0..fanout-1 (A5).
+ * Outputs: d_out_row_ptr int64[n_targets+1] = exclusive prefix of min(fanout, N)
+ * (the sub-graph CSR row pointer, L166); d_out_nbrs int64[cap n_targets*fanout]
+ * = sampled global ids; d_out_pos int32[same] (nullable) = positions in the
+ * adjacency list; d_out_num_edges (nullable) = device int64 total.
+ * seed: the per-batch rng_seed; if d_seed is non-NULL the seed is read from that
+ * device uint64 instead (so a captured CUDA graph can be replayed with new seeds).
+ * Requires 1 <= fanout <= 32 (WG_ERR_UNSUPPORTED above 32). */
+wg_status wg_sample_neighbors(wg_dsm_t h, const int64_t* d_targets, int64_t n_targets,
+                              const int64_t* d_n_targets, int32_t fanout, uint64_t seed,
+                              const uint64_t* d_seed, int32_t hop, int64_t* d_out_row_ptr,
+                              int64_t* d_out_nbrs, int32_t* d_out_pos, int64_t* d_out_num_edges,
+                              wg_stream_t stream);
+
+/* Append Unique op: U = the targets first, in input order,
+ * with their index as sub-graph id (L160, L166), then every neighbour id not seen
+ * before, numbered continuously after the targets in order of first appearance
+ * in d_nbrs (A7; the paper's hash-bucket order is nondeterministic).  A
+ * neighbour equal to a target takes the target's id (A9).  Duplicate targets
+ * latch WG_DEVERR_DUP_TARGET (A8).
+ * Outputs: d_out_unique int64[cap n_targets+n_nbrs]; d_out_num_unique device
+ * int64 (nullable); d_out_sub_col int32[n_nbrs] = sub-graph id of each sampled
+ * neighbour (with d_out_row_ptr of the sampling op this is the sub-graph CSR,
+ * L166); d_out_dup_count int32[cap n_targets+n_nbrs] (nullable) = how many
+ * times each sub-graph node was sampled as a neighbour (the duplicate count, L186).
+ * Requires n_targets + n_nbrs <= max_batch_keys and < 2^31. */
+wg_status wg_append_unique(wg_dsm_t h, const int64_t* d_targets, int64_t n_targets,
+                           const int64_t* d_n_targets, const int64_t* d_nbrs, int64_t n_nbrs,
+                           const int64_t* d_n_nbrs, int64_t* d_out_unique, int64_t* d_out_num_unique,
+                           int32_t* d_out_sub_col, int32_t* d_out_dup_count, wg_stream_t stream);
+
+/* Global gather: d_out[i][:] = the feature row of node
+ * d_ids[i], in input order, read from the owner's shard (local HBM or a peer's
+ * over NVLink) by one kernel ("a single gather kernel in each GPU", L182).  Rows
+ * are copied as raw bytes: d_out is dense, row i at i * feat_dim * elt_size.
+ * Repeated ids are allowed. */
+wg_status wg_gather(wg_dsm_t h, const int64_t* d_ids, int64_t n_ids, const int64_t* d_n_ids,
+                    void* d_out, wg_stream_t stream);
+
+/* Read (and optionally clear) the latched device error word.  Synchronises the
+ * handle's device. */
+wg_status wg_device_error(wg_dsm_t h, uint32_t* code, int32_t clear);
+
+/* Clear the append-unique hash table and restart its epoch counter (needed only
+ * after WG_DEVERR_EPOCH, i.e. after ~8M wg_append_unique calls).  Stream-ordered. */
+wg_status wg_dsm_reset_workspace(wg_dsm_t h, wg_stream_t stream);
+
+/* Thread-local message describing the last non-OK status. */
+const char* wg_last_error(void);
+
+/* Library version string. */
+const char* wg_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* WG_H_ */

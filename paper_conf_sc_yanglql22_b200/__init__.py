@@ -1,0 +1,11 @@
+"""B200-native WholeGraph mini-batch preparation (Yang et al., SC'22).
+
+The hot path -- multi-hop neighbour sampling, append-unique and global gather
+over a multi-GPU distributed shared memory -- runs in hand-written sm_100a CUDA
+kernels behind the C ABI declared in include/wg.h (libwg.so).  This package is
+the thin Python binding (argument marshalling) plus the batch pipeline.
+"""
+
+from ._lib import LIB_PATH, WgError, lib  # noqa: F401
+from .dsm import DSM, ThreadAllgather, TorchDistAllgather, local_num_edges, shard_csr  # noqa: F401
+from .pipeline import MiniBatchPipeline, capacities, required_keys  # noqa: F401

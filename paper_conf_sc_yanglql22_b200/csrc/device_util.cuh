@@ -1,0 +1,152 @@
+// device_util.cuh -- device helpers of the CUDA path: Philox, warp/block scans,
+// single-pass decoupled look-back, cache-hinted vector loads.
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace wg {
+
+constexpr unsigned FULL_MASK = 0xffffffffu;
+
+// Philox4x32-10 (Salmon et al. SC'11), the counter-based generator of reading A3.
+__device__ __forceinline__ uint4 philox4x32_10(uint4 c, uint2 k) {
+#pragma unroll
+  for (int r = 0; r < 10; ++r) {
+    if (r) {
+      k.x += 0x9E3779B9u;
+      k.y += 0xBB67AE85u;
+    }
+    const unsigned hi0 = __umulhi(0xD2511F53u, c.x), lo0 = 0xD2511F53u * c.x;
+    const unsigned hi1 = __umulhi(0xCD9E8D57u, c.z), lo1 = 0xCD9E8D57u * c.z;
+    c = make_uint4(hi1 ^ c.y ^ k.x, lo1, hi0 ^ c.w ^ k.y, lo0);
+  }
+  return c;
+}
+
+__device__ __forceinline__ unsigned long long ld_volatile_u64(const unsigned long long* p) {
+  return *reinterpret_cast<const volatile unsigned long long*>(p);
+}
+__device__ __forceinline__ void st_volatile_u64(unsigned long long* p, unsigned long long v) {
+  *reinterpret_cast<volatile unsigned long long*>(p) = v;
+}
+
+// 16-byte read-only load that does not allocate in L1 (each feature byte is read once).
+__device__ __forceinline__ uint4 ld_nc_na_v4(const void* p) {
+  uint4 r;
+  asm("ld.global.nc.L1::no_allocate.v4.u32 {%0,%1,%2,%3}, [%4];"
+      : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+      : "l"(p));
+  return r;
+}
+__device__ __forceinline__ unsigned ld_nc_na_u32(const void* p) {
+  unsigned r;
+  asm("ld.global.nc.L1::no_allocate.u32 %0, [%1];" : "=r"(r) : "l"(p));
+  return r;
+}
+__device__ __forceinline__ unsigned short ld_nc_na_u16(const void* p) {
+  unsigned short r;
+  asm("ld.global.nc.L1::no_allocate.u16 %0, [%1];" : "=h"(r) : "l"(p));
+  return r;
+}
+
+template <typename T>
+__device__ __forceinline__ T warp_inclusive_sum(T v, int lane) {
+#pragma unroll
+  for (int d = 1; d < 32; d <<= 1) {
+    T o = __shfl_up_sync(FULL_MASK, v, d);
+    if (lane >= d) v += o;
+  }
+  return v;
+}
+
+template <typename T>
+__device__ __forceinline__ T warp_sum(T v) {
+#pragma unroll
+  for (int d = 16; d > 0; d >>= 1) v += __shfl_xor_sync(FULL_MASK, v, d);
+  return v;
+}
+
+// Block-wide exclusive sum for NT threads (NT multiple of 32, <= 1024).
+// warp_tot must have room for NT/32 values.  Returns the exclusive prefix;
+// *total receives the block aggregate (in every thread).
+template <int NT, typename T>
+__device__ __forceinline__ T block_exclusive_sum(T v, T* warp_tot, T* total) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  T inc = warp_inclusive_sum(v, lane);
+  if (lane == 31) warp_tot[warp] = inc;
+  __syncthreads();
+  if (warp == 0) {
+    T w = lane < NT / 32 ? warp_tot[lane] : T(0);
+    T wi = warp_inclusive_sum(w, lane);
+    if (lane < NT / 32) warp_tot[lane] = wi - w;  // exclusive warp offsets
+    if (lane == NT / 32 - 1) warp_tot[NT / 32] = wi;
+  }
+  __syncthreads();
+  *total = warp_tot[NT / 32];
+  return warp_tot[warp] + inc - v;
+}
+
+// ---------------------------------------------------------------- decoupled look-back
+// Tile status word: bits 63..62 = flag (0 none, 1 aggregate, 2 inclusive prefix),
+// bits 61..0 = value.  Flag and value share one 64-bit word, so publication needs
+// no fence.  Called by ALL 32 lanes of one warp; returns the tile's exclusive
+// prefix in every lane and publishes the inclusive prefix.
+constexpr unsigned long long LB_AGG = 1ull << 62, LB_PRE = 2ull << 62, LB_VAL = (1ull << 62) - 1;
+
+__device__ __forceinline__ unsigned long long tile_lookback(unsigned long long* status, long tile,
+                                                            unsigned long long aggregate) {
+  const int lane = threadIdx.x & 31;
+  if (tile == 0) {
+    if (lane == 0) st_volatile_u64(&status[0], LB_PRE | aggregate);
+    return 0;
+  }
+  if (lane == 0) st_volatile_u64(&status[tile], LB_AGG | aggregate);
+  unsigned long long excl = 0;
+  long pred = tile - 1;
+  for (;;) {
+    const long idx = pred - lane;
+    unsigned long long s = idx >= 0 ? ld_volatile_u64(&status[idx]) : LB_PRE;
+    while (__any_sync(FULL_MASK, (s >> 62) == 0)) {
+      if ((s >> 62) == 0) {
+        __nanosleep(20);
+        s = ld_volatile_u64(&status[idx]);
+      }
+    }
+    const unsigned pmask = __ballot_sync(FULL_MASK, (s >> 62) == 2);
+    const int stop = pmask ? __ffs(pmask) - 1 : 31;
+    unsigned long long v = lane <= stop ? (s & LB_VAL) : 0ull;
+    excl += warp_sum(v);
+    if (pmask) break;
+    pred -= 32;
+  }
+  if (lane == 0) st_volatile_u64(&status[tile], LB_PRE | (excl + aggregate));
+  return excl;
+}
+
+// Last-block cleanup: every block calls this once at its very end (all threads).
+// Returns true (in every thread of the block) for the block that finished last;
+// by then no other block of this launch reads the look-back status any more.
+__device__ __forceinline__ bool finish_block(unsigned* done, int* smem_flag) {
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    __threadfence();
+    const unsigned prev = atomicAdd(done, 1u);
+    *smem_flag = (prev == gridDim.x - 1);
+  }
+  __syncthreads();
+  return *smem_flag != 0;
+}
+
+__device__ __forceinline__ void latch_error(unsigned* ctrl_err, unsigned bits) { atomicOr(ctrl_err, bits); }
+
+__device__ __forceinline__ unsigned long long fmix64(unsigned long long k) {
+  k ^= k >> 33;
+  k *= 0xff51afd7ed558ccdull;
+  k ^= k >> 33;
+  k *= 0xc4ceb9fe1a85ec53ull;
+  k ^= k >> 33;
+  return k;
+}
+
+}  // namespace wg

@@ -1,0 +1,354 @@
+// dsm.cu -- the multi-GPU distributed shared memory (section III-B)
+// and the C-ABI entry points of include/wg.h.
+//
+// Each rank allocates ONE slab on its GPU holding its three shards
+//   [ row_ptr int64[n_local+1] | col_idx int64[e_local] | feat[n_local][stride] ]
+// (256-byte aligned sub-offsets; cudaMalloc of >= 2 MB uses 2 MB pages, so TLB reach
+// covers the shards with few entries), exports a CUDA IPC handle, allgathers a fixed
+// record {pid, device pointer, IPC handle, geometry} through the caller's callback
+// (L100), opens every peer's handle with cudaIpcOpenMemHandle (L100-106) -- a peer
+// in the SAME process (in-process virtual ranks) is used directly -- and keeps the
+// per-rank base pointers as the "memory pointer table" (L106), which travels to
+// every kernel by value inside ShardView.
+#include <unistd.h>
+
+#include <cstdio>
+#include <cstring>
+#include <string>
+
+#include "device_util.cuh"
+#include "wg_internal.cuh"
+
+namespace wg {
+
+static thread_local std::string g_last_error;
+
+void set_error(const std::string& msg) { g_last_error = msg; }
+wg_status fail(wg_status s, const std::string& msg) {
+  g_last_error = msg;
+  return s;
+}
+
+static int64_t round_up(int64_t x, int64_t a) { return (x + a - 1) / a * a; }
+
+static int64_t local_rows(int64_t n, int rank, int world) {
+  return n > rank ? (n - rank + world - 1) / world : 0;
+}
+
+struct PeerRecord {
+  int64_t pid;
+  uint64_t dev_ptr;
+  int64_t slab_bytes;
+  int64_t n_local;
+  int64_t e_local;
+  int64_t off_col;
+  int64_t off_feat;
+  int64_t num_nodes;
+  int64_t feat_stride;
+  int32_t world;
+  int32_t rank;
+  cudaIpcMemHandle_t handle;
+};
+
+static wg_status barrier(wg_dsm* h) {
+  if (h->world == 1) return WG_OK;
+  if (h->allgather(nullptr, nullptr, 0, h->ctx) != 0) return fail(WG_ERR_COLLECTIVE, "barrier: allgather callback failed");
+  return WG_OK;
+}
+
+static void free_workspace(wg_dsm* h) {
+  Workspace& w = h->ws;
+  cudaFree(w.hkeys);
+  cudaFree(w.hvals);
+  cudaFree(w.status_sample);
+  cudaFree(w.status_unique);
+  cudaFree(w.excl);
+  cudaFree(w.ctrl);
+  w = Workspace{};
+}
+
+static wg_status alloc_workspace(wg_dsm* h, int64_t max_keys) {
+  Workspace& w = h->ws;
+  if (max_keys < 1) max_keys = 1;
+  int64_t cap = 1024;
+  while (cap < 2 * max_keys) cap <<= 1;  // load factor <= 0.5
+  w.hcap = cap;
+  w.max_keys = max_keys;
+  w.status_cap = max_keys / 256 + 2;
+  if (cudaMalloc(&w.hkeys, cap * 8) != cudaSuccess || cudaMalloc(&w.hvals, cap * 8) != cudaSuccess ||
+      cudaMalloc(&w.status_sample, w.status_cap * 8) != cudaSuccess ||
+      cudaMalloc(&w.status_unique, w.status_cap * 8) != cudaSuccess ||
+      cudaMalloc(&w.excl, max_keys * 4) != cudaSuccess || cudaMalloc(&w.ctrl, CTRL_WORDS * 4) != cudaSuccess) {
+    cudaGetLastError();
+    free_workspace(h);
+    return fail(WG_ERR_OOM, "workspace allocation failed");
+  }
+  WG_CUDA_TRY(cudaMemset(w.hkeys, 0, cap * 8));
+  WG_CUDA_TRY(cudaMemset(w.hvals, 0xff, cap * 8));
+  WG_CUDA_TRY(cudaMemset(w.status_sample, 0, w.status_cap * 8));
+  WG_CUDA_TRY(cudaMemset(w.status_unique, 0, w.status_cap * 8));
+  unsigned ctrl[CTRL_WORDS] = {0};
+  ctrl[CTRL_EPOCH] = 1;
+  WG_CUDA_TRY(cudaMemcpy(w.ctrl, ctrl, sizeof(ctrl), cudaMemcpyHostToDevice));
+  return WG_OK;
+}
+
+static void release(wg_dsm* h) {
+  for (int r = 0; r < h->world; ++r)
+    if (h->peer_opened[r]) cudaIpcCloseMemHandle(h->peer_base[r]);
+  free_workspace(h);
+  if (h->slab) cudaFree(h->slab);
+  delete h;
+}
+
+}  // namespace wg
+
+using namespace wg;
+
+extern "C" {
+
+const char* wg_last_error(void) { return g_last_error.c_str(); }
+const char* wg_version(void) { return "wholegraph-b200 0.1 (sm_100a)"; }
+
+wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
+  if (!out) return fail(WG_ERR_INVALID_ARG, "out is NULL");
+  *out = nullptr;
+  if (!d) return fail(WG_ERR_INVALID_ARG, "desc is NULL");
+  if (d->world_size < 1 || d->world_size > WG_MAX_WORLD || d->rank < 0 || d->rank >= d->world_size)
+    return fail(WG_ERR_INVALID_ARG, "rank/world_size out of range");
+  if (d->num_nodes < 0 || d->num_nodes >= (int64_t(1) << 40) || d->local_num_edges < 0 || d->feat_dim < 0 ||
+      d->max_batch_keys < 0 || d->max_batch_keys >= (int64_t(1) << 31))
+    return fail(WG_ERR_INVALID_ARG, "sizes out of range (num_nodes < 2^40, max_batch_keys < 2^31)");
+  if (d->feat_dtype < WG_F32 || d->feat_dtype > WG_BF16) return fail(WG_ERR_INVALID_ARG, "feat_dtype");
+  if (d->world_size > 1 && !d->allgather) return fail(WG_ERR_INVALID_ARG, "allgather callback required for W > 1");
+
+  WG_CUDA_TRY(cudaSetDevice(d->device));
+  int major = 0, minor = 0, sms = 0;
+  WG_CUDA_TRY(cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, d->device));
+  WG_CUDA_TRY(cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, d->device));
+  WG_CUDA_TRY(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, d->device));
+  if (major * 10 + minor < 100) return fail(WG_ERR_UNSUPPORTED, "needs an sm_100 (Blackwell) device");
+
+  wg_dsm* h = new wg_dsm();
+  h->rank = d->rank;
+  h->world = d->world_size;
+  h->device = d->device;
+  h->n = d->num_nodes;
+  h->feat_dim = d->feat_dim;
+  h->elt = d->feat_dtype == WG_F32 ? 4 : 2;
+  h->row_bytes = h->feat_dim * h->elt;
+  h->feat_stride = round_up(h->row_bytes, 16);
+  h->allgather = d->allgather;
+  h->ctx = d->ctx;
+  h->sm_count = sms;
+  h->n_local = local_rows(h->n, h->rank, h->world);
+  h->e_local = d->local_num_edges;
+
+  // ---- this rank's slab
+  const int64_t off_col = round_up((h->n_local + 1) * 8, 256);
+  const int64_t off_feat = round_up(off_col + h->e_local * 8, 256);
+  h->slab_bytes = (size_t)round_up(off_feat + h->n_local * h->feat_stride, 256);
+  if (cudaMalloc(&h->slab, h->slab_bytes) != cudaSuccess) {
+    cudaGetLastError();
+    h->slab = nullptr;
+    release(h);
+    return fail(WG_ERR_OOM, "shard allocation of " + std::to_string(h->slab_bytes) + " bytes failed");
+  }
+  wg_status st = alloc_workspace(h, d->max_batch_keys);
+  if (st != WG_OK) {
+    std::string m = g_last_error;
+    release(h);
+    return fail(st, m);
+  }
+
+  // ---- export + allgather the IPC handles (L100)
+  PeerRecord mine;
+  std::memset(&mine, 0, sizeof(mine));
+  mine.pid = (int64_t)getpid();
+  mine.dev_ptr = (uint64_t)(uintptr_t)h->slab;
+  mine.slab_bytes = (int64_t)h->slab_bytes;
+  mine.n_local = h->n_local;
+  mine.e_local = h->e_local;
+  mine.off_col = off_col;
+  mine.off_feat = off_feat;
+  mine.num_nodes = h->n;
+  mine.feat_stride = h->feat_stride;
+  mine.world = h->world;
+  mine.rank = h->rank;
+  PeerRecord all[WG_MAX_WORLD];
+  std::memset(all, 0, sizeof(all));
+  if (h->world > 1) {
+    if (cudaIpcGetMemHandle(&mine.handle, h->slab) != cudaSuccess) {
+      cudaGetLastError();
+      release(h);
+      return fail(WG_ERR_PEER_ACCESS, "cudaIpcGetMemHandle failed");
+    }
+    if (h->allgather(&mine, all, sizeof(PeerRecord), h->ctx) != 0) {
+      release(h);
+      return fail(WG_ERR_COLLECTIVE, "allgather of IPC handles failed");
+    }
+  } else {
+    all[0] = mine;
+  }
+  for (int r = 0; r < h->world; ++r) {
+    if (all[r].rank != r || all[r].world != h->world || all[r].num_nodes != h->n ||
+        all[r].feat_stride != h->feat_stride) {
+      release(h);
+      return fail(WG_ERR_INVALID_ARG, "ranks disagree on world_size / num_nodes / feat_dim");
+    }
+  }
+
+  // ---- open peers (L100-106) and build the memory pointer table (L106)
+  for (int r = 0; r < h->world; ++r) {
+    h->n_local_of[r] = all[r].n_local;
+    h->e_local_of[r] = all[r].e_local;
+    if (r == h->rank) {
+      h->peer_base[r] = h->slab;
+    } else if (all[r].pid == mine.pid) {
+      h->peer_base[r] = (void*)(uintptr_t)all[r].dev_ptr;  // same process: plain device pointer
+    } else {
+      void* p = nullptr;
+      cudaError_t e = cudaIpcOpenMemHandle(&p, all[r].handle, cudaIpcMemLazyEnablePeerAccess);
+      if (e != cudaSuccess) {
+        cudaGetLastError();
+        release(h);
+        return fail(WG_ERR_PEER_ACCESS, std::string("cudaIpcOpenMemHandle: ") + cudaGetErrorString(e));
+      }
+      h->peer_base[r] = p;
+      h->peer_opened[r] = true;
+    }
+    uint8_t* b = static_cast<uint8_t*>(h->peer_base[r]);
+    h->view.row_ptr[r] = reinterpret_cast<const int64_t*>(b);
+    h->view.col[r] = reinterpret_cast<const int64_t*>(b + all[r].off_col);
+    h->view.feat[r] = b + all[r].off_feat;
+  }
+  h->view.n = h->n;
+  h->view.feat_stride = h->feat_stride;
+  h->view.world = h->world;
+  h->view.log2w = -1;
+  for (int k = 0; k <= 3; ++k)
+    if ((1 << k) == h->world) h->view.log2w = k;
+  // Zero this rank's row_ptr sentinel so an unfilled shard reads as degree 0.
+  if (cudaMemset(h->slab, 0, (h->n_local + 1) * 8) != cudaSuccess) {
+    cudaGetLastError();
+    release(h);
+    return fail(WG_ERR_CUDA, "memset row_ptr");
+  }
+  if (cudaDeviceSynchronize() != cudaSuccess || barrier(h) != WG_OK) {
+    release(h);
+    return fail(WG_ERR_COLLECTIVE, "create: final barrier failed");
+  }
+  *out = h;
+  return WG_OK;
+}
+
+wg_status wg_dsm_local_view(wg_dsm_t h, int64_t** row_ptr, int64_t** col, void** feat, int64_t* n_local_rows,
+                            int64_t* stride) {
+  if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
+  uint8_t* b = static_cast<uint8_t*>(h->slab);
+  if (row_ptr) *row_ptr = const_cast<int64_t*>(h->view.row_ptr[h->rank]);
+  if (col) *col = const_cast<int64_t*>(h->view.col[h->rank]);
+  if (feat) *feat = const_cast<uint8_t*>(h->view.feat[h->rank]);
+  (void)b;
+  if (n_local_rows) *n_local_rows = h->n_local;
+  if (stride) *stride = h->feat_stride;
+  return WG_OK;
+}
+
+wg_status wg_dsm_shard_info(wg_dsm_t h, int32_t r, int64_t* n_local_rows, int64_t* local_num_edges) {
+  if (!h || r < 0 || r >= h->world) return fail(WG_ERR_INVALID_ARG, "bad handle or rank");
+  if (n_local_rows) *n_local_rows = h->n_local_of[r];
+  if (local_num_edges) *local_num_edges = h->e_local_of[r];
+  return WG_OK;
+}
+
+wg_status wg_dsm_destroy(wg_dsm_t h) {
+  if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
+  cudaSetDevice(h->device);
+  cudaDeviceSynchronize();
+  wg_status s1 = barrier(h);  // nobody reads a peer any more
+  for (int r = 0; r < h->world; ++r)
+    if (h->peer_opened[r]) {
+      cudaIpcCloseMemHandle(h->peer_base[r]);
+      h->peer_opened[r] = false;
+    }
+  wg_status s2 = barrier(h);  // nobody maps ours any more
+  release(h);
+  if (s1 != WG_OK) return s1;
+  return s2;
+}
+
+wg_status wg_sample_neighbors(wg_dsm_t h, const int64_t* d_targets, int64_t n_targets, const int64_t* d_n_targets,
+                              int32_t fanout, uint64_t seed, const uint64_t* d_seed, int32_t hop,
+                              int64_t* d_out_row_ptr, int64_t* d_out_nbrs, int32_t* d_out_pos,
+                              int64_t* d_out_num_edges, wg_stream_t stream) {
+  if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
+  if (fanout < 1) return fail(WG_ERR_INVALID_ARG, "fanout must be >= 1");
+  if (fanout > 32) return fail(WG_ERR_UNSUPPORTED, "fanout > 32 (warp path only)");
+  if (n_targets < 0 || (n_targets > 0 && !d_targets) || !d_out_row_ptr || (n_targets > 0 && !d_out_nbrs))
+    return fail(WG_ERR_INVALID_ARG, "null pointer or negative size");
+  if (hop < 0) return fail(WG_ERR_INVALID_ARG, "hop must be >= 0");
+  if (n_targets > h->ws.max_keys) return fail(WG_ERR_CAPACITY, "n_targets exceeds max_batch_keys");
+  if (n_targets * (int64_t)fanout >= (int64_t(1) << 40)) return fail(WG_ERR_INVALID_ARG, "too many edges");
+  cudaSetDevice(h->device);
+  cudaError_t e = launch_sample(h, d_targets, n_targets, d_n_targets, fanout, seed, d_seed, hop, d_out_row_ptr,
+                                d_out_nbrs, d_out_pos, d_out_num_edges, (cudaStream_t)stream);
+  if (e != cudaSuccess) return fail(WG_ERR_CUDA, std::string("sample launch: ") + cudaGetErrorString(e));
+  return WG_OK;
+}
+
+wg_status wg_append_unique(wg_dsm_t h, const int64_t* d_targets, int64_t n_targets, const int64_t* d_n_targets,
+                           const int64_t* d_nbrs, int64_t n_nbrs, const int64_t* d_n_nbrs, int64_t* d_out_unique,
+                           int64_t* d_out_num_unique, int32_t* d_out_sub_col, int32_t* d_out_dup_count,
+                           wg_stream_t stream) {
+  if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
+  if (n_targets < 0 || n_nbrs < 0) return fail(WG_ERR_INVALID_ARG, "negative size");
+  if ((n_targets > 0 && !d_targets) || (n_nbrs > 0 && (!d_nbrs || !d_out_sub_col)) ||
+      (n_targets + n_nbrs > 0 && !d_out_unique))
+    return fail(WG_ERR_INVALID_ARG, "null pointer");
+  if (n_targets + n_nbrs > h->ws.max_keys)
+    return fail(WG_ERR_CAPACITY, "n_targets + n_nbrs exceeds max_batch_keys");
+  cudaSetDevice(h->device);
+  cudaError_t e = launch_append_unique(h, d_targets, n_targets, d_n_targets, d_nbrs, n_nbrs, d_n_nbrs, d_out_unique,
+                                       d_out_num_unique, d_out_sub_col, d_out_dup_count, (cudaStream_t)stream);
+  if (e != cudaSuccess) return fail(WG_ERR_CUDA, std::string("append_unique launch: ") + cudaGetErrorString(e));
+  return WG_OK;
+}
+
+wg_status wg_gather(wg_dsm_t h, const int64_t* d_ids, int64_t n_ids, const int64_t* d_n_ids, void* d_out,
+                    wg_stream_t stream) {
+  if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
+  if (n_ids < 0 || (n_ids > 0 && (!d_ids || !d_out))) return fail(WG_ERR_INVALID_ARG, "null pointer or negative size");
+  if (h->row_bytes == 0) return fail(WG_ERR_INVALID_ARG, "DSM has no feature table");
+  if (h->row_bytes % 2 != 0) return fail(WG_ERR_UNSUPPORTED, "odd row size");
+  const int64_t vb = (h->row_bytes % 16 == 0) ? 16 : (h->row_bytes % 4 == 0) ? 4 : 2;
+  if (n_ids * (h->row_bytes / 2) >= (int64_t(1) << 31) || n_ids * (h->row_bytes / vb) >= (int64_t(1) << 31))
+    return fail(WG_ERR_UNSUPPORTED, "gather too large for one launch (split the id list)");
+  cudaSetDevice(h->device);
+  if (n_ids == 0 && !d_n_ids) return WG_OK;
+  cudaError_t e = launch_gather(h, d_ids, n_ids, d_n_ids, d_out, (cudaStream_t)stream);
+  if (e != cudaSuccess) return fail(WG_ERR_CUDA, std::string("gather launch: ") + cudaGetErrorString(e));
+  return WG_OK;
+}
+
+wg_status wg_device_error(wg_dsm_t h, uint32_t* code, int32_t clear) {
+  if (!h || !code) return fail(WG_ERR_INVALID_ARG, "null argument");
+  cudaSetDevice(h->device);
+  WG_CUDA_TRY(cudaDeviceSynchronize());
+  WG_CUDA_TRY(cudaMemcpy(code, h->ws.ctrl + CTRL_ERR, 4, cudaMemcpyDeviceToHost));
+  if (clear) WG_CUDA_TRY(cudaMemset(h->ws.ctrl + CTRL_ERR, 0, 4));
+  return WG_OK;
+}
+
+wg_status wg_dsm_reset_workspace(wg_dsm_t h, wg_stream_t stream) {
+  if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
+  cudaSetDevice(h->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  WG_CUDA_TRY(cudaMemsetAsync(h->ws.hkeys, 0, h->ws.hcap * 8, st));
+  WG_CUDA_TRY(cudaMemsetAsync(h->ws.hvals, 0xff, h->ws.hcap * 8, st));
+  static const unsigned one = 1;
+  WG_CUDA_TRY(cudaMemcpyAsync(h->ws.ctrl + CTRL_EPOCH, &one, 4, cudaMemcpyHostToDevice, st));
+  return WG_OK;
+}
+
+}  // extern "C"

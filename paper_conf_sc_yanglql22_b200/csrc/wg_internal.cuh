@@ -1,0 +1,95 @@
+// wg_internal.cuh -- internal definitions shared by the libwg.so translation units.
+// (Product code; shares nothing with oracle/.)
+#pragma once
+
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <string>
+
+#include "wg.h"
+
+namespace wg {
+
+// ------------------------------------------------------------------ errors
+void set_error(const std::string& msg);
+wg_status fail(wg_status s, const std::string& msg);
+#define WG_CUDA_TRY(expr)                                                                  \
+  do {                                                                                     \
+    cudaError_t e_ = (expr);                                                               \
+    if (e_ != cudaSuccess)                                                                 \
+      return ::wg::fail(WG_ERR_CUDA, std::string(#expr) + ": " + cudaGetErrorString(e_));  \
+  } while (0)
+
+// ------------------------------------------------------------------ shard view
+// The "memory pointer table": one base pointer per rank, passed
+// BY VALUE as a kernel parameter (constant bank; no global load per access).
+struct ShardView {
+  const int64_t* row_ptr[WG_MAX_WORLD];
+  const int64_t* col[WG_MAX_WORLD];
+  const uint8_t* feat[WG_MAX_WORLD];
+  int64_t n;            // num_nodes
+  int64_t feat_stride;  // bytes between feature rows in a shard (multiple of 16)
+  int32_t world;
+  int32_t log2w;        // log2(world) if world is a power of two, else -1
+};
+
+__device__ __forceinline__ void owner_local(const ShardView& s, int64_t v, int& o, int64_t& l) {
+  if (s.log2w >= 0) {
+    o = (int)(v & (int64_t)(s.world - 1));
+    l = v >> s.log2w;
+  } else {
+    o = (int)(v % s.world);
+    l = v / s.world;
+  }
+}
+
+// ------------------------------------------------------------------ workspace
+// Device-side scratch owned by the handle.  Everything that must be "fresh" per
+// call is either epoch-tagged (hash table) or reset by the last block of the
+// kernel that used it (scan status + done counters), so no memset is needed per
+// call and every op is CUDA-graph capturable.
+struct Workspace {
+  unsigned long long* hkeys = nullptr;   // [hcap] (epoch << 40) | node id
+  unsigned long long* hvals = nullptr;   // [hcap] ((EPOCH_MAX - epoch) << 40) | first position
+  int64_t hcap = 0;                      // power of two
+  unsigned long long* status_sample = nullptr;  // decoupled look-back tile status
+  unsigned long long* status_unique = nullptr;
+  int64_t status_cap = 0;
+  int32_t* excl = nullptr;               // [max_keys] exclusive scan of first-occurrence flags
+  unsigned* ctrl = nullptr;              // [16] control words (see CTRL_*)
+  int64_t max_keys = 0;
+};
+enum { CTRL_ERR = 0, CTRL_EPOCH = 1, CTRL_DONE_SAMPLE = 2, CTRL_DONE_UNIQUE = 3, CTRL_WORDS = 16 };
+constexpr unsigned EPOCH_MAX = (1u << 23) - 1;
+
+}  // namespace wg
+
+// ------------------------------------------------------------------ host handle
+struct wg_dsm {
+  int rank = 0, world = 1, device = 0;
+  int64_t n = 0, n_local = 0, e_local = 0, feat_dim = 0, elt = 4, row_bytes = 0, feat_stride = 0;
+  int64_t n_local_of[WG_MAX_WORLD] = {0};
+  int64_t e_local_of[WG_MAX_WORLD] = {0};
+  void* slab = nullptr;                 // this rank's allocation
+  size_t slab_bytes = 0;
+  void* peer_base[WG_MAX_WORLD] = {nullptr};
+  bool peer_opened[WG_MAX_WORLD] = {false};  // opened through cudaIpcOpenMemHandle
+  wg::ShardView view{};
+  wg::Workspace ws{};
+  wg_allgather_fn allgather = nullptr;
+  void* ctx = nullptr;
+  int sm_count = 148;
+};
+
+namespace wg {
+// launchers (stream-ordered); arguments already validated by the ABI layer
+cudaError_t launch_sample(wg_dsm* h, const int64_t* targets, int64_t cap, const int64_t* d_n, int fanout,
+                          uint64_t seed, const uint64_t* d_seed, int hop, int64_t* out_row_ptr,
+                          int64_t* out_nbrs, int32_t* out_pos, int64_t* d_num_edges, cudaStream_t st);
+cudaError_t launch_append_unique(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t* d_nT,
+                                 const int64_t* nbrs, int64_t capE, const int64_t* d_nE, int64_t* U,
+                                 int64_t* d_nU, int32_t* sub_col, int32_t* dup, cudaStream_t st);
+cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int64_t* d_n, void* out,
+                          cudaStream_t st);
+}  // namespace wg

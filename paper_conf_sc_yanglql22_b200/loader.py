@@ -1,0 +1,90 @@
+"""Setup helpers: build a DSM for one of the synthetic presets (not on the hot path).
+
+Small graphs are generated on the host (synth.graph) and copied in; large ones are
+generated per shard directly on the device (synth.gpu).  Either way the rows are
+identical (tests/test_gpu_synth.py).
+"""
+
+import time
+
+import numpy as np
+import torch
+
+from synth import features as sfeat
+from synth import graph as sgraph
+from synth import presets as spre
+
+from .dsm import DSM, local_num_edges
+from .pipeline import required_keys
+
+
+def build_dsm(preset, rank=0, world=1, device=None, allgather=None, max_seeds=None, on_device=None,
+              feat_dim=None, feat_dtype=None, extra_keys=0):
+    """Create and fill a DSM for ``preset`` (a synth.presets.Preset).  Returns (dsm, info)."""
+    device = torch.device("cuda", torch.cuda.current_device() if device is None else device)
+    spec = preset.graph()
+    fd = preset.feat_dim if feat_dim is None else feat_dim
+    fdt = preset.feat_dtype if feat_dtype is None else feat_dtype
+    S = preset.seeds_per_batch if max_seeds is None else max_seeds
+    keys = max(required_keys(spec.n, preset.fanouts, S), extra_keys, 1)
+    on_device = (spec.n > 200_000) if on_device is None else on_device
+    info = {}
+    t0 = time.perf_counter()
+    if on_device:
+        from synth import gpu as sgpu
+        rp, col = sgpu.shard_csr_gpu(spec, rank, world, device)
+        e_local = col.numel()
+    else:
+        g_rp, g_col = sgraph.csr(spec)
+        e_local = local_num_edges(g_rp, rank, world)
+    info["gen_s"] = time.perf_counter() - t0
+    t1 = time.perf_counter()
+    dsm = DSM(spec.n, e_local, fd, fdt, keys, rank=rank, world_size=world, device=device.index, allgather=allgather)
+    torch.cuda.synchronize(device)
+    info["create_s"] = time.perf_counter() - t1
+    if on_device:
+        lrp, lcol, lfeat = dsm.local_view()
+        lrp.copy_(rp)
+        if e_local:
+            lcol.copy_(col)
+        del rp, col
+        if fd:
+            from synth import gpu as sgpu
+            sgpu.fill_features_gpu(lfeat, spre.FEAT_SEED, rank, world, fd, sfeat.WG_DTYPE_CODE[fdt])
+    else:
+        dsm.fill_from_global_csr(g_rp, g_col)
+        if fd:
+            v = sgraph.shard_rows(spec.n, rank, world)
+            dsm.fill_features(sfeat.feature_bytes(spre.FEAT_SEED, v, fd, fdt))
+    torch.cuda.synchronize(device)
+    if allgather is not None and world > 1:
+        allgather(None, None, 0, None)  # barrier: every shard filled before anyone reads
+    info["e_local"] = e_local
+    info["fill_s"] = time.perf_counter() - t0 - info["gen_s"] - info["create_s"]
+    return dsm, info
+
+
+def host_row_provider(spec, row_ptr=None, col=None):
+    """Adjacency rows for the oracle: slices of a host CSR if given, else regenerated
+    per node from the generator (any n)."""
+    if row_ptr is not None:
+        def rows(T):
+            T = np.asarray(T, dtype=np.int64)
+            starts, ends = row_ptr[T], row_ptr[T + 1]
+            lens = ends - starts
+            ptr = np.zeros(len(T) + 1, dtype=np.int64)
+            ptr[1:] = np.cumsum(lens)
+            idx = np.repeat(starts - ptr[:-1], lens) + np.arange(ptr[-1], dtype=np.int64)
+            return ptr, col[idx]
+        return rows
+    return lambda T: sgraph.rows_native(spec, T)
+
+
+def host_feat_provider(preset, feat_dim=None, feat_dtype=None):
+    fd = preset.feat_dim if feat_dim is None else feat_dim
+    fdt = preset.feat_dtype if feat_dtype is None else feat_dtype
+
+    def feats(ids):
+        u = np.unique(np.asarray(ids, dtype=np.int64))
+        return u, sfeat.feature_bytes_native(spre.FEAT_SEED, u, fd, fdt)
+    return feats

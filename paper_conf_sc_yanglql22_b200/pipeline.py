@@ -1,0 +1,136 @@
+"""Multi-hop mini-batch preparation: "Multi-layer sub-graph sampling can be done by
+simply stacking multiple single-layer sub-graph sampling", then
+the global gather of the last frontier's features (L176).
+
+All buffers are preallocated from host upper bounds (T_{h+1} = U_h <= min(n,
+T_h (1 + M_h))) and every op reads the previous op's DEVICE count, so a whole batch
+is enqueued without a host sync and can be captured once as a CUDA graph and
+replayed with new seeds / rng_seed written into device buffers.
+"""
+
+import torch
+
+from .dsm import DSM
+
+
+def capacities(n, fanouts, max_seeds):
+    T, E, U = [], [], []
+    t = min(max_seeds, n)
+    for m in fanouts:
+        T.append(t)
+        E.append(t * m)
+        u = min(n, t + t * m)
+        U.append(u)
+        t = u
+    return T, E, U
+
+
+def required_keys(n, fanouts, max_seeds):
+    T, E, _ = capacities(n, fanouts, max_seeds)
+    return max(t + e for t, e in zip(T, E))
+
+
+class MiniBatchPipeline:
+    def __init__(self, dsm: DSM, fanouts, max_seeds, with_pos=False, with_dup=False):
+        self.dsm, self.fanouts, self.max_seeds = dsm, list(fanouts), max_seeds
+        self.with_pos, self.with_dup = with_pos, with_dup
+        dev = dsm.device
+        self.T_cap, self.E_cap, self.U_cap = capacities(dsm.num_nodes, fanouts, max_seeds)
+        if required_keys(dsm.num_nodes, fanouts, max_seeds) > dsm.max_batch_keys:
+            raise ValueError("DSM workspace too small for this pipeline (max_batch_keys)")
+        i64 = dict(dtype=torch.int64, device=dev)
+        i32 = dict(dtype=torch.int32, device=dev)
+        self.seeds = torch.zeros(max(self.max_seeds, 1), **i64)
+        self.n_seeds = torch.zeros(1, **i64)
+        self.rng_seed = torch.zeros(1, **i64)       # uint64 bit pattern
+        self.hops = []
+        for h, m in enumerate(self.fanouts):
+            T, E, U = self.T_cap[h], self.E_cap[h], self.U_cap[h]
+            self.hops.append(dict(
+                row_ptr=torch.zeros(T + 1, **i64), nbrs=torch.zeros(max(E, 1), **i64),
+                pos=torch.zeros(max(E, 1), **i32) if with_pos else None,
+                num_edges=torch.zeros(1, **i64), unique=torch.zeros(max(T + E, 1), **i64),
+                num_unique=torch.zeros(1, **i64), sub_col=torch.zeros(max(E, 1), **i32),
+                dup=torch.zeros(max(T + E, 1), **i32) if with_dup else None))
+        self.X = torch.zeros((max(self.U_cap[-1], 1), dsm.row_bytes), dtype=torch.uint8, device=dev) \
+            if dsm.row_bytes else None
+        self.graph = None
+
+    # -- enqueue one batch (reads seeds / n_seeds / rng_seed from device buffers)
+    def enqueue(self, stream=None, gather=True):
+        d = self.dsm
+        tgt, tcap, tn = self.seeds, self.max_seeds, self.n_seeds
+        for h, m in enumerate(self.fanouts):
+            b = self.hops[h]
+            d.sample_neighbors(tgt, m, 0, h, n_targets_dev=tn, seed_dev=self.rng_seed, out_row_ptr=b["row_ptr"],
+                               out_nbrs=b["nbrs"], out_pos=b["pos"], out_num_edges=b["num_edges"], cap=tcap,
+                               stream=stream)
+            d.append_unique(tgt, b["nbrs"], n_targets=tcap, n_nbrs=self.E_cap[h], n_targets_dev=tn,
+                            n_nbrs_dev=b["num_edges"], out_unique=b["unique"], out_num_unique=b["num_unique"],
+                            out_sub_col=b["sub_col"], out_dup=b["dup"], stream=stream)
+            tgt, tcap, tn = b["unique"], self.U_cap[h], b["num_unique"]
+        if gather and self.X is not None:
+            self.enqueue_gather(stream)
+
+    def enqueue_gather(self, stream=None):
+        last = self.hops[-1]
+        self.dsm.gather(last["unique"], n_ids=self.U_cap[-1], n_ids_dev=last["num_unique"], out=self.X, stream=stream)
+
+    def set_inputs(self, seeds: torch.Tensor, rng_seed: int, stream=None):
+        """Copy this batch's seed nodes (device or pinned host int64) and rng_seed
+        into the pipeline's device buffers (stream-ordered)."""
+        n = seeds.numel()
+        if n > self.max_seeds:
+            raise ValueError("too many seeds")
+        s = stream or torch.cuda.current_stream()
+        with torch.cuda.stream(s):
+            self.seeds[:n].copy_(seeds, non_blocking=True)
+            self.n_seeds.fill_(n)
+            self.rng_seed.fill_(to_i64(rng_seed))
+
+    def run(self, seeds, rng_seed, stream=None):
+        self.set_inputs(seeds, rng_seed, stream)
+        if self.graph is not None:
+            self.graph.replay()
+        else:
+            self.enqueue(stream)
+
+    def capture(self):
+        """Capture enqueue() as one CUDA graph (call after a warm-up run)."""
+        g = torch.cuda.CUDAGraph()
+        s = torch.cuda.Stream(device=self.dsm.device)
+        s.wait_stream(torch.cuda.current_stream())
+        with torch.cuda.graph(g, stream=s):
+            self.enqueue()
+        torch.cuda.current_stream().wait_stream(s)
+        self.graph = g
+        return g
+
+    # -- results (host sync)
+    def counts(self):
+        out = []
+        for b in self.hops:
+            out.append((int(b["num_edges"].item()), int(b["num_unique"].item())))
+        return out
+
+    def result(self, h):
+        """Host copies of hop h's outputs, trimmed to the device counts."""
+        b = self.hops[h]
+        nT = int(self.n_seeds.item()) if h == 0 else int(self.hops[h - 1]["num_unique"].item())
+        e, u = int(b["num_edges"].item()), int(b["num_unique"].item())
+        r = dict(row_ptr=b["row_ptr"][: nT + 1].cpu().numpy(), nbrs=b["nbrs"][:e].cpu().numpy(),
+                 unique=b["unique"][:u].cpu().numpy(), sub_col=b["sub_col"][:e].cpu().numpy())
+        if b["pos"] is not None:
+            r["pos"] = b["pos"][:e].cpu().numpy()
+        if b["dup"] is not None:
+            r["dup"] = b["dup"][:u].cpu().numpy()
+        return r
+
+    def features(self):
+        u = int(self.hops[-1]["num_unique"].item())
+        return self.X[:u].cpu().numpy()
+
+
+def to_i64(x: int) -> int:
+    x &= (1 << 64) - 1
+    return x - (1 << 64) if x >= (1 << 63) else x

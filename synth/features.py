@@ -38,3 +38,16 @@ def feature_bytes(feat_seed: int, v, dim: int, dtype: str) -> np.ndarray:
     """Row bytes [len(v), dim*elt] (uint8) of nodes v."""
     b = feature_bits(feat_seed, v, dim, dtype)
     return b.view(np.uint8).reshape(b.shape[0], -1)
+
+
+def feature_bytes_native(feat_seed: int, v, dim: int, dtype: str) -> np.ndarray:
+    """Same bytes as feature_bytes(), computed by the C++ host generator (fast)."""
+    import ctypes
+    from .graph import _native_lib
+    v = np.ascontiguousarray(np.asarray(v, dtype=np.int64).reshape(-1))
+    eb, _ = DTYPES[dtype]
+    out = np.zeros((len(v), dim * eb), dtype=np.uint8)
+    if len(v) and dim:
+        _native_lib().genh_features(feat_seed, v.ctypes.data_as(ctypes.c_void_p), len(v), dim,
+                                    WG_DTYPE_CODE[dtype], out.ctypes.data_as(ctypes.c_void_p))
+    return out

@@ -107,3 +107,47 @@ def shard_rows(n: int, rank: int, world: int) -> np.ndarray:
     """Global ids owned by ``rank`` under o(v) = v mod W, in local-row order l(v) = v div W
     (PAPER.md L110 hash partition)."""
     return np.arange(rank, n, world, dtype=np.int64)
+
+
+# ------------------------------------------------------------------ native host generator
+_native = None
+
+
+def _native_lib():
+    """synth/csrc/gen_host.cpp -> synth/libwggen_host.so (built on demand with g++)."""
+    global _native
+    if _native is None:
+        import ctypes
+        import os
+        import subprocess
+        here = os.path.dirname(os.path.abspath(__file__))
+        src = os.path.join(here, "csrc", "gen_host.cpp")
+        so = os.path.join(here, "libwggen_host.so")
+        if not os.path.exists(so) or os.path.getmtime(so) < os.path.getmtime(src):
+            tmp = so + f".tmp{os.getpid()}"
+            subprocess.check_call(["g++", "-O2", "-std=c++17", "-ffp-contract=off", "-shared", "-fPIC", src, "-o", tmp])
+            os.replace(tmp, so)
+        L = ctypes.CDLL(so)
+        P = ctypes.c_void_p
+        L.genh_rows.argtypes = [ctypes.c_int64, ctypes.c_double, ctypes.c_int64, ctypes.c_uint64, P, ctypes.c_int64,
+                                P, P]
+        L.genh_rows.restype = ctypes.c_int
+        L.genh_features.argtypes = [ctypes.c_uint64, P, ctypes.c_int64, ctypes.c_int64, ctypes.c_int, P]
+        L.genh_features.restype = ctypes.c_int
+        _native = L
+    return _native
+
+
+def rows_native(spec: GraphSpec, v):
+    """Same result as rows(), computed by the C++ host generator (fast)."""
+    import ctypes
+    L = _native_lib()
+    v = np.ascontiguousarray(np.asarray(v, dtype=np.int64).reshape(-1))
+    ptr = np.zeros(len(v) + 1, dtype=np.int64)
+    vp = v.ctypes.data_as(ctypes.c_void_p) if len(v) else None
+    L.genh_rows(spec.n, float(spec.d_min), spec.dmax, spec.graph_seed, vp, len(v),
+                ptr.ctypes.data_as(ctypes.c_void_p), None)
+    col = np.zeros(max(int(ptr[-1]), 1), dtype=np.int64)
+    L.genh_rows(spec.n, float(spec.d_min), spec.dmax, spec.graph_seed, vp, len(v),
+                ptr.ctypes.data_as(ctypes.c_void_p), col.ctypes.data_as(ctypes.c_void_p))
+    return ptr, col[: ptr[-1]]

@@ -1,0 +1,53 @@
+"""Shared helpers for the -m gpu parity tests: run the CUDA path through the C ABI
+(python binding) and the CPU oracle on the same seeded inputs."""
+
+import numpy as np
+import torch
+
+import oracle
+import paper_conf_sc_yanglql22_b200 as pkg
+from paper_conf_sc_yanglql22_b200 import loader
+
+
+def csr_from_rows(rows):
+    rp = np.zeros(len(rows) + 1, dtype=np.int64)
+    rp[1:] = np.cumsum([len(r) for r in rows])
+    col = np.concatenate([np.asarray(r, dtype=np.int64) for r in rows]) if rp[-1] else np.zeros(0, np.int64)
+    return rp, col
+
+
+def make_dsm(row_ptr, col, feat_rows=None, feat_dim=0, feat_dtype="fp32", max_keys=1 << 16, rank=0, world=1,
+             allgather=None):
+    n = len(row_ptr) - 1
+    dsm = pkg.DSM(n, pkg.local_num_edges(row_ptr, rank, world), feat_dim, feat_dtype, max_keys, rank=rank,
+                  world_size=world, allgather=allgather)
+    dsm.fill_from_global_csr(row_ptr, col)
+    if feat_dim:
+        dsm.fill_features(feat_rows[rank::world])
+    torch.cuda.synchronize()
+    if allgather is not None and world > 1:
+        allgather(None, None, 0, None)
+    return dsm
+
+
+def oracle_hop(row_ptr, col, T, M, seed, hop):
+    rows = loader.host_row_provider(None, row_ptr, col)
+    adj_ptr, adj = rows(np.asarray(T, dtype=np.int64))
+    return oracle.sample_hop(adj_ptr, adj, T, M, seed, hop)
+
+
+def gpu_hop(dsm, T, M, seed, hop):
+    t = torch.from_numpy(np.asarray(T, dtype=np.int64)).cuda()
+    rp, nb, pos, ne = dsm.sample_neighbors(t, M, seed, hop, with_pos=True)
+    torch.cuda.synchronize()
+    e = int(ne.item())
+    return rp.cpu().numpy(), nb[:e].cpu().numpy(), pos[:e].cpu().numpy()
+
+
+def gpu_unique(dsm, T, nbrs, with_dup=True):
+    t = torch.from_numpy(np.asarray(T, dtype=np.int64)).cuda()
+    nb = torch.from_numpy(np.asarray(nbrs, dtype=np.int64)).cuda()
+    U, nU, sc, dup = dsm.append_unique(t, nb, with_dup=with_dup)
+    torch.cuda.synchronize()
+    u = int(nU.item())
+    return U[:u].cpu().numpy(), sc[:len(nbrs)].cpu().numpy(), (dup[:u].cpu().numpy() if with_dup else None)

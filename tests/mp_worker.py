@@ -1,0 +1,63 @@
+"""Worker for the multi-process tests (one process per rank; env RANK/WORLD_SIZE/
+MASTER_ADDR/MASTER_PORT).  Mode "ipc": every rank drives cuda:0 (one-GPU box), the
+DSM handles are exchanged over gloo and opened with cudaIpcOpenMemHandle; mode
+"gloo-host": CPU-only check of the host-side collective plumbing."""
+
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
+import torch.distributed as dist  # noqa: E402
+
+
+def main():
+    mode = sys.argv[1]
+    dist.init_process_group("gloo", init_method="env://")
+    rank, world = dist.get_rank(), dist.get_world_size()
+    if mode == "gloo-host":
+        from paper_conf_sc_yanglql22_b200.dsm import TorchDistAllgather
+        ag = TorchDistAllgather()
+        import ctypes
+        send = (ctypes.c_uint8 * 16)(*([rank + 1] * 16))
+        recv = (ctypes.c_uint8 * (16 * world))()
+        assert ag(ctypes.addressof(send), ctypes.addressof(recv), 16, None) == 0
+        got = bytes(recv)
+        assert got == b"".join(bytes([r + 1] * 16) for r in range(world)), got
+        assert ag(None, None, 0, None) == 0     # barrier
+        print("GLOO OK", flush=True)
+    elif mode == "ipc":
+        import oracle
+        import paper_conf_sc_yanglql22_b200 as pkg
+        from paper_conf_sc_yanglql22_b200 import loader
+        from synth import graph, presets, seeds
+        torch.cuda.set_device(0)
+        p = presets.get("tiny")
+        ag = pkg.TorchDistAllgather()
+        dsm, _ = loader.build_dsm(p, rank=rank, world=world, allgather=ag, on_device=False)
+        rp, col = graph.csr(p.graph())
+        rows = loader.host_row_provider(p.graph(), rp, col)
+        feats = loader.host_feat_provider(p)
+        pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
+        for b in seeds.rank_batches(4, rank, world):
+            S = seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, b)
+            rs = seeds.rng_seed(presets.RNG_BASE, b)
+            pipe.run(torch.from_numpy(S).cuda(), rs)
+            torch.cuda.synchronize()
+            ref = oracle.minibatch(rows, feats, S, p.fanouts, rs)
+            for h in range(len(p.fanouts)):
+                got, exp = pipe.result(h), ref["hops"][h]
+                for k in ("row_ptr", "nbrs", "pos", "unique", "sub_col", "dup"):
+                    assert np.array_equal(got[k], exp[k]), (rank, b, h, k)
+            assert np.array_equal(pipe.features(), ref["X"])
+        assert dsm.device_error() == 0
+        dsm.destroy()
+        print("PARITY OK", flush=True)
+    dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,83 @@
+"""W > 1 on one GPU: in-process virtual ranks (threads, same pid -> direct pointers)
+and two processes sharing the GPU through real CUDA IPC handles.  Outputs must be
+byte-identical to the oracle (and hence W-invariant, SURVEY.md 8(c) "W-invariance")."""
+
+import os
+import subprocess
+import sys
+import threading
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_sc_yanglql22_b200 as pkg
+from paper_conf_sc_yanglql22_b200 import loader
+from synth import graph, presets, seeds
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def _create_all(p, W):
+    ag = pkg.ThreadAllgather(W)
+    out = [None] * W
+    errs = []
+
+    def run(r):
+        try:
+            out[r] = loader.build_dsm(p, rank=r, world=W, allgather=ag.for_rank(r), on_device=False)[0]
+        except Exception as e:  # pragma: no cover
+            errs.append(e)
+    ths = [threading.Thread(target=run, args=(r,)) for r in range(W)]
+    [t.start() for t in ths]
+    [t.join() for t in ths]
+    assert not errs, errs
+    return out
+
+
+def _destroy_all(dsms):
+    ths = [threading.Thread(target=d.destroy) for d in dsms]
+    [t.start() for t in ths]
+    [t.join() for t in ths]
+
+
+@pytest.mark.parametrize("W", [2, 3, 4, 8])
+def test_virtual_ranks_w_invariance(W):
+    p = presets.get("tiny")
+    rp, col = graph.csr(p.graph())
+    dsms = _create_all(p, W)
+    rows = loader.host_row_provider(p.graph(), rp, col)
+    feats = loader.host_feat_provider(p)
+    for r, dsm in enumerate(dsms):
+        assert dsm.shard_info(r)[0] == len(graph.shard_rows(p.n, r, W))
+        pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
+        for b in seeds.rank_batches(2 * W, r, W):
+            S = seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, b)
+            rs = seeds.rng_seed(presets.RNG_BASE, b)
+            pipe.run(torch.from_numpy(S).cuda(), rs)
+            torch.cuda.synchronize()
+            ref = oracle.minibatch(rows, feats, S, p.fanouts, rs)
+            for h in range(len(p.fanouts)):
+                got, exp = pipe.result(h), ref["hops"][h]
+                for k in ("row_ptr", "nbrs", "pos", "unique", "sub_col", "dup"):
+                    assert np.array_equal(got[k], exp[k]), (W, r, b, h, k)
+            assert np.array_equal(pipe.features(), ref["X"])
+        assert dsm.device_error() == 0
+    _destroy_all(dsms)
+
+
+def test_two_processes_cuda_ipc():
+    """torchrun-style 2 ranks (gloo for the handle allgather) on the SAME GPU: rank 1
+    reads rank 0's shard through cudaIpcOpenMemHandle and vice versa."""
+    env = dict(os.environ, MASTER_ADDR="127.0.0.1", MASTER_PORT=str(29500 + os.getpid() % 1000), WORLD_SIZE="2")
+    procs = []
+    for r in range(2):
+        e = dict(env, RANK=str(r), LOCAL_RANK=str(r))
+        procs.append(subprocess.Popen([sys.executable, os.path.join(ROOT, "tests", "mp_worker.py"), "ipc"],
+                                      env=e, stdout=subprocess.PIPE, stderr=subprocess.STDOUT))
+    outs = [p.communicate(timeout=600)[0].decode() for p in procs]
+    for p, o in zip(procs, outs):
+        assert p.returncode == 0, o
+        assert "PARITY OK" in o, o

@@ -1,0 +1,178 @@
+"""Parity of the CUDA path (through the C ABI) with the CPU oracle: bit-exact
+(tolerance 0) for sampled ids, positions, the sub-graph CSR, the unique/renumber
+maps, the duplicate counts and the gathered feature bytes (BASELINE.json
+north_star)."""
+
+import numpy as np
+import pytest
+import torch
+
+import oracle
+import paper_conf_sc_yanglql22_b200 as pkg
+from paper_conf_sc_yanglql22_b200 import loader
+from synth import features, graph, presets, seeds
+
+from gpu_helpers import csr_from_rows, gpu_hop, gpu_unique, make_dsm, oracle_hop
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def tiny():
+    p = presets.get("tiny")
+    rp, col = graph.csr(p.graph())
+    return p, rp, col
+
+
+def _check_batch(pipe, ref, fanouts):
+    for h in range(len(fanouts)):
+        got, exp = pipe.result(h), ref["hops"][h]
+        for k in ("row_ptr", "nbrs", "pos", "unique", "sub_col", "dup"):
+            assert np.array_equal(got[k], exp[k]), f"hop {h}: {k}"
+    assert np.array_equal(pipe.features(), ref["X"])
+
+
+def test_tiny_pipeline_many_batches(tiny):
+    """Config 1 (10k nodes, [10,5], 512 seeds): 20 batches, every array bit-exact."""
+    p, rp, col = tiny
+    dsm, _ = loader.build_dsm(p, on_device=False)
+    pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
+    rows = loader.host_row_provider(p.graph(), rp, col)
+    feats = loader.host_feat_provider(p)
+    for b in range(20):
+        S = seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, b)
+        rs = seeds.rng_seed(presets.RNG_BASE, b)
+        pipe.run(torch.from_numpy(S).cuda(), rs)
+        torch.cuda.synchronize()
+        ref = oracle.minibatch(rows, feats, S, p.fanouts, rs)
+        _check_batch(pipe, ref, p.fanouts)
+    assert dsm.device_error() == 0
+    dsm.destroy()
+
+
+def test_tiny_cuda_graph_replay(tiny):
+    """The captured batch graph replays with new seeds / rng_seed and stays bit-exact."""
+    p, rp, col = tiny
+    dsm, _ = loader.build_dsm(p, on_device=False)
+    pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
+    S0 = seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 0)
+    pipe.run(torch.from_numpy(S0).cuda(), 1)
+    torch.cuda.synchronize()
+    pipe.capture()
+    rows = loader.host_row_provider(p.graph(), rp, col)
+    feats = loader.host_feat_provider(p)
+    for b in (3, 4, 5):
+        n = 100 + 150 * (b - 3)      # fewer seeds than the capacity: device counts drive the graph
+        S = seeds.seed_nodes(p.n, n, presets.SEED_BASE, b)
+        rs = seeds.rng_seed(presets.RNG_BASE, b)
+        pipe.run(torch.from_numpy(S).cuda(), rs)
+        torch.cuda.synchronize()
+        _check_batch(pipe, oracle.minibatch(rows, feats, S, p.fanouts, rs), p.fanouts)
+    assert dsm.device_error() == 0
+    dsm.destroy()
+
+
+def _edge_graph():
+    """Degrees 0, 1, M-1, M, M+1 for several M, a 2^20 hub, and nodes whose rows
+    are all each other (so a hop can add no new node)."""
+    rng = np.random.default_rng(11)
+    n = 5000
+    rows = []
+    for v in range(n):
+        kind = v % 11
+        d = [0, 1, 4, 5, 6, 9, 10, 11, 31, 32, 33][kind]
+        rows.append(np.sort(rng.choice(n, size=d, replace=False)))
+    hub = 4999
+    rows[hub] = np.arange(1 << 20, dtype=np.int64) % n  # multi-edge hub row (positions are what is sampled)
+    rows[0], rows[1], rows[2] = np.array([1, 2]), np.array([0, 2]), np.array([0, 1])
+    return n, csr_from_rows(rows)
+
+
+@pytest.mark.parametrize("M", [1, 5, 8, 9, 16, 17, 25, 32])
+def test_sample_edge_cases(M):
+    n, (rp, col) = _edge_graph()
+    dsm = make_dsm(rp, col, max_keys=1 << 16)
+    T = np.concatenate([np.arange(0, 200), [4999, 4998, 4997, n - 1 - 11]]).astype(np.int64)
+    for hop, seed in ((0, 0x1234), (3, 0xFFFFFFFFFFFFFFFF)):
+        g = gpu_hop(dsm, T, M, seed, hop)
+        o = oracle_hop(rp, col, T, M, seed, hop)
+        for a, b in zip(g, o):
+            assert np.array_equal(a, b)
+    # single target, and empty target list
+    g = gpu_hop(dsm, np.array([4999]), M, 7, 1)
+    assert np.array_equal(g[1], oracle_hop(rp, col, np.array([4999]), M, 7, 1)[1])
+    rp0, nb0, _ = gpu_hop(dsm, np.zeros(0, np.int64), M, 7, 1)
+    assert list(rp0) == [0] and len(nb0) == 0
+    assert dsm.device_error() == 0
+    dsm.destroy()
+
+
+def test_sample_bad_ids_latch_error():
+    n, (rp, col) = _edge_graph()
+    dsm = make_dsm(rp, col)
+    rp_g, nb, _ = gpu_hop(dsm, np.array([5, -1, n + 3, 7]), 4, 1, 0)
+    assert dsm.device_error() & 0x1
+    assert rp_g[2] - rp_g[1] == 0 and rp_g[3] - rp_g[2] == 0   # invalid ids read as degree 0
+    dsm.destroy()
+
+
+def test_append_unique_random_vs_oracle():
+    n, (rp, col) = _edge_graph()
+    dsm = make_dsm(rp, col, max_keys=1 << 20)
+    rng = np.random.default_rng(5)
+    for trial in range(30):
+        pool = int(rng.integers(1, 4000))
+        nT = int(rng.integers(0, min(pool, 3000) + 1))
+        T = rng.choice(pool, size=nT, replace=False).astype(np.int64)
+        nE = int(rng.integers(0, 200_000))
+        # power-law-ish repeats (hubs) plus overlap with the targets
+        nbrs = np.minimum((rng.random(nE) ** 3 * pool).astype(np.int64), pool - 1)
+        U, sc, dup = gpu_unique(dsm, T, nbrs)
+        Uo, sco, dupo = oracle.append_unique(T, nbrs)
+        assert np.array_equal(U, Uo) and np.array_equal(sc, sco) and np.array_equal(dup, dupo)
+    assert dsm.device_error() == 0
+    # duplicate targets latch the error bit
+    gpu_unique(dsm, np.array([3, 4, 3]), np.array([1, 2]))
+    assert dsm.device_error() & 0x2
+    # all neighbours are targets; empty neighbour list
+    U, sc, _ = gpu_unique(dsm, np.array([40, 10, 30]), np.array([30, 40, 40]))
+    assert list(U) == [40, 10, 30] and list(sc) == [2, 0, 0]
+    U, sc, _ = gpu_unique(dsm, np.array([40, 10]), np.zeros(0, np.int64))
+    assert list(U) == [40, 10]
+    dsm.destroy()
+
+
+@pytest.mark.parametrize("dim,dtype", [(4, "fp32"), (32, "fp32"), (100, "fp32"), (1024, "fp32"), (768, "fp16"),
+                                       (3, "fp32"), (1, "fp16"), (7, "bf16")])
+def test_gather_rows(dim, dtype):
+    """Row sizes 16 B .. 4 KB and non-multiples of 16 B; repeated, sorted, reversed, empty id lists."""
+    n = 3000
+    rp = np.zeros(n + 1, dtype=np.int64)
+    feat = features.feature_bytes(presets.FEAT_SEED, np.arange(n), dim, dtype)
+    dsm = make_dsm(rp, np.zeros(0, np.int64), feat, dim, dtype)
+    rng = np.random.default_rng(dim)
+    for ids in (rng.integers(0, n, 5000), np.arange(n), np.arange(n)[::-1], np.full(77, n - 1), np.zeros(0)):
+        ids = np.asarray(ids, dtype=np.int64)
+        X = dsm.gather(torch.from_numpy(ids).cuda())
+        torch.cuda.synchronize()
+        exp = oracle.gather(feat, np.arange(n), ids)
+        assert np.array_equal(X[:len(ids)].cpu().numpy(), exp)
+    assert dsm.device_error() == 0
+    dsm.destroy()
+
+
+def test_determinism_two_runs(tiny):
+    p, rp, col = tiny
+    dsm, _ = loader.build_dsm(p, on_device=False)
+    pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
+    S = torch.from_numpy(seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 9)).cuda()
+    outs = []
+    for _ in range(2):
+        pipe.run(S, 99)
+        torch.cuda.synchronize()
+        outs.append([pipe.result(h) for h in range(2)] + [pipe.features()])
+    for a, b in zip(outs[0][:2], outs[1][:2]):
+        for k in a:
+            assert np.array_equal(a[k], b[k])
+    assert np.array_equal(outs[0][2], outs[1][2])
+    dsm.destroy()

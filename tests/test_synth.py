@@ -63,3 +63,19 @@ def test_seed_nodes_unique_and_rank_batches():
 def test_shard_rows():
     assert list(graph.shard_rows(10, 1, 4)) == [1, 5, 9]
     assert sum(len(graph.shard_rows(11, r, 3)) for r in range(3)) == 11
+
+
+def test_native_host_generator_matches_numpy():
+    for name in ("tiny", "products", "papers100m", "mag240m"):
+        spec = presets.get(name).graph()
+        rng = np.random.default_rng(1)
+        v = np.concatenate([[0, 1, spec.n - 1], rng.integers(0, spec.n, 300)]).astype(np.int64)
+        p1, c1 = graph.rows(spec, v)
+        p2, c2 = graph.rows_native(spec, v)
+        assert np.array_equal(p1, p2) and np.array_equal(c1, c2), name
+
+
+def test_native_features_match_numpy():
+    v = np.array([0, 5, 2**33 + 7, 123456789], dtype=np.int64)
+    for dtype, dim in (("fp32", 100), ("fp16", 768), ("bf16", 3)):
+        assert np.array_equal(features.feature_bytes(9, v, dim, dtype), features.feature_bytes_native(9, v, dim, dtype))
