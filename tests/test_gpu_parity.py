@@ -152,7 +152,7 @@ def test_gather_rows(dim, dtype):
     dsm = make_dsm(rp, np.zeros(0, np.int64), feat, dim, dtype)
     rng = np.random.default_rng(dim)
     for ids in (rng.integers(0, n, 5000), np.arange(n), np.arange(n)[::-1], np.full(77, n - 1), np.zeros(0)):
-        ids = np.asarray(ids, dtype=np.int64)
+        ids = np.ascontiguousarray(ids, dtype=np.int64)
         X = dsm.gather(torch.from_numpy(ids).cuda())
         torch.cuda.synchronize()
         exp = oracle.gather(feat, np.arange(n), ids)
