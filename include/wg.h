@@ -93,7 +93,7 @@ typedef struct {
 /* Create the DSM (section III-B).  COLLECTIVE over the W ranks.
  * Each rank allocates its shard slab on its device -- row_ptr int64[n_local+1],
  * col_idx int64[local_num_edges], features [n_local][row stride] with the row
- * stride rounded up to 16 bytes -- exports a CUDA IPC handle, allgathers the
+ * stride rounded up to 64 bytes (the DRAM access granule) -- exports a CUDA IPC handle, allgathers the
  * handles (L100), opens every peer's handle (L100-106; same-process peers are used
  * directly) and keeps the W base pointers as the "memory pointer table" (L106),
  * passed by value to every kernel.  n_local = number of v in [0,n) with v mod W == rank.
@@ -155,6 +155,25 @@ wg_status wg_append_unique(wg_dsm_t h, const int64_t* d_targets, int64_t n_targe
                            const int64_t* d_n_targets, const int64_t* d_nbrs, int64_t n_nbrs,
                            const int64_t* d_n_nbrs, int64_t* d_out_unique, int64_t* d_out_num_unique,
                            int32_t* d_out_sub_col, int32_t* d_out_dup_count, wg_stream_t stream);
+
+/* One whole hop of mini-batch preparation = wg_sample_neighbors followed by
+ * wg_append_unique on its output ("stacking multiple
+ * single-layer sub-graph sampling"), with identical results, fused for B200: the
+ * sampling kernel also performs the hash-table inserts of Append Unique (targets
+ * in its count phase, each neighbour right after its load), so a hop is one
+ * sampling kernel + one flag/scan kernel + one relabel kernel.  The relabel
+ * (which fills d_out_sub_col / d_out_dup_count) is launched on side_stream when
+ * it is non-NULL (forked from `stream` with an event); the caller must make its
+ * consumers wait for side_stream, and must join it before issuing a fifth
+ * append-unique on the handle (the workspace keeps a ring of 4 scan buffers).
+ * Arguments are those of the two calls; n_nbrs = n_targets * fanout and the
+ * neighbour count is d_out_num_edges (required here).  Requires
+ * n_targets * (1 + fanout) <= max_batch_keys. */
+wg_status wg_sample_hop(wg_dsm_t h, const int64_t* d_targets, int64_t n_targets, const int64_t* d_n_targets,
+                        int32_t fanout, uint64_t seed, const uint64_t* d_seed, int32_t hop, int64_t* d_out_row_ptr,
+                        int64_t* d_out_nbrs, int32_t* d_out_pos, int64_t* d_out_num_edges, int64_t* d_out_unique,
+                        int64_t* d_out_num_unique, int32_t* d_out_sub_col, int32_t* d_out_dup_count,
+                        wg_stream_t stream, wg_stream_t side_stream);
 
 /* Global gather: d_out[i][:] = the feature row of node
  * d_ids[i], in input order, read from the owner's shard (local HBM or a peer's

@@ -13,6 +13,7 @@
 #include <unistd.h>
 
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 
@@ -62,7 +63,8 @@ static void free_workspace(wg_dsm* h) {
   cudaFree(w.hvals);
   cudaFree(w.status_sample);
   cudaFree(w.status_unique);
-  cudaFree(w.excl);
+  for (int k = 0; k < EXCL_RING; ++k) cudaFree(w.excl[k]);
+  cudaFree(w.slot_of);
   cudaFree(w.ctrl);
   w = Workspace{};
 }
@@ -74,11 +76,13 @@ static wg_status alloc_workspace(wg_dsm* h, int64_t max_keys) {
   while (cap < 2 * max_keys) cap <<= 1;  // load factor <= 0.5
   w.hcap = cap;
   w.max_keys = max_keys;
-  w.status_cap = max_keys / 256 + 2;
+  w.status_cap = max_keys / 32 + 2;  // sampler tiles hold >= 32 targets, flag tiles 1024 positions
   if (cudaMalloc(&w.hkeys, cap * 8) != cudaSuccess || cudaMalloc(&w.hvals, cap * 8) != cudaSuccess ||
       cudaMalloc(&w.status_sample, w.status_cap * 8) != cudaSuccess ||
       cudaMalloc(&w.status_unique, w.status_cap * 8) != cudaSuccess ||
-      cudaMalloc(&w.excl, max_keys * 4) != cudaSuccess || cudaMalloc(&w.ctrl, CTRL_WORDS * 4) != cudaSuccess) {
+      cudaMalloc(&w.excl[0], max_keys * 4) != cudaSuccess || cudaMalloc(&w.excl[1], max_keys * 4) != cudaSuccess ||
+      cudaMalloc(&w.excl[2], max_keys * 4) != cudaSuccess || cudaMalloc(&w.excl[3], max_keys * 4) != cudaSuccess ||
+      cudaMalloc(&w.slot_of, max_keys * 4) != cudaSuccess || cudaMalloc(&w.ctrl, CTRL_WORDS * 4) != cudaSuccess) {
     cudaGetLastError();
     free_workspace(h);
     return fail(WG_ERR_OOM, "workspace allocation failed");
@@ -94,6 +98,7 @@ static wg_status alloc_workspace(wg_dsm* h, int64_t max_keys) {
 }
 
 static void release(wg_dsm* h) {
+  if (h->fork_event) cudaEventDestroy(h->fork_event);
   for (int r = 0; r < h->world; ++r)
     if (h->peer_opened[r]) cudaIpcCloseMemHandle(h->peer_base[r]);
   free_workspace(h);
@@ -137,10 +142,14 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
   h->feat_dim = d->feat_dim;
   h->elt = d->feat_dtype == WG_F32 ? 4 : 2;
   h->row_bytes = h->feat_dim * h->elt;
-  h->feat_stride = round_up(h->row_bytes, 16);
+  h->feat_stride = round_up(h->row_bytes, 64);  // 64 B = the DRAM access granule: no row straddles an extra one
   h->allgather = d->allgather;
   h->ctx = d->ctx;
   h->sm_count = sms;
+  {
+    const char* f = getenv("WG_FUSE_INSERT");  // A/B switch: 1 = hash inserts inside the sampler
+    h->fuse_insert = f && f[0] == '1';
+  }
   h->n_local = local_rows(h->n, h->rank, h->world);
   h->e_local = d->local_num_edges;
 
@@ -153,6 +162,12 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
     h->slab = nullptr;
     release(h);
     return fail(WG_ERR_OOM, "shard allocation of " + std::to_string(h->slab_bytes) + " bytes failed");
+  }
+  if (cudaEventCreateWithFlags(&h->fork_event, cudaEventDisableTiming) != cudaSuccess) {
+    cudaGetLastError();
+    h->fork_event = nullptr;
+    release(h);
+    return fail(WG_ERR_CUDA, "cudaEventCreate failed");
   }
   wg_status st = alloc_workspace(h, d->max_batch_keys);
   if (st != WG_OK) {
@@ -245,11 +260,9 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
 wg_status wg_dsm_local_view(wg_dsm_t h, int64_t** row_ptr, int64_t** col, void** feat, int64_t* n_local_rows,
                             int64_t* stride) {
   if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
-  uint8_t* b = static_cast<uint8_t*>(h->slab);
   if (row_ptr) *row_ptr = const_cast<int64_t*>(h->view.row_ptr[h->rank]);
   if (col) *col = const_cast<int64_t*>(h->view.col[h->rank]);
   if (feat) *feat = const_cast<uint8_t*>(h->view.feat[h->rank]);
-  (void)b;
   if (n_local_rows) *n_local_rows = h->n_local;
   if (stride) *stride = h->feat_stride;
   return WG_OK;
@@ -292,7 +305,7 @@ wg_status wg_sample_neighbors(wg_dsm_t h, const int64_t* d_targets, int64_t n_ta
   if (n_targets * (int64_t)fanout >= (int64_t(1) << 40)) return fail(WG_ERR_INVALID_ARG, "too many edges");
   cudaSetDevice(h->device);
   cudaError_t e = launch_sample(h, d_targets, n_targets, d_n_targets, fanout, seed, d_seed, hop, d_out_row_ptr,
-                                d_out_nbrs, d_out_pos, d_out_num_edges, (cudaStream_t)stream);
+                                d_out_nbrs, d_out_pos, d_out_num_edges, false, (cudaStream_t)stream);
   if (e != cudaSuccess) return fail(WG_ERR_CUDA, std::string("sample launch: ") + cudaGetErrorString(e));
   return WG_OK;
 }
@@ -310,7 +323,33 @@ wg_status wg_append_unique(wg_dsm_t h, const int64_t* d_targets, int64_t n_targe
     return fail(WG_ERR_CAPACITY, "n_targets + n_nbrs exceeds max_batch_keys");
   cudaSetDevice(h->device);
   cudaError_t e = launch_append_unique(h, d_targets, n_targets, d_n_targets, d_nbrs, n_nbrs, d_n_nbrs, d_out_unique,
-                                       d_out_num_unique, d_out_sub_col, d_out_dup_count, (cudaStream_t)stream);
+                                       d_out_num_unique, d_out_sub_col, d_out_dup_count, false, (cudaStream_t)stream,
+                                       nullptr);
+  if (e != cudaSuccess) return fail(WG_ERR_CUDA, std::string("append_unique launch: ") + cudaGetErrorString(e));
+  return WG_OK;
+}
+
+wg_status wg_sample_hop(wg_dsm_t h, const int64_t* d_targets, int64_t n_targets, const int64_t* d_n_targets,
+                        int32_t fanout, uint64_t seed, const uint64_t* d_seed, int32_t hop, int64_t* d_out_row_ptr,
+                        int64_t* d_out_nbrs, int32_t* d_out_pos, int64_t* d_out_num_edges, int64_t* d_out_unique,
+                        int64_t* d_out_num_unique, int32_t* d_out_sub_col, int32_t* d_out_dup_count,
+                        wg_stream_t stream, wg_stream_t side_stream) {
+  if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
+  if (fanout < 1) return fail(WG_ERR_INVALID_ARG, "fanout must be >= 1");
+  if (fanout > 32) return fail(WG_ERR_UNSUPPORTED, "fanout > 32 (warp path only)");
+  if (n_targets < 0 || hop < 0 || !d_out_row_ptr || !d_out_num_edges ||
+      (n_targets > 0 && (!d_targets || !d_out_nbrs || !d_out_unique || !d_out_sub_col)))
+    return fail(WG_ERR_INVALID_ARG, "null pointer or negative size");
+  const int64_t n_nbrs = n_targets * (int64_t)fanout;
+  if (n_targets + n_nbrs > h->ws.max_keys) return fail(WG_ERR_CAPACITY, "n_targets*(1+fanout) exceeds max_batch_keys");
+  cudaSetDevice(h->device);
+  cudaStream_t st = (cudaStream_t)stream;
+  cudaError_t e = launch_sample(h, d_targets, n_targets, d_n_targets, fanout, seed, d_seed, hop, d_out_row_ptr,
+                                d_out_nbrs, d_out_pos, d_out_num_edges, h->fuse_insert, st);
+  if (e != cudaSuccess) return fail(WG_ERR_CUDA, std::string("sample launch: ") + cudaGetErrorString(e));
+  e = launch_append_unique(h, d_targets, n_targets, d_n_targets, d_out_nbrs, n_nbrs, d_out_num_edges, d_out_unique,
+                           d_out_num_unique, d_out_sub_col, d_out_dup_count, h->fuse_insert, st,
+                           (cudaStream_t)side_stream);
   if (e != cudaSuccess) return fail(WG_ERR_CUDA, std::string("append_unique launch: ") + cudaGetErrorString(e));
   return WG_OK;
 }

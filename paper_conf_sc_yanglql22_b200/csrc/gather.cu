@@ -104,7 +104,20 @@ cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int6
   GatherArgs a{h->view, ids, cap, d_n, static_cast<uint8_t*>(out), h->ws.ctrl, FastDiv((unsigned)(rb / vb))};
   const int64_t total = cap * (rb / vb);
   int64_t blocks = (total + GATHER_THREADS * GATHER_UNROLL - 1) / (GATHER_THREADS * GATHER_UNROLL);
-  const int64_t max_blocks = (int64_t)h->sm_count * 8;
+  // one full wave: resident blocks per SM (from the occupancy calculator) x SMs
+  static int occ[3] = {0, 0, 0};
+  const int which = vb == 16 ? 0 : (vb == 4 ? 1 : 2);
+  if (!occ[which]) {
+    int nb = 0;
+    if (vb == 16)
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<uint4>, GATHER_THREADS, 0);
+    else if (vb == 4)
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<unsigned>, GATHER_THREADS, 0);
+    else
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<unsigned short>, GATHER_THREADS, 0);
+    occ[which] = nb > 0 ? nb : 4;
+  }
+  const int64_t max_blocks = (int64_t)h->sm_count * occ[which];
   blocks = blocks < 1 ? 1 : (blocks > max_blocks ? max_blocks : blocks);
   if (vb == 16)
     gather_kernel<uint4><<<(unsigned)blocks, GATHER_THREADS, 0, st>>>(a);

@@ -1,0 +1,66 @@
+// hash.cuh -- the append-unique hash table (PAPER.md: "The key of our GPU
+// hash table is nodeID"; Warpcore-style open addressing [33]).
+//
+// Slot s: hkeys[s] = (epoch << 40) | node id, hvals[s] = ((EPOCH_MAX - epoch) << 40) |
+// first position.  A key from an older epoch reads as an empty slot and an older
+// value always loses an atomicMin against the current epoch, so the table is never
+// cleared between calls.  Linear probing, fmix64 hash, load factor <= 0.5.
+#pragma once
+
+#include "device_util.cuh"
+#include "wg_internal.cuh"
+
+namespace wg {
+
+constexpr unsigned long long KEY_MASK = (1ull << 40) - 1;
+
+struct HashTable {
+  unsigned long long* keys;
+  unsigned long long* vals;
+  unsigned long long mask;  // capacity - 1
+};
+
+__device__ __forceinline__ unsigned long long stored_key(unsigned epoch, int64_t key) {
+  return ((unsigned long long)epoch << 40) | (unsigned long long)key;
+}
+
+__device__ __forceinline__ unsigned long long pack_pos(unsigned epoch, int64_t q) {
+  return ((unsigned long long)(EPOCH_MAX - epoch) << 40) | (unsigned long long)q;
+}
+
+// Returns the slot holding `stored` (claiming an empty one if needed), or -1 if full.
+__device__ __forceinline__ long long hash_insert(const HashTable& t, unsigned long long stored, unsigned epoch) {
+  unsigned long long slot = fmix64(stored & KEY_MASK) & t.mask;
+  for (unsigned long long probe = 0; probe <= t.mask; ++probe) {
+    unsigned long long cur = ld_volatile_u64(&t.keys[slot]);
+    for (;;) {
+      if (cur == stored) return (long long)slot;
+      if ((unsigned)(cur >> 40) == epoch) break;  // occupied by another key this epoch
+      const unsigned long long prev = atomicCAS(&t.keys[slot], cur, stored);
+      if (prev == cur || prev == stored) return (long long)slot;
+      cur = prev;
+    }
+    slot = (slot + 1) & t.mask;
+  }
+  return -1;
+}
+
+__device__ __forceinline__ long long hash_find(const HashTable& t, unsigned long long stored, unsigned epoch) {
+  unsigned long long slot = fmix64(stored & KEY_MASK) & t.mask;
+  for (unsigned long long probe = 0; probe <= t.mask; ++probe) {
+    const unsigned long long cur = t.keys[slot];
+    if (cur == stored) return (long long)slot;
+    if ((unsigned)(cur >> 40) != epoch) return -1;  // empty: not present
+    slot = (slot + 1) & t.mask;
+  }
+  return -1;
+}
+
+// Insert `key` at position q, recording the minimum position.  Returns the slot or -1.
+__device__ __forceinline__ long long hash_insert_min(const HashTable& t, int64_t key, int64_t q, unsigned epoch) {
+  const long long slot = hash_insert(t, stored_key(epoch, key), epoch);
+  if (slot >= 0) atomicMin(&t.vals[slot], pack_pos(epoch, q));
+  return slot;
+}
+
+}  // namespace wg

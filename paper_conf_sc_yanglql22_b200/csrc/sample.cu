@@ -1,6 +1,6 @@
 // sample.cu -- multi-GPU sampling op (Algorithm 1).
 //
-// One single-pass kernel per hop.  A block owns a tile of TILE targets:
+// One single-pass kernel per hop.  A block owns a tile of 32..128 targets (sample_tile):
 //   count phase   one thread per target loads the (row_ptr[l], row_ptr[l+1]) pair
 //                 from the owner's shard (local HBM or a peer over NVLink), computes
 //                 cnt = min(M, deg), block-scans it and resolves the tile's global
@@ -17,14 +17,24 @@
 //                 equals Algorithm 1 for every draw vector (it is the same
 //                 sequential Fisher-Yates function).
 //                 Lane i then loads col[start + res_i] (local or peer) and writes
-//                 it at out_nbrs[offset + i], in draw order (A5).
-#include "device_util.cuh"
-#include "wg_internal.cuh"
+//                 it at out_nbrs[offset + i], in draw order (A5).  Each warp works
+//                 on UNR rounds at once so UNR independent neighbour loads are in
+//                 flight per lane (the loads are latency-bound random 8 B reads).
+// FUSED = true additionally performs the insert pass of Append Unique (unique.cu)
+// in the same kernel: targets are inserted in the count phase (position k) and each
+// sampled neighbour right after its load (position nT + p), so a whole hop needs
+// only this kernel, the flag scan and the (off-critical-path) relabel.
+#include "hash.cuh"
 
 namespace wg {
 
 constexpr int SAMPLE_THREADS = 256;
-constexpr int SAMPLE_TILE = 256;  // targets per block (one per thread in the count phase)
+constexpr int SAMPLE_UNR = 4;  // rounds per warp, all in flight at once
+// targets per block: (SAMPLE_THREADS / G) targets per round x SAMPLE_UNR rounds, i.e. 128 / 64 / 32 for
+// G = 8 / 16 / 32.  Small tiles spread even a 1024-target hop over many SMs (the kernel is latency-bound)
+// and leave each lane exactly one round of SAMPLE_UNR independent neighbour loads.
+template <int G>
+constexpr int sample_tile() { return (SAMPLE_THREADS / G) * SAMPLE_UNR; }
 
 struct SampleArgs {
   ShardView s;
@@ -41,10 +51,13 @@ struct SampleArgs {
   int64_t* d_num_edges;
   unsigned long long* status;
   unsigned* ctrl;
+  HashTable ht;      // FUSED only
+  int32_t* slot_of;  // FUSED only: slot of every position [targets ; neighbours]
 };
 
-template <int G>
+template <int G, bool FUSED>
 __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs a) {
+  constexpr int SAMPLE_TILE = sample_tile<G>();
   __shared__ int64_t sm_v[SAMPLE_TILE];
   __shared__ int64_t sm_start[SAMPLE_TILE];
   __shared__ int64_t sm_off[SAMPLE_TILE];
@@ -63,6 +76,7 @@ __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs
       nT = nT < 0 ? 0 : a.cap;
     }
   }
+  const unsigned epoch = FUSED ? a.ctrl[CTRL_EPOCH] : 0u;
   const int64_t tile_start = (int64_t)blockIdx.x * SAMPLE_TILE;
 
   if (nT == 0) {
@@ -76,10 +90,11 @@ __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs
     const int64_t idx = tile_start + tid;
     unsigned deg = 0;
     int64_t v = -1, start = 0;
-    if (idx < nT) {
+    if (tid < SAMPLE_TILE && idx < nT) {
       v = a.targets[idx];
       if (v < 0 || v >= a.s.n) {
         latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_ID_RANGE);
+        if (FUSED) a.slot_of[idx] = -1;
       } else {
         int o;
         int64_t l;
@@ -91,6 +106,11 @@ __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs
           latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DEGREE);
         else
           deg = (unsigned)d;
+        if (FUSED) {
+          const long long slot = hash_insert_min(a.ht, v, idx, epoch);
+          if (slot < 0) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_CAPACITY);
+          a.slot_of[idx] = (int32_t)slot;
+        }
       }
     }
     const int cnt = (int)min((unsigned)M, deg);
@@ -102,12 +122,14 @@ __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs
     }
     __syncthreads();
     const int64_t off = (int64_t)sm_prefix + excl;
-    sm_v[tid] = v;
-    sm_start[tid] = start;
-    sm_deg[tid] = deg;
-    sm_off[tid] = off;
-    if (idx < nT) a.out_row_ptr[idx] = off;
-    if (idx == nT - 1) {
+    if (tid < SAMPLE_TILE) {
+      sm_v[tid] = v;
+      sm_start[tid] = start;
+      sm_deg[tid] = deg;
+      sm_off[tid] = off;
+    }
+    if (tid < SAMPLE_TILE && idx < nT) a.out_row_ptr[idx] = off;
+    if (tid < SAMPLE_TILE && idx == nT - 1) {
       a.out_row_ptr[nT] = off + cnt;
       if (a.d_num_edges) *a.d_num_edges = off + cnt;
     }
@@ -116,57 +138,90 @@ __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs
     // ---------------- sample phase
     const unsigned long long seed = a.d_seed ? *a.d_seed : a.seed;
     const uint2 key = make_uint2((unsigned)(seed & 0xffffffffu), (unsigned)(seed >> 32));
-    constexpr int TPW = 32 / G;           // targets per warp step
-    const int g = lane / G;               // target slot within the warp
-    const int i = lane % G;               // draw index
+    constexpr int TPW = 32 / G;                  // targets per warp per round
+    constexpr int TPR = SAMPLE_THREADS / G;      // targets per block per round
+    const int g = lane / G;                      // target slot within the warp
+    const int i = lane % G;                      // draw index
     const int tile_n = (int)min((int64_t)SAMPLE_TILE, nT - tile_start);
-    for (int base = warp * TPW; base < tile_n; base += (SAMPLE_THREADS / 32) * TPW) {
-      const int k = base + g;
-      const bool active = k < tile_n;
-      int64_t tv = 0, tstart = 0, toff = 0;
-      unsigned N = 0;
-      if (active) {
-        tv = sm_v[k];
-        tstart = sm_start[k];
-        N = sm_deg[k];
-        toff = sm_off[k];
-      }
-      const bool full = N <= (unsigned)M;
-      const bool draw = active && !full && i < M;
-      unsigned r = 0;
-      if (draw) {
-        const uint4 x = philox4x32_10(
-            make_uint4((unsigned)(i >> 2), (unsigned)a.hop, (unsigned)((uint64_t)tv & 0xffffffffu),
-                       (unsigned)((uint64_t)tv >> 32)),
-            key);
-        const unsigned xi = (i & 3) == 0 ? x.x : (i & 3) == 1 ? x.y : (i & 3) == 2 ? x.z : x.w;
-        r = __umulhi(xi, N - (unsigned)i);  // floor(x * (N-i) / 2^32), in [0, N-1-i]
-      }
-      const unsigned long long mkey =
-          draw ? (((unsigned long long)g << 32) | r) : (0xffffffff00000000ull | (unsigned)lane);
-      const unsigned same = __match_any_sync(FULL_MASK, mkey);
-      const unsigned below = same & ((1u << lane) - 1u);
-      const int prev = below ? 31 - __clz(below) : -1;  // previous draw with value r
-      const bool is_last = (same >> lane) == 1u;        // no later draw with value r
-      sm_chain[warp][lane] = (unsigned)i;
-      __syncwarp();
-      if (draw && is_last && r >= N - (unsigned)M) sm_chain[warp][g * G + (int)(N - 1u - r)] = (unsigned)i;
-      __syncwarp();
-      unsigned c = sm_chain[warp][lane];
-      for (int s = 1; s < M; s <<= 1) c = __shfl_sync(FULL_MASK, c, g * G + (int)c);
-      const unsigned last = N - c - 1u;
-      const unsigned lastp = __shfl_sync(FULL_MASK, last, prev >= 0 ? prev : lane);
-      const unsigned pos = full ? (unsigned)i : (prev < 0 ? r : lastp);
-      const bool valid = active && (full ? (unsigned)i < N : i < M);
-      if (valid) {
-        int o;
+    for (int r0 = 0; r0 < SAMPLE_UNR; r0 += SAMPLE_UNR) {  // one round-chunk per tile (see sample_tile)
+      if (r0 * TPR >= tile_n) break;  // block-uniform
+      const int64_t* src[SAMPLE_UNR];
+      int64_t dst[SAMPLE_UNR];
+      unsigned pos[SAMPLE_UNR];
+      bool ok[SAMPLE_UNR];
+#pragma unroll
+      for (int u = 0; u < SAMPLE_UNR; ++u) {
+        const int k = (r0 + u) * TPR + warp * TPW + g;
+        const bool active = k < tile_n;
+        int64_t tv = 0, tstart = 0, toff = 0;
+        unsigned N = 0;
+        if (active) {
+          tv = sm_v[k];
+          tstart = sm_start[k];
+          N = sm_deg[k];
+          toff = sm_off[k];
+        }
+        const bool full = N <= (unsigned)M;
+        const bool draw = active && !full && i < M;
+        unsigned r = 0;
+        if (draw) {
+          const uint4 x = philox4x32_10(
+              make_uint4((unsigned)(i >> 2), (unsigned)a.hop, (unsigned)((uint64_t)tv & 0xffffffffu),
+                         (unsigned)((uint64_t)tv >> 32)),
+              key);
+          const unsigned xi = (i & 3) == 0 ? x.x : (i & 3) == 1 ? x.y : (i & 3) == 2 ? x.z : x.w;
+          r = __umulhi(xi, N - (unsigned)i);  // floor(x * (N-i) / 2^32), in [0, N-1-i]
+        }
+        const unsigned long long mkey =
+            draw ? (((unsigned long long)g << 32) | r) : (0xffffffff00000000ull | (unsigned)lane);
+        const unsigned same = __match_any_sync(FULL_MASK, mkey);
+        const unsigned below = same & ((1u << lane) - 1u);
+        const int prev = below ? 31 - __clz(below) : -1;  // previous draw with value r
+        const bool is_last = (same >> lane) == 1u;        // no later draw with value r
+        sm_chain[warp][lane] = (unsigned)i;
+        __syncwarp();
+        if (draw && is_last && r >= N - (unsigned)M) sm_chain[warp][g * G + (int)(N - 1u - r)] = (unsigned)i;
+        __syncwarp();
+        unsigned c = sm_chain[warp][lane];
+        for (int s = 1; s < M; s <<= 1) c = __shfl_sync(FULL_MASK, c, g * G + (int)c);
+        const unsigned last = N - c - 1u;
+        const unsigned lastp = __shfl_sync(FULL_MASK, last, prev >= 0 ? prev : lane);
+        __syncwarp();
+        pos[u] = full ? (unsigned)i : (prev < 0 ? r : lastp);
+        ok[u] = active && (full ? (unsigned)i < N : i < M);
+        int o = 0;
         int64_t l;
-        owner_local(a.s, tv, o, l);
-        const int64_t nb = a.s.col[o][tstart + pos];
-        a.out_nbrs[toff + i] = nb;
-        if (a.out_pos) a.out_pos[toff + i] = (int32_t)pos;
+        if (ok[u]) owner_local(a.s, tv, o, l);
+        src[u] = a.s.col[o] + tstart + pos[u];
+        dst[u] = toff + i;
       }
-      __syncwarp();
+      int64_t nb[SAMPLE_UNR];
+#pragma unroll
+      for (int u = 0; u < SAMPLE_UNR; ++u) nb[u] = ok[u] ? *src[u] : -1;
+#pragma unroll
+      for (int u = 0; u < SAMPLE_UNR; ++u) {
+        if (ok[u]) {
+          a.out_nbrs[dst[u]] = nb[u];
+          if (a.out_pos) a.out_pos[dst[u]] = (int32_t)pos[u];
+        }
+      }
+      if (FUSED) {
+#pragma unroll
+        for (int u = 0; u < SAMPLE_UNR; ++u) {
+          const bool valid = ok[u] && nb[u] >= 0 && nb[u] < a.s.n;
+          if (ok[u] && !valid) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_ID_RANGE);
+          const unsigned long long mk = valid ? (unsigned long long)nb[u] : (0x8000000000000000ull | (unsigned)lane);
+          const unsigned same = __match_any_sync(FULL_MASK, mk);
+          const int leader = __ffs(same) - 1;  // lowest lane = smallest position among equal keys
+          long long slot = -1;
+          if (valid && leader == lane) {
+            slot = hash_insert_min(a.ht, nb[u], nT + dst[u], epoch);
+            if (slot < 0) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_CAPACITY);
+          }
+          slot = __shfl_sync(FULL_MASK, slot, leader);
+          if (ok[u]) a.slot_of[nT + dst[u]] = valid ? (int32_t)slot : -1;
+        }
+      }
     }
   }
 
@@ -177,9 +232,19 @@ __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs
   }
 }
 
+template <bool FUSED>
+static void launch_sample_t(const SampleArgs& a, int fanout, dim3 grid, cudaStream_t st) {
+  if (fanout <= 8)
+    sample_kernel<8, FUSED><<<grid, SAMPLE_THREADS, 0, st>>>(a);
+  else if (fanout <= 16)
+    sample_kernel<16, FUSED><<<grid, SAMPLE_THREADS, 0, st>>>(a);
+  else
+    sample_kernel<32, FUSED><<<grid, SAMPLE_THREADS, 0, st>>>(a);
+}
+
 cudaError_t launch_sample(wg_dsm* h, const int64_t* targets, int64_t cap, const int64_t* d_n, int fanout,
                           uint64_t seed, const uint64_t* d_seed, int hop, int64_t* out_row_ptr,
-                          int64_t* out_nbrs, int32_t* out_pos, int64_t* d_num_edges, cudaStream_t st) {
+                          int64_t* out_nbrs, int32_t* out_pos, int64_t* d_num_edges, bool fused, cudaStream_t st) {
   SampleArgs a;
   a.s = h->view;
   a.targets = targets;
@@ -195,14 +260,15 @@ cudaError_t launch_sample(wg_dsm* h, const int64_t* targets, int64_t cap, const 
   a.d_num_edges = d_num_edges;
   a.status = h->ws.status_sample;
   a.ctrl = h->ws.ctrl;
-  const int64_t tiles = cap > 0 ? (cap + SAMPLE_TILE - 1) / SAMPLE_TILE : 1;
-  dim3 grid((unsigned)tiles), block(SAMPLE_THREADS);
-  if (fanout <= 8)
-    sample_kernel<8><<<grid, block, 0, st>>>(a);
-  else if (fanout <= 16)
-    sample_kernel<16><<<grid, block, 0, st>>>(a);
+  a.ht = HashTable{h->ws.hkeys, h->ws.hvals, (unsigned long long)h->ws.hcap - 1};
+  a.slot_of = h->ws.slot_of;
+  const int tile = fanout <= 8 ? sample_tile<8>() : fanout <= 16 ? sample_tile<16>() : sample_tile<32>();
+  const int64_t tiles = cap > 0 ? (cap + tile - 1) / tile : 1;
+  dim3 grid((unsigned)tiles);
+  if (fused)
+    launch_sample_t<true>(a, fanout, grid, st);
   else
-    sample_kernel<32><<<grid, block, 0, st>>>(a);
+    launch_sample_t<false>(a, fanout, grid, st);
   return cudaGetLastError();
 }
 

@@ -1,31 +1,31 @@
 // unique.cu -- Append Unique op with first-appearance numbering (A7).
 //
-// Keys live in an open-addressing hash table (the paper's "GPU hash table ... key
-// is nodeID", L160-166; Warpcore-style insertion [33]) that stays in L2.  Instead
-// of the paper's per-bucket count of -1 values (whose order depends on the
+// Keys live in the open-addressing hash table of hash.cuh, which stays in L2.
+// Instead of the paper's per-bucket count of -1 values (whose order depends on the
 // insertion race), every key records the MINIMUM position at which it occurs in
 // the concatenated list [targets ; neighbours]; a neighbour position p is a "first
 // occurrence" iff that minimum equals nT + p, and the new ids are nT + exclusive
 // scan of the first-occurrence flags.  The result is deterministic and equals the
-// sequential definition.  Three kernels:
+// sequential definition.  Kernels:
 //   insert   all nT+nE keys; __match_any_sync elects one lane per distinct key in a
-//            warp; CAS claims a slot, atomicMin records the first position.
-//   flag     single-pass scan over neighbour positions (decoupled look-back): looks
-//            up the min position, writes U for first occurrences, the scan, and
-//            handles the targets (U[k] = T[k], duplicate-target check).  Its last
-//            block advances the table epoch.
-//   relabel  sub_col[p] = id of nbrs[p]; optional duplicate counts (L186).
-// The table is never cleared: keys carry an epoch tag (bits 40..62) and stale slots
-// read as empty, so no per-call memset is needed.
-#include "device_util.cuh"
-#include "wg_internal.cuh"
+//            warp; CAS claims a slot, atomicMin records the first position; every
+//            position remembers its slot (slot_of).  (Fused into the sampler by
+//            wg_sample_hop, sample.cu.)
+//   flag     single-pass scan over neighbour positions (decoupled look-back): reads
+//            the min position through slot_of (one dependent L2 read, no probing),
+//            writes U for first occurrences and the scan, and handles the targets
+//            (U[k] = T[k], duplicate-target check).  Its last block advances the
+//            table epoch.
+//   relabel  sub_col[p] = id of nbrs[p]; optional duplicate counts (L186).  Nothing
+//            downstream in the batch needs it before the end, so it may run on a
+//            side stream.
+#include "hash.cuh"
 
 namespace wg {
 
 constexpr int UQ_THREADS = 256;
 constexpr int UQ_ITEMS = 4;
 constexpr int UQ_TILE = UQ_THREADS * UQ_ITEMS;  // neighbour positions per flag tile
-constexpr unsigned long long KEY_MASK = (1ull << 40) - 1;
 
 struct UniqueArgs {
   const int64_t* T;
@@ -39,9 +39,8 @@ struct UniqueArgs {
   int32_t* sub_col;
   int32_t* dup;
   int32_t* excl;
-  unsigned long long* hkeys;
-  unsigned long long* hvals;
-  unsigned long long hmask;
+  int32_t* slot_of;
+  HashTable ht;
   unsigned long long* status;
   unsigned* ctrl;
   int64_t n;
@@ -66,39 +65,6 @@ __device__ __forceinline__ void load_counts(const UniqueArgs& a, int64_t& nT, in
   }
 }
 
-// Returns the slot holding `stored` (claiming an empty one if needed), or -1 if full.
-__device__ __forceinline__ long long hash_insert(const UniqueArgs& a, unsigned long long stored,
-                                                 unsigned epoch) {
-  unsigned long long slot = fmix64(stored & KEY_MASK) & a.hmask;
-  for (unsigned long long probe = 0; probe <= a.hmask; ++probe) {
-    unsigned long long cur = ld_volatile_u64(&a.hkeys[slot]);
-    for (;;) {
-      if (cur == stored) return (long long)slot;
-      if ((unsigned)(cur >> 40) == epoch) break;  // occupied by another key this epoch
-      const unsigned long long prev = atomicCAS(&a.hkeys[slot], cur, stored);
-      if (prev == cur || prev == stored) return (long long)slot;
-      cur = prev;
-    }
-    slot = (slot + 1) & a.hmask;
-  }
-  return -1;
-}
-
-__device__ __forceinline__ long long hash_find(const UniqueArgs& a, unsigned long long stored, unsigned epoch) {
-  unsigned long long slot = fmix64(stored & KEY_MASK) & a.hmask;
-  for (unsigned long long probe = 0; probe <= a.hmask; ++probe) {
-    const unsigned long long cur = a.hkeys[slot];
-    if (cur == stored) return (long long)slot;
-    if ((unsigned)(cur >> 40) != epoch) return -1;  // empty: not present
-    slot = (slot + 1) & a.hmask;
-  }
-  return -1;
-}
-
-__device__ __forceinline__ unsigned long long pack_pos(unsigned epoch, int64_t q) {
-  return ((unsigned long long)(EPOCH_MAX - epoch) << 40) | (unsigned long long)q;
-}
-
 __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueArgs a) {
   int64_t nT, nE;
   load_counts(a, nT, nE);
@@ -115,28 +81,26 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueA
       key = q < nT ? a.T[q] : a.nbrs[q - nT];
       if (key < 0 || key >= a.n) {
         latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_ID_RANGE);
+        a.slot_of[q] = -1;
         valid = false;
       }
     }
     const unsigned long long mk = valid ? (unsigned long long)key : (0x8000000000000000ull | (unsigned)lane);
     const unsigned same = __match_any_sync(FULL_MASK, mk);
-    // the lowest lane of each group of equal keys holds the smallest position
-    if (valid && (same & ((1u << lane) - 1u)) == 0u) {
-      const unsigned long long stored = ((unsigned long long)epoch << 40) | (unsigned long long)key;
-      const long long slot = hash_insert(a, stored, epoch);
-      if (slot < 0)
-        latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_CAPACITY);
-      else
-        atomicMin(&a.hvals[slot], pack_pos(epoch, q));
+    const int leader = __ffs(same) - 1;  // lowest lane = smallest position among equal keys
+    long long slot = -1;
+    if (valid && leader == lane) {
+      slot = hash_insert_min(a.ht, key, q, epoch);
+      if (slot < 0) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_CAPACITY);
     }
+    slot = __shfl_sync(FULL_MASK, slot, leader);
+    if (valid) a.slot_of[q] = (int32_t)slot;
   }
 }
 
-__device__ __forceinline__ int64_t min_pos_of(const UniqueArgs& a, int64_t key, unsigned epoch) {
-  const unsigned long long stored = ((unsigned long long)epoch << 40) | (unsigned long long)key;
-  const long long slot = hash_find(a, stored, epoch);
+__device__ __forceinline__ int64_t min_pos_at(const UniqueArgs& a, int32_t slot) {
   if (slot < 0) return -1;
-  return (int64_t)(a.hvals[slot] & KEY_MASK);
+  return (int64_t)(a.ht.vals[slot] & KEY_MASK);
 }
 
 __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArgs a) {
@@ -150,38 +114,40 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArg
 
   // targets: U[k] = T[k] (targets first, original order, L160); duplicate check (A8)
   for (int64_t k = (int64_t)blockIdx.x * UQ_THREADS + tid; k < nT; k += (int64_t)gridDim.x * UQ_THREADS) {
-    const int64_t key = a.T[k];
-    a.U[k] = key;
+    a.U[k] = a.T[k];
     if (a.dup) a.dup[k] = 0;
-    if (key >= 0 && key < a.n) {
-      const int64_t mp = min_pos_of(a, key, epoch);
-      if (mp != k) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DUP_TARGET);
-    }
+    const int32_t slot = a.slot_of[k];
+    if (slot >= 0 && min_pos_at(a, slot) != k) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DUP_TARGET);
   }
 
   const int64_t tile_start = (int64_t)blockIdx.x * UQ_TILE;
   if (nE == 0) {
     if (blockIdx.x == 0 && tid == 0 && a.d_nU) *a.d_nU = nT;
   } else if (tile_start < nE) {
-    int64_t keys[UQ_ITEMS];
-    int first[UQ_ITEMS];
+    int32_t slots[UQ_ITEMS];
+    int64_t mps[UQ_ITEMS];
+    const int64_t p0 = tile_start + (int64_t)tid * UQ_ITEMS;
+    // coalesced 16-byte read of this thread's 4 slots when aligned (p0 is a multiple of 4)
+    if (p0 + UQ_ITEMS <= nE && (nT & 3) == 0) {
+      const int4 s4 = *reinterpret_cast<const int4*>(a.slot_of + nT + p0);
+      slots[0] = s4.x; slots[1] = s4.y; slots[2] = s4.z; slots[3] = s4.w;
+    } else {
+#pragma unroll
+      for (int j = 0; j < UQ_ITEMS; ++j) slots[j] = (p0 + j < nE) ? a.slot_of[nT + p0 + j] : -1;
+    }
+#pragma unroll
+    for (int j = 0; j < UQ_ITEMS; ++j) mps[j] = min_pos_at(a, slots[j]);  // independent L2 reads
     int cnt = 0;
+    int first[UQ_ITEMS];
 #pragma unroll
     for (int j = 0; j < UQ_ITEMS; ++j) {
-      const int64_t p = tile_start + (int64_t)tid * UQ_ITEMS + j;
-      first[j] = 0;
-      keys[j] = -1;
+      const int64_t p = p0 + j;
+      first[j] = (p < nE) && (mps[j] == nT + p);
       if (p < nE) {
-        const int64_t key = a.nbrs[p];
-        keys[j] = key;
-        int64_t mp = -1;
-        if (key >= 0 && key < a.n) mp = min_pos_of(a, key, epoch);
-        if (mp < 0 && key >= 0 && key < a.n) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_CAPACITY);
-        first[j] = (mp == nT + p);
-        a.sub_col[p] = (int32_t)mp;  // temporary: min position (relabel turns it into an id)
+        a.sub_col[p] = (int32_t)mps[j];  // temporary: min position (relabel turns it into an id)
         if (a.dup) a.dup[nT + p] = 0;
-        cnt += first[j];
       }
+      cnt += first[j];
     }
     int agg;
     const int ex = block_exclusive_sum<UQ_THREADS>(cnt, sm_wtot, &agg);
@@ -193,10 +159,10 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArg
     int64_t run = (int64_t)sm_prefix + ex;
 #pragma unroll
     for (int j = 0; j < UQ_ITEMS; ++j) {
-      const int64_t p = tile_start + (int64_t)tid * UQ_ITEMS + j;
+      const int64_t p = p0 + j;
       if (p < nE) {
         a.excl[p] = (int32_t)run;
-        if (first[j]) a.U[nT + run] = keys[j];
+        if (first[j]) a.U[nT + run] = a.nbrs[p];
         run += first[j];
         if (p == nE - 1 && a.d_nU) *a.d_nU = nT + run;
       }
@@ -230,7 +196,8 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_relabel_kernel(const Unique
 
 cudaError_t launch_append_unique(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t* d_nT,
                                  const int64_t* nbrs, int64_t capE, const int64_t* d_nE, int64_t* U,
-                                 int64_t* d_nU, int32_t* sub_col, int32_t* dup, cudaStream_t st) {
+                                 int64_t* d_nU, int32_t* sub_col, int32_t* dup, bool inserted, cudaStream_t st,
+                                 cudaStream_t side) {
   UniqueArgs a;
   a.T = T;
   a.capT = capT;
@@ -242,24 +209,34 @@ cudaError_t launch_append_unique(wg_dsm* h, const int64_t* T, int64_t capT, cons
   a.d_nU = d_nU;
   a.sub_col = sub_col;
   a.dup = dup;
-  a.excl = h->ws.excl;
-  a.hkeys = h->ws.hkeys;
-  a.hvals = h->ws.hvals;
-  a.hmask = (unsigned long long)h->ws.hcap - 1;
+  a.excl = h->ws.excl[h->excl_next];
+  h->excl_next = (h->excl_next + 1) % EXCL_RING;
+  a.slot_of = h->ws.slot_of;
+  a.ht = HashTable{h->ws.hkeys, h->ws.hvals, (unsigned long long)h->ws.hcap - 1};
   a.status = h->ws.status_unique;
   a.ctrl = h->ws.ctrl;
   a.n = h->n;
   const int64_t total = capT + capE;
   const int64_t max_blocks = (int64_t)h->sm_count * 8;
-  int64_t ib = (total + UQ_THREADS - 1) / UQ_THREADS;
-  ib = ib < 1 ? 1 : (ib > max_blocks ? max_blocks : ib);
-  unique_insert_kernel<<<(unsigned)ib, UQ_THREADS, 0, st>>>(a);
+  if (!inserted) {
+    int64_t ib = (total + UQ_THREADS - 1) / UQ_THREADS;
+    ib = ib < 1 ? 1 : (ib > max_blocks ? max_blocks : ib);
+    unique_insert_kernel<<<(unsigned)ib, UQ_THREADS, 0, st>>>(a);
+  }
   int64_t fb = capE > 0 ? (capE + UQ_TILE - 1) / UQ_TILE : 1;
   unique_flag_kernel<<<(unsigned)fb, UQ_THREADS, 0, st>>>(a);
   if (capE > 0) {
     int64_t rb = (capE + UQ_THREADS - 1) / UQ_THREADS;
     rb = rb > max_blocks ? max_blocks : rb;
-    unique_relabel_kernel<<<(unsigned)rb, UQ_THREADS, 0, st>>>(a);
+    cudaStream_t rs = st;
+    if (side && side != st) {
+      cudaError_t e = cudaEventRecord(h->fork_event, st);
+      if (e != cudaSuccess) return e;
+      e = cudaStreamWaitEvent(side, h->fork_event, 0);
+      if (e != cudaSuccess) return e;
+      rs = side;
+    }
+    unique_relabel_kernel<<<(unsigned)rb, UQ_THREADS, 0, rs>>>(a);
   }
   return cudaGetLastError();
 }

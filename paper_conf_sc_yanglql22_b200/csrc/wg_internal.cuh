@@ -56,12 +56,16 @@ struct Workspace {
   unsigned long long* status_sample = nullptr;  // decoupled look-back tile status
   unsigned long long* status_unique = nullptr;
   int64_t status_cap = 0;
-  int32_t* excl = nullptr;               // [max_keys] exclusive scan of first-occurrence flags
+  int32_t* excl[4] = {nullptr, nullptr, nullptr, nullptr};  // ring of [max_keys] exclusive scans of
+                                         // first-occurrence flags (a relabel on a side stream may
+                                         // still read one while the next hops write the others)
+  int32_t* slot_of = nullptr;            // [max_keys] hash slot of every position of the current call
   unsigned* ctrl = nullptr;              // [16] control words (see CTRL_*)
   int64_t max_keys = 0;
 };
 enum { CTRL_ERR = 0, CTRL_EPOCH = 1, CTRL_DONE_SAMPLE = 2, CTRL_DONE_UNIQUE = 3, CTRL_WORDS = 16 };
 constexpr unsigned EPOCH_MAX = (1u << 23) - 1;
+constexpr int EXCL_RING = 4;
 
 }  // namespace wg
 
@@ -80,16 +84,20 @@ struct wg_dsm {
   wg_allgather_fn allgather = nullptr;
   void* ctx = nullptr;
   int sm_count = 148;
+  bool fuse_insert = false;             // wg_sample_hop: inserts inside the sampler (else a separate pass)
+  int excl_next = 0;                    // next excl ring slot (host-side, per call)
+  cudaEvent_t fork_event = nullptr;     // relabel fork onto a side stream
 };
 
 namespace wg {
 // launchers (stream-ordered); arguments already validated by the ABI layer
 cudaError_t launch_sample(wg_dsm* h, const int64_t* targets, int64_t cap, const int64_t* d_n, int fanout,
                           uint64_t seed, const uint64_t* d_seed, int hop, int64_t* out_row_ptr,
-                          int64_t* out_nbrs, int32_t* out_pos, int64_t* d_num_edges, cudaStream_t st);
+                          int64_t* out_nbrs, int32_t* out_pos, int64_t* d_num_edges, bool fused, cudaStream_t st);
 cudaError_t launch_append_unique(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t* d_nT,
                                  const int64_t* nbrs, int64_t capE, const int64_t* d_nE, int64_t* U,
-                                 int64_t* d_nU, int32_t* sub_col, int32_t* dup, cudaStream_t st);
+                                 int64_t* d_nU, int32_t* sub_col, int32_t* dup, bool inserted, cudaStream_t st,
+                                 cudaStream_t side);
 cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int64_t* d_n, void* out,
                           cudaStream_t st);
 }  // namespace wg

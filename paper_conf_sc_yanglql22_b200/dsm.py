@@ -194,6 +194,33 @@ class DSM:
                                      _ptr(out_dup), _stream(stream)))
         return out_unique, out_num_unique, out_sub_col, out_dup
 
+    def sample_hop(self, targets, fanout, seed, hop, n_targets_dev=None, seed_dev=None, out=None, cap=None,
+                   with_pos=False, with_dup=False, stream=None, side_stream=None):
+        """One fused hop = sample_neighbors + append_unique (same results; wg_sample_hop).
+        ``out`` = dict of preallocated buffers (row_ptr, nbrs, pos, num_edges, unique,
+        num_unique, sub_col, dup).  If ``side_stream`` is given the relabel runs there
+        and the caller must wait for it before reading sub_col / dup."""
+        cap = targets.numel() if cap is None else cap
+        dev = self.device
+        E = max(cap * fanout, 1)
+        o = dict(out or {})
+        i64 = dict(dtype=torch.int64, device=dev)
+        i32 = dict(dtype=torch.int32, device=dev)
+        o.setdefault("row_ptr", torch.empty(cap + 1, **i64))
+        o.setdefault("nbrs", torch.empty(E, **i64))
+        o.setdefault("pos", torch.empty(E, **i32) if with_pos else None)
+        o.setdefault("num_edges", torch.empty(1, **i64))
+        o.setdefault("unique", torch.empty(max(cap + cap * fanout, 1), **i64))
+        o.setdefault("num_unique", torch.empty(1, **i64))
+        o.setdefault("sub_col", torch.empty(E, **i32))
+        o.setdefault("dup", torch.empty(max(cap + cap * fanout, 1), **i32) if with_dup else None)
+        check(lib().wg_sample_hop(self.h, _ptr(targets), cap, _ptr(n_targets_dev), fanout,
+                                  ctypes.c_uint64(seed & ((1 << 64) - 1)), _ptr(seed_dev), hop, _ptr(o["row_ptr"]),
+                                  _ptr(o["nbrs"]), _ptr(o["pos"]), _ptr(o["num_edges"]), _ptr(o["unique"]),
+                                  _ptr(o["num_unique"]), _ptr(o["sub_col"]), _ptr(o["dup"]), _stream(stream),
+                                  _stream(side_stream) if side_stream is not None else None))
+        return o
+
     def gather(self, ids, n_ids=None, n_ids_dev=None, out=None, stream=None):
         """Global gather: out[i] = feature row of ids[i] (uint8 rows)."""
         n = ids.numel() if n_ids is None else n_ids

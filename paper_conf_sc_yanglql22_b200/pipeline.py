@@ -31,8 +31,10 @@ def required_keys(n, fanouts, max_seeds):
 
 
 class MiniBatchPipeline:
-    def __init__(self, dsm: DSM, fanouts, max_seeds, with_pos=False, with_dup=False):
+    def __init__(self, dsm: DSM, fanouts, max_seeds, with_pos=False, with_dup=False, fused=True):
         self.dsm, self.fanouts, self.max_seeds = dsm, list(fanouts), max_seeds
+        self.fused = fused
+        self.side = torch.cuda.Stream(device=dsm.device) if fused else None
         self.with_pos, self.with_dup = with_pos, with_dup
         dev = dsm.device
         self.T_cap, self.E_cap, self.U_cap = capacities(dsm.num_nodes, fanouts, max_seeds)
@@ -58,19 +60,31 @@ class MiniBatchPipeline:
 
     # -- enqueue one batch (reads seeds / n_seeds / rng_seed from device buffers)
     def enqueue(self, stream=None, gather=True):
+        """Enqueue every hop (fused wg_sample_hop: sample + append-unique; the
+        relabel of each hop runs on a side stream, joined at the end) and, unless
+        gather=False, the feature gather."""
         d = self.dsm
+        main = stream or torch.cuda.current_stream(d.device)
+        if self.fused:
+            self.side.wait_stream(main)
         tgt, tcap, tn = self.seeds, self.max_seeds, self.n_seeds
         for h, m in enumerate(self.fanouts):
             b = self.hops[h]
-            d.sample_neighbors(tgt, m, 0, h, n_targets_dev=tn, seed_dev=self.rng_seed, out_row_ptr=b["row_ptr"],
-                               out_nbrs=b["nbrs"], out_pos=b["pos"], out_num_edges=b["num_edges"], cap=tcap,
-                               stream=stream)
-            d.append_unique(tgt, b["nbrs"], n_targets=tcap, n_nbrs=self.E_cap[h], n_targets_dev=tn,
-                            n_nbrs_dev=b["num_edges"], out_unique=b["unique"], out_num_unique=b["num_unique"],
-                            out_sub_col=b["sub_col"], out_dup=b["dup"], stream=stream)
+            if self.fused:
+                d.sample_hop(tgt, m, 0, h, n_targets_dev=tn, seed_dev=self.rng_seed, out=b, cap=tcap, stream=main,
+                             side_stream=self.side)
+            else:
+                d.sample_neighbors(tgt, m, 0, h, n_targets_dev=tn, seed_dev=self.rng_seed, out_row_ptr=b["row_ptr"],
+                                   out_nbrs=b["nbrs"], out_pos=b["pos"], out_num_edges=b["num_edges"], cap=tcap,
+                                   stream=main)
+                d.append_unique(tgt, b["nbrs"], n_targets=tcap, n_nbrs=self.E_cap[h], n_targets_dev=tn,
+                                n_nbrs_dev=b["num_edges"], out_unique=b["unique"], out_num_unique=b["num_unique"],
+                                out_sub_col=b["sub_col"], out_dup=b["dup"], stream=main)
             tgt, tcap, tn = b["unique"], self.U_cap[h], b["num_unique"]
         if gather and self.X is not None:
-            self.enqueue_gather(stream)
+            self.enqueue_gather(main)
+        if self.fused:
+            main.wait_stream(self.side)
 
     def enqueue_gather(self, stream=None):
         last = self.hops[-1]
