@@ -38,6 +38,7 @@ def parse():
     ap.add_argument("--no-graph", action="store_true", help="launch ops eagerly instead of graph replay")
     ap.add_argument("--cpu-sample-s", type=float, default=12.0, help="target seconds of oracle work (cpu_baseline)")
     ap.add_argument("--e2e-steps", type=int, default=20)
+    ap.add_argument("--concurrency", type=int, default=4, help="independent batches in flight per GPU (streams)")
     ap.add_argument("--out", default=None, help="also append the JSON line to this file")
     return ap.parse_args()
 
@@ -194,44 +195,75 @@ def bench_wg(args):
         ag = pkg.TorchDistAllgather(device=dev)
     p = presets.get(args.config)
     S = p.seeds_per_batch
+    P = max(1, args.concurrency)
     t0 = time.perf_counter()
     dsm, info = loader.build_dsm(p, rank=rank, world=world, device=local, allgather=ag)
     setup_s = time.perf_counter() - t0
-    pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, S)
-    nsteps = args.warmup + args.steps
-    my_batches = [k * world + rank for k in range(nsteps)]
+    # P independent batch pipelines on P streams; pipeline j > 0 runs on a workspace fork of the DSM
+    handles = [dsm] + [dsm.fork() for _ in range(P - 1)]
+    pipes = [pkg.MiniBatchPipeline(h, p.fanouts, S) for h in handles]
+    streams = [torch.cuda.Stream(device=dev) for _ in range(P)]
+    n_single = args.warmup + args.steps
+    n_conc = args.warmup + args.steps * P
+    my_batches = [k * world + rank for k in range(n_single + n_conc)]
     seeds_dev = [torch.from_numpy(seeds.seed_nodes(p.n, S, presets.SEED_BASE, b)).to(dev) for b in my_batches]
     rngs = [seeds.rng_seed(presets.RNG_BASE, b) for b in my_batches]
     flush = None if args.no_flush else torch.empty(512 << 20, dtype=torch.uint8, device=dev)
 
-    # warm-up (eager), then capture prep and gather as two graphs
+    # warm-up (eager), then capture each pipeline as two graphs (prep, gather) on its stream
     for k in range(args.warmup):
-        pipe.run(seeds_dev[k], rngs[k])
+        for pl in pipes:
+            pl.run(seeds_dev[k], rngs[k])
     torch.cuda.synchronize()
-    g_prep = g_gather = None
-    if not args.no_graph:
-        s = torch.cuda.Stream(device=dev)
-        s.wait_stream(torch.cuda.current_stream())
-        g_prep, g_gather = torch.cuda.CUDAGraph(), torch.cuda.CUDAGraph()
-        with torch.cuda.graph(g_prep, stream=s):
-            pipe.enqueue(gather=False)
-        with torch.cuda.graph(g_gather, stream=s):
-            pipe.enqueue_gather()
-        torch.cuda.current_stream().wait_stream(s)
-        torch.cuda.synchronize()
-        for k in range(args.warmup):     # warm the graphs too
-            pipe.set_inputs(seeds_dev[k], rngs[k])
-            g_prep.replay()
-            g_gather.replay()
-        torch.cuda.synchronize()
-    err = dsm.device_error()
-    assert err == 0, f"device error {err:#x} during warm-up"
+    graphs = []
+    for pl, st in zip(pipes, streams):
+        if args.no_graph:
+            graphs.append((None, None))
+            continue
+        st.wait_stream(torch.cuda.current_stream())
+        gp, gg = torch.cuda.CUDAGraph(), torch.cuda.CUDAGraph()
+        with torch.cuda.graph(gp, stream=st):
+            pl.enqueue(gather=False)
+        with torch.cuda.graph(gg, stream=st):
+            pl.enqueue_gather()
+        graphs.append((gp, gg))
+    torch.cuda.synchronize()
 
-    stream = torch.cuda.current_stream()
-    ev = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
+    def launch(j, k, st):
+        """batch k on pipeline j, stream st (inputs already resident in HBM)."""
+        pl, (gp, gg) = pipes[j], graphs[j]
+        with torch.cuda.stream(st):
+            pl.set_inputs(seeds_dev[k], rngs[k])
+            if gp is not None:
+                gp.replay()
+            else:
+                pl.enqueue(gather=False)
+        return pl, gg
+
+    def gather(j, st):
+        pl, (gp, gg) = pipes[j], graphs[j]
+        with torch.cuda.stream(st):
+            if gg is not None:
+                gg.replay()
+            else:
+                pl.enqueue_gather()
+
+    for k in range(args.warmup):     # warm the graphs
+        for j in range(P):
+            launch(j, k, streams[j])
+            gather(j, streams[j])
+    torch.cuda.synchronize()
+    for h in handles:
+        err = h.device_error()
+        assert err == 0, f"device error {err:#x} during warm-up"
+
+    main = torch.cuda.current_stream()
+    clocks = ClockSampler(local)
+
+    # ---- pass A: one batch at a time (single-batch latency + the gather roofline)
+    evA = [[torch.cuda.Event(enable_timing=True) for _ in range(3)] for _ in range(args.steps)]
     rows_gathered = torch.zeros(args.steps, dtype=torch.int64, device=dev)
     hop_counts = torch.zeros((args.steps, len(p.fanouts), 2), dtype=torch.int64, device=dev)
-    clocks = ClockSampler(local)
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
@@ -241,37 +273,52 @@ def bench_wg(args):
         k = args.warmup + i
         if flush is not None:
             flush.fill_(i & 0xFF)
-        ev[i][0].record(stream)
-        pipe.set_inputs(seeds_dev[k], rngs[k])
-        if g_prep is not None:
-            g_prep.replay()
-        else:
-            pipe.enqueue(gather=False)
-        ev[i][1].record(stream)
-        if g_gather is not None:
-            g_gather.replay()
-        else:
-            pipe.enqueue_gather()
-        ev[i][2].record(stream)
-        rows_gathered[i:i + 1].copy_(pipe.hops[-1]["num_unique"])
-        for h, b in enumerate(pipe.hops):
+        evA[i][0].record(main)
+        pl, _ = launch(0, k, main)
+        evA[i][1].record(main)
+        gather(0, main)
+        evA[i][2].record(main)
+        rows_gathered[i:i + 1].copy_(pl.hops[-1]["num_unique"])
+        for h, b in enumerate(pl.hops):
             hop_counts[i, h, 0:1].copy_(b["num_edges"])
             hop_counts[i, h, 1:2].copy_(b["num_unique"])
+    torch.cuda.synchronize()
+    step_ms = [evA[i][0].elapsed_time(evA[i][2]) for i in range(args.steps)]
+    gather_ms = [evA[i][1].elapsed_time(evA[i][2]) for i in range(args.steps)]
+
+    # ---- pass B: P independent batches in flight on P streams (the throughput number)
+    evB = [[torch.cuda.Event(enable_timing=True) for _ in range(2)] for _ in range(args.steps)]
+    for i in range(args.steps):
+        if flush is not None:
+            flush.fill_(i & 0xFF)
+        evB[i][0].record(main)
+        for j in range(P):
+            streams[j].wait_stream(main)
+            launch(j, n_single + args.warmup + i * P + j, streams[j])
+            gather(j, streams[j])
+        for j in range(P):
+            main.wait_stream(streams[j])
+        evB[i][1].record(main)
     torch.cuda.synchronize()
     if world > 1:
         dist.barrier()
     wall = time.perf_counter() - wall0
     clk = clocks.stop()
-    step_ms = [ev[i][0].elapsed_time(ev[i][2]) for i in range(args.steps)]
-    gather_ms = [ev[i][1].elapsed_time(ev[i][2]) for i in range(args.steps)]
-    dev_s = sum(step_ms) / 1e3
-    err = dsm.device_error()
-    assert err == 0, f"device error {err:#x} in the timed region"
-    if world > 1:
-        t = torch.tensor([dev_s], dtype=torch.float64, device=dev)
+    conc_ms = [evB[i][0].elapsed_time(evB[i][1]) for i in range(args.steps)]
+    for h in handles:
+        err = h.device_error()
+        assert err == 0, f"device error {err:#x} in the timed region"
+
+    def max_over_ranks(x):
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64, device=dev)
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        dev_s = float(t.item())
-    value = world * S * args.steps / dev_s
+        return float(t.item())
+    dev_s_single = max_over_ranks(sum(step_ms) / 1e3)
+    dev_s_conc = max_over_ranks(sum(conc_ms) / 1e3)
+    value_single = world * S * args.steps / dev_s_single
+    value_conc = world * S * P * args.steps / dev_s_conc
     rb = dsm.row_bytes
     rows = rows_gathered.cpu().numpy()
     hc = hop_counts.cpu().numpy()
@@ -279,37 +326,33 @@ def bench_wg(args):
     alg_bytes = float(2 * rows.sum() * rb)           # read + write per gathered row (W=1: all local HBM)
     peak, peak_src = peaks()
     achieved = alg_bytes / gather_s / 1e9
+    bound = "hbm"
     if world > 1:
         remote = (world - 1) / world
         bound = "nvlink" if remote * rows.mean() * rb / 770e9 > 2 * rows.mean() * rb / (peak * 1e9) else "hbm"
-    else:
-        bound = "hbm"
 
     # ---- e2e through the public API with pinned host buffers (H2D seeds, D2H counts)
     e2e_times = []
     d2h = torch.empty((len(p.fanouts), 2), dtype=torch.int64, pin_memory=True)
-    host_seeds = [seeds_dev[k % nsteps].cpu().pin_memory() for k in range(args.e2e_steps)]
+    host_seeds = [seeds_dev[k % n_single].cpu().pin_memory() for k in range(args.e2e_steps)]
+    pl0, (gp0, gg0) = pipes[0], graphs[0]
     for i in range(args.e2e_steps + 2):
         hs = host_seeds[i % len(host_seeds)]
         torch.cuda.synchronize()
         t = time.perf_counter()
-        pipe.set_inputs(hs, rngs[i % nsteps])
-        if g_prep is not None:
-            g_prep.replay()
-            g_gather.replay()
+        pl0.set_inputs(hs, rngs[i % n_single])
+        if gp0 is not None:
+            gp0.replay()
+            gg0.replay()
         else:
-            pipe.enqueue()
-        for h, b in enumerate(pipe.hops):
+            pl0.enqueue()
+        for h, b in enumerate(pl0.hops):
             d2h[h, 0:1].copy_(b["num_edges"], non_blocking=True)
             d2h[h, 1:2].copy_(b["num_unique"], non_blocking=True)
         torch.cuda.current_stream().synchronize()
         if i >= 2:
             e2e_times.append(time.perf_counter() - t)
-    e2e_val = S / statistics.mean(e2e_times)
-    if world > 1:
-        t = torch.tensor([statistics.mean(e2e_times)], dtype=torch.float64, device=dev)
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        e2e_val = world * S / float(t.item())
+    e2e_val = world * S / max_over_ranks(statistics.mean(e2e_times))
 
     line = None
     if rank == 0:
@@ -319,39 +362,56 @@ def bench_wg(args):
             cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
                    "sample": f"{done} whole batches of {S} seeds (fanout {p.fanouts} + gather) of the same workload, "
                              f"{s_spent:.1f} s of single-threaded oracle work (row regeneration untimed)"}
+        cfg = workload_config(p, world, flush is not None)
+        cfg["concurrent_batches_per_gpu"] = P
         line = {
-            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": 1e3 * dev_s / args.steps, "higher_is_better": True,
+            "metric": METRIC, "value": value_conc, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 1e3 * dev_s_conc / args.steps, "higher_is_better": True,
             "scaling": "weak", "vs_baseline": None, "dtype": "int64 ids + fp32 feature bytes",
             "data": "synthetic (seeded power-law graph + procedural features, see DESIGN.md)",
-            "config": workload_config(p, world, flush is not None),
+            "config": cfg,
+            "single_batch": {"value": value_single, "unit": UNIT, "ms_per_batch": 1e3 * dev_s_single / args.steps,
+                             "ms_per_batch_median": statistics.median(step_ms)},
             "roofline": {"kernel": "wg::gather_kernel", "bound": bound, "achieved": achieved, "peak": peak,
-                         "unit": "GB/s", "frac": achieved / peak, "traffic": None,
+                         "unit": "GB/s", "frac": achieved / peak, "traffic": gather_traffic(),
                          "peak_source": peak_src,
                          "algorithmic_bytes_per_launch": alg_bytes / args.steps,
-                         "gather_ms_per_step": 1e3 * gather_s / args.steps,
-                         "gather_share_of_step": gather_s / dev_s},
+                         "gather_ms_per_launch": 1e3 * gather_s / args.steps,
+                         "gather_share_of_single_batch": gather_s / (sum(step_ms) / 1e3),
+                         "timed_in": "pass A (one batch at a time, events on the launching stream)"},
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_val, "unit": UNIT, "h2d_bytes_per_step": S * 8,
                     "d2h_bytes_per_step": int(d2h.numel() * 8),
-                    "note": "public API (MiniBatchPipeline.run): pinned-host seeds H2D, per-hop counts D2H, "
-                            "host-timed incl. sync"},
-            "gpu_launches": args.steps * (4 * len(p.fanouts) + 1),
+                    "note": "public API (MiniBatchPipeline.run), one batch per step: pinned-host seeds H2D, "
+                            "per-hop counts D2H, host-timed incl. sync"},
+            "gpu_launches": args.steps * (4 * len(p.fanouts) + 1) * (1 + P),
             "clocks": clk,
             "wall_s_timed_region": wall,
             "workload_stats": {"edges_per_hop_mean": hc[:, :, 0].mean(0).tolist(),
                                "unique_per_hop_mean": hc[:, :, 1].mean(0).tolist(),
-                               "unique_bound_per_hop": pipe.U_cap, "rows_gathered_mean": float(rows.mean()),
+                               "unique_bound_per_hop": pipes[0].U_cap, "rows_gathered_mean": float(rows.mean()),
                                "row_bytes": rb},
             "setup": {"total_s": setup_s, **info},
-            "step_ms_median": statistics.median(step_ms),
         }
         emit(line, args)
     torch.cuda.synchronize()
+    for h in handles[1:]:
+        h.destroy()
     dsm.destroy()
     if world > 1:
         dist.destroy_process_group()
     return line
+
+
+def gather_traffic():
+    """dram read+write bytes per launch of the gather kernel from the committed
+    `ncu --set full` summary (profiles/latest_gather_ncu.json), or None."""
+    pth = os.path.join(ROOT, "profiles", "latest_gather_ncu.json")
+    if not os.path.exists(pth):
+        return None
+    with open(pth) as f:
+        d = json.load(f)
+    return d.get("dram_bytes_per_launch")
 
 
 def main():

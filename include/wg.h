@@ -112,6 +112,14 @@ wg_status wg_dsm_local_view(wg_dsm_t h, int64_t** d_row_ptr, int64_t** d_col_idx
 /* Geometry of rank r's shard (any r): local rows and local CSR entries. */
 wg_status wg_dsm_shard_info(wg_dsm_t h, int32_t r, int64_t* n_local_rows, int64_t* local_num_edges);
 
+/* A second handle on the SAME shards with its own workspace (hash table, scan
+ * state, error word), so independent batches can be prepared concurrently on
+ * different streams (each handle's calls stay on one stream at a time).  Not
+ * collective; no memory is mapped or copied.  max_batch_keys = 0 copies the
+ * parent's.  Destroy forks (wg_dsm_destroy, not collective for a fork) before
+ * their parent. */
+wg_status wg_dsm_fork(wg_dsm_t parent, int64_t max_batch_keys, wg_dsm_t* out);
+
 /* Destroy (COLLECTIVE): barrier (no rank still reads a peer), close the peer
  * mappings, barrier (no peer still maps ours), free the shard and workspace.
  * The caller must have synchronised every stream that used the handle. */
@@ -132,7 +140,8 @@ wg_status wg_dsm_destroy(wg_dsm_t h);
  * adjacency list; d_out_num_edges (nullable) = device int64 total.
  * seed: the per-batch rng_seed; if d_seed is non-NULL the seed is read from that
  * device uint64 instead (so a captured CUDA graph can be replayed with new seeds).
- * Requires 1 <= fanout <= 32 (WG_ERR_UNSUPPORTED above 32). */
+ * Requires 1 <= fanout <= 32 (WG_ERR_UNSUPPORTED above 32) and n_targets * fanout <=
+ * max_batch_keys (the padded per-target slots live in the workspace). */
 wg_status wg_sample_neighbors(wg_dsm_t h, const int64_t* d_targets, int64_t n_targets,
                               const int64_t* d_n_targets, int32_t fanout, uint64_t seed,
                               const uint64_t* d_seed, int32_t hop, int64_t* d_out_row_ptr,
@@ -159,9 +168,10 @@ wg_status wg_append_unique(wg_dsm_t h, const int64_t* d_targets, int64_t n_targe
 /* One whole hop of mini-batch preparation = wg_sample_neighbors followed by
  * wg_append_unique on its output ("stacking multiple
  * single-layer sub-graph sampling"), with identical results, fused for B200: the
- * sampling kernel also performs the hash-table inserts of Append Unique (targets
- * in its count phase, each neighbour right after its load), so a hop is one
- * sampling kernel + one flag/scan kernel + one relabel kernel.  The relabel
+ * sampling kernel writes padded per-target slots without any scan, the insert
+ * pass of Append Unique reads them directly, and ONE single-pass scan both
+ * compacts the sampler output into the CSR (row_ptr, neighbours, positions) and
+ * numbers the first occurrences -- four kernels, no host sync.  The relabel
  * (which fills d_out_sub_col / d_out_dup_count) is launched on side_stream when
  * it is non-NULL (forked from `stream` with an event); the caller must make its
  * consumers wait for side_stream, and must join it before issuing a fifth

@@ -59,12 +59,14 @@ static wg_status barrier(wg_dsm* h) {
 
 static void free_workspace(wg_dsm* h) {
   Workspace& w = h->ws;
-  cudaFree(w.hkeys);
-  cudaFree(w.hvals);
+  cudaFree(w.hslots);
   cudaFree(w.status_sample);
   cudaFree(w.status_unique);
   for (int k = 0; k < EXCL_RING; ++k) cudaFree(w.excl[k]);
   cudaFree(w.slot_of);
+  cudaFree(w.nbrs_pad);
+  cudaFree(w.pos_pad);
+  cudaFree(w.cnt);
   cudaFree(w.ctrl);
   w = Workspace{};
 }
@@ -73,22 +75,24 @@ static wg_status alloc_workspace(wg_dsm* h, int64_t max_keys) {
   Workspace& w = h->ws;
   if (max_keys < 1) max_keys = 1;
   int64_t cap = 1024;
-  while (cap < 2 * max_keys) cap <<= 1;  // load factor <= 0.5
+  while (cap < max_keys + max_keys / 2) cap <<= 1;  // worst-case load <= 2/3 (typical batches: ~0.3)
   w.hcap = cap;
   w.max_keys = max_keys;
   w.status_cap = max_keys / 32 + 2;  // sampler tiles hold >= 32 targets, flag tiles 1024 positions
-  if (cudaMalloc(&w.hkeys, cap * 8) != cudaSuccess || cudaMalloc(&w.hvals, cap * 8) != cudaSuccess ||
+  if (cudaMalloc(&w.hslots, cap * sizeof(HashSlot)) != cudaSuccess ||
       cudaMalloc(&w.status_sample, w.status_cap * 8) != cudaSuccess ||
       cudaMalloc(&w.status_unique, w.status_cap * 8) != cudaSuccess ||
       cudaMalloc(&w.excl[0], max_keys * 4) != cudaSuccess || cudaMalloc(&w.excl[1], max_keys * 4) != cudaSuccess ||
       cudaMalloc(&w.excl[2], max_keys * 4) != cudaSuccess || cudaMalloc(&w.excl[3], max_keys * 4) != cudaSuccess ||
-      cudaMalloc(&w.slot_of, max_keys * 4) != cudaSuccess || cudaMalloc(&w.ctrl, CTRL_WORDS * 4) != cudaSuccess) {
+      cudaMalloc(&w.slot_of, max_keys * 4) != cudaSuccess || cudaMalloc(&w.nbrs_pad, max_keys * 8) != cudaSuccess ||
+      cudaMalloc(&w.pos_pad, max_keys * 4) != cudaSuccess || cudaMalloc(&w.cnt, max_keys * 4) != cudaSuccess ||
+      cudaMalloc(&w.ctrl, CTRL_WORDS * 4) != cudaSuccess) {
     cudaGetLastError();
     free_workspace(h);
     return fail(WG_ERR_OOM, "workspace allocation failed");
   }
-  WG_CUDA_TRY(cudaMemset(w.hkeys, 0, cap * 8));
-  WG_CUDA_TRY(cudaMemset(w.hvals, 0xff, cap * 8));
+  WG_CUDA_TRY(cudaMemset(w.hslots, 0xff, cap * sizeof(HashSlot)));                   // val = all ones
+  WG_CUDA_TRY(cudaMemset2D(w.hslots, sizeof(HashSlot), 0, sizeof(unsigned long long), cap));  // key = 0 (empty)
   WG_CUDA_TRY(cudaMemset(w.status_sample, 0, w.status_cap * 8));
   WG_CUDA_TRY(cudaMemset(w.status_unique, 0, w.status_cap * 8));
   unsigned ctrl[CTRL_WORDS] = {0};
@@ -99,6 +103,12 @@ static wg_status alloc_workspace(wg_dsm* h, int64_t max_keys) {
 
 static void release(wg_dsm* h) {
   if (h->fork_event) cudaEventDestroy(h->fork_event);
+  if (h->parent) {  // a workspace fork owns only its workspace
+    free_workspace(h);
+    h->parent->live_forks -= 1;
+    delete h;
+    return;
+  }
   for (int r = 0; r < h->world; ++r)
     if (h->peer_opened[r]) cudaIpcCloseMemHandle(h->peer_base[r]);
   free_workspace(h);
@@ -146,10 +156,6 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
   h->allgather = d->allgather;
   h->ctx = d->ctx;
   h->sm_count = sms;
-  {
-    const char* f = getenv("WG_FUSE_INSERT");  // A/B switch: 1 = hash inserts inside the sampler
-    h->fuse_insert = f && f[0] == '1';
-  }
   h->n_local = local_rows(h->n, h->rank, h->world);
   h->e_local = d->local_num_edges;
 
@@ -275,10 +281,47 @@ wg_status wg_dsm_shard_info(wg_dsm_t h, int32_t r, int64_t* n_local_rows, int64_
   return WG_OK;
 }
 
+wg_status wg_dsm_fork(wg_dsm_t parent, int64_t max_batch_keys, wg_dsm_t* out) {
+  if (!out) return fail(WG_ERR_INVALID_ARG, "out is NULL");
+  *out = nullptr;
+  if (!parent || parent->parent) return fail(WG_ERR_INVALID_ARG, "parent must be a DSM created by wg_dsm_create");
+  if (max_batch_keys < 0 || max_batch_keys >= (int64_t(1) << 31)) return fail(WG_ERR_INVALID_ARG, "max_batch_keys");
+  WG_CUDA_TRY(cudaSetDevice(parent->device));
+  wg_dsm* h = new wg_dsm();
+  *h = *parent;  // geometry, pointer table, callbacks
+  h->ws = Workspace{};
+  h->fork_event = nullptr;
+  h->parent = parent;
+  h->live_forks = 0;
+  h->excl_next = 0;
+  for (int r = 0; r < WG_MAX_WORLD; ++r) h->peer_opened[r] = false;  // mappings stay owned by the parent
+  h->slab = nullptr;
+  parent->live_forks += 1;
+  if (cudaEventCreateWithFlags(&h->fork_event, cudaEventDisableTiming) != cudaSuccess) {
+    cudaGetLastError();
+    h->fork_event = nullptr;
+    release(h);
+    return fail(WG_ERR_CUDA, "cudaEventCreate failed");
+  }
+  wg_status st = alloc_workspace(h, max_batch_keys ? max_batch_keys : parent->ws.max_keys);
+  if (st != WG_OK) {
+    std::string m = g_last_error;
+    release(h);
+    return fail(st, m);
+  }
+  *out = h;
+  return WG_OK;
+}
+
 wg_status wg_dsm_destroy(wg_dsm_t h) {
   if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
   cudaSetDevice(h->device);
   cudaDeviceSynchronize();
+  if (h->parent) {  // a fork: not collective
+    release(h);
+    return WG_OK;
+  }
+  if (h->live_forks > 0) return fail(WG_ERR_INVALID_ARG, "destroy the handle's forks first");
   wg_status s1 = barrier(h);  // nobody reads a peer any more
   for (int r = 0; r < h->world; ++r)
     if (h->peer_opened[r]) {
@@ -301,11 +344,12 @@ wg_status wg_sample_neighbors(wg_dsm_t h, const int64_t* d_targets, int64_t n_ta
   if (n_targets < 0 || (n_targets > 0 && !d_targets) || !d_out_row_ptr || (n_targets > 0 && !d_out_nbrs))
     return fail(WG_ERR_INVALID_ARG, "null pointer or negative size");
   if (hop < 0) return fail(WG_ERR_INVALID_ARG, "hop must be >= 0");
-  if (n_targets > h->ws.max_keys) return fail(WG_ERR_CAPACITY, "n_targets exceeds max_batch_keys");
+  if (n_targets * (int64_t)fanout > h->ws.max_keys)
+    return fail(WG_ERR_CAPACITY, "n_targets * fanout exceeds max_batch_keys");
   if (n_targets * (int64_t)fanout >= (int64_t(1) << 40)) return fail(WG_ERR_INVALID_ARG, "too many edges");
   cudaSetDevice(h->device);
   cudaError_t e = launch_sample(h, d_targets, n_targets, d_n_targets, fanout, seed, d_seed, hop, d_out_row_ptr,
-                                d_out_nbrs, d_out_pos, d_out_num_edges, false, (cudaStream_t)stream);
+                                d_out_nbrs, d_out_pos, d_out_num_edges, (cudaStream_t)stream);
   if (e != cudaSuccess) return fail(WG_ERR_CUDA, std::string("sample launch: ") + cudaGetErrorString(e));
   return WG_OK;
 }
@@ -323,8 +367,7 @@ wg_status wg_append_unique(wg_dsm_t h, const int64_t* d_targets, int64_t n_targe
     return fail(WG_ERR_CAPACITY, "n_targets + n_nbrs exceeds max_batch_keys");
   cudaSetDevice(h->device);
   cudaError_t e = launch_append_unique(h, d_targets, n_targets, d_n_targets, d_nbrs, n_nbrs, d_n_nbrs, d_out_unique,
-                                       d_out_num_unique, d_out_sub_col, d_out_dup_count, false, (cudaStream_t)stream,
-                                       nullptr);
+                                       d_out_num_unique, d_out_sub_col, d_out_dup_count, (cudaStream_t)stream);
   if (e != cudaSuccess) return fail(WG_ERR_CUDA, std::string("append_unique launch: ") + cudaGetErrorString(e));
   return WG_OK;
 }
@@ -343,14 +386,10 @@ wg_status wg_sample_hop(wg_dsm_t h, const int64_t* d_targets, int64_t n_targets,
   const int64_t n_nbrs = n_targets * (int64_t)fanout;
   if (n_targets + n_nbrs > h->ws.max_keys) return fail(WG_ERR_CAPACITY, "n_targets*(1+fanout) exceeds max_batch_keys");
   cudaSetDevice(h->device);
-  cudaStream_t st = (cudaStream_t)stream;
-  cudaError_t e = launch_sample(h, d_targets, n_targets, d_n_targets, fanout, seed, d_seed, hop, d_out_row_ptr,
-                                d_out_nbrs, d_out_pos, d_out_num_edges, h->fuse_insert, st);
-  if (e != cudaSuccess) return fail(WG_ERR_CUDA, std::string("sample launch: ") + cudaGetErrorString(e));
-  e = launch_append_unique(h, d_targets, n_targets, d_n_targets, d_out_nbrs, n_nbrs, d_out_num_edges, d_out_unique,
-                           d_out_num_unique, d_out_sub_col, d_out_dup_count, h->fuse_insert, st,
-                           (cudaStream_t)side_stream);
-  if (e != cudaSuccess) return fail(WG_ERR_CUDA, std::string("append_unique launch: ") + cudaGetErrorString(e));
+  cudaError_t e = launch_hop(h, d_targets, n_targets, d_n_targets, fanout, seed, d_seed, hop, d_out_row_ptr,
+                             d_out_nbrs, d_out_pos, d_out_num_edges, d_out_unique, d_out_num_unique, d_out_sub_col,
+                             d_out_dup_count, (cudaStream_t)stream, (cudaStream_t)side_stream);
+  if (e != cudaSuccess) return fail(WG_ERR_CUDA, std::string("hop launch: ") + cudaGetErrorString(e));
   return WG_OK;
 }
 
@@ -383,8 +422,8 @@ wg_status wg_dsm_reset_workspace(wg_dsm_t h, wg_stream_t stream) {
   if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
   cudaSetDevice(h->device);
   cudaStream_t st = (cudaStream_t)stream;
-  WG_CUDA_TRY(cudaMemsetAsync(h->ws.hkeys, 0, h->ws.hcap * 8, st));
-  WG_CUDA_TRY(cudaMemsetAsync(h->ws.hvals, 0xff, h->ws.hcap * 8, st));
+  WG_CUDA_TRY(cudaMemsetAsync(h->ws.hslots, 0xff, h->ws.hcap * sizeof(HashSlot), st));
+  WG_CUDA_TRY(cudaMemset2DAsync(h->ws.hslots, sizeof(HashSlot), 0, sizeof(unsigned long long), h->ws.hcap, st));
   static const unsigned one = 1;
   WG_CUDA_TRY(cudaMemcpyAsync(h->ws.ctrl + CTRL_EPOCH, &one, 4, cudaMemcpyHostToDevice, st));
   return WG_OK;

@@ -1,10 +1,11 @@
 // hash.cuh -- the append-unique hash table (PAPER.md: "The key of our GPU
 // hash table is nodeID"; Warpcore-style open addressing [33]).
 //
-// Slot s: hkeys[s] = (epoch << 40) | node id, hvals[s] = ((EPOCH_MAX - epoch) << 40) |
-// first position.  A key from an older epoch reads as an empty slot and an older
+// Slot s (16 B, key and value in the same 32 B sector so an insert touches one
+// sector): key = (epoch << 40) | node id, val = ((EPOCH_MAX - epoch) << 40) | first
+// position.  A key from an older epoch reads as an empty slot and an older
 // value always loses an atomicMin against the current epoch, so the table is never
-// cleared between calls.  Linear probing, fmix64 hash, load factor <= 0.5.
+// cleared between calls.  Linear probing, fmix64 hash, worst-case load <= 2/3.
 #pragma once
 
 #include "device_util.cuh"
@@ -15,8 +16,7 @@ namespace wg {
 constexpr unsigned long long KEY_MASK = (1ull << 40) - 1;
 
 struct HashTable {
-  unsigned long long* keys;
-  unsigned long long* vals;
+  HashSlot* slots;
   unsigned long long mask;  // capacity - 1
 };
 
@@ -32,11 +32,11 @@ __device__ __forceinline__ unsigned long long pack_pos(unsigned epoch, int64_t q
 __device__ __forceinline__ long long hash_insert(const HashTable& t, unsigned long long stored, unsigned epoch) {
   unsigned long long slot = fmix64(stored & KEY_MASK) & t.mask;
   for (unsigned long long probe = 0; probe <= t.mask; ++probe) {
-    unsigned long long cur = ld_volatile_u64(&t.keys[slot]);
+    unsigned long long cur = ld_volatile_u64(&t.slots[slot].key);
     for (;;) {
       if (cur == stored) return (long long)slot;
       if ((unsigned)(cur >> 40) == epoch) break;  // occupied by another key this epoch
-      const unsigned long long prev = atomicCAS(&t.keys[slot], cur, stored);
+      const unsigned long long prev = atomicCAS(&t.slots[slot].key, cur, stored);
       if (prev == cur || prev == stored) return (long long)slot;
       cur = prev;
     }
@@ -48,7 +48,7 @@ __device__ __forceinline__ long long hash_insert(const HashTable& t, unsigned lo
 __device__ __forceinline__ long long hash_find(const HashTable& t, unsigned long long stored, unsigned epoch) {
   unsigned long long slot = fmix64(stored & KEY_MASK) & t.mask;
   for (unsigned long long probe = 0; probe <= t.mask; ++probe) {
-    const unsigned long long cur = t.keys[slot];
+    const unsigned long long cur = t.slots[slot].key;
     if (cur == stored) return (long long)slot;
     if ((unsigned)(cur >> 40) != epoch) return -1;  // empty: not present
     slot = (slot + 1) & t.mask;
@@ -59,7 +59,7 @@ __device__ __forceinline__ long long hash_find(const HashTable& t, unsigned long
 // Insert `key` at position q, recording the minimum position.  Returns the slot or -1.
 __device__ __forceinline__ long long hash_insert_min(const HashTable& t, int64_t key, int64_t q, unsigned epoch) {
   const long long slot = hash_insert(t, stored_key(epoch, key), epoch);
-  if (slot >= 0) atomicMin(&t.vals[slot], pack_pos(epoch, q));
+  if (slot >= 0) atomicMin(&t.slots[slot].val, pack_pos(epoch, q));
   return slot;
 }
 

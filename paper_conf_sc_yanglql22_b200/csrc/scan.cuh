@@ -1,0 +1,74 @@
+// scan.cuh -- block-wide decoupled look-back for the single-pass scans.
+//
+// The whole block (not one warp) inspects NT predecessor tiles per step, so the
+// exclusive prefix of tile t resolves in ~t / NT dependent L2 round trips instead of
+// ~t / 32: with ~1000 tiles in flight this is what keeps the scans from serialising.
+#pragma once
+
+#include "device_util.cuh"
+
+namespace wg {
+
+template <int NT>
+struct LookbackSmem {
+  unsigned pmask[NT / 32];
+  unsigned long long part[NT / 32];
+  int stop;
+  int found;
+};
+
+// Called by ALL threads of the block.  Publishes `aggregate` for tile `tile`, resolves
+// the tile's exclusive prefix (returned in every thread) and publishes the inclusive
+// prefix.  Status word format as in device_util.cuh (LB_AGG / LB_PRE / LB_VAL).
+template <int NT>
+__device__ __forceinline__ unsigned long long block_lookback(unsigned long long* status, long tile,
+                                                             unsigned long long aggregate, LookbackSmem<NT>& sm) {
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  if (tile == 0) {
+    if (tid == 0) st_volatile_u64(&status[0], LB_PRE | aggregate);
+    return 0ull;
+  }
+  if (tid == 0) st_volatile_u64(&status[tile], LB_AGG | aggregate);
+  unsigned long long excl = 0;
+  long pred = tile - 1;
+  for (;;) {
+    const long idx = pred - tid;
+    unsigned long long s = idx >= 0 ? ld_volatile_u64(&status[idx]) : LB_PRE;
+    while ((s >> 62) == 0) {
+      __nanosleep(32);
+      s = ld_volatile_u64(&status[idx]);
+    }
+    const unsigned pm = __ballot_sync(FULL_MASK, (s >> 62) == 2);
+    if (lane == 0) sm.pmask[warp] = pm;
+    __syncthreads();
+    if (tid == 0) {
+      int stop = NT - 1, found = 0;
+      for (int w = 0; w < NT / 32; ++w)
+        if (sm.pmask[w]) {
+          stop = w * 32 + __ffs(sm.pmask[w]) - 1;  // closest predecessor holding an inclusive prefix
+          found = 1;
+          break;
+        }
+      sm.stop = stop;
+      sm.found = found;
+    }
+    __syncthreads();
+    const int stop = sm.stop;
+    const bool found = sm.found != 0;
+    unsigned long long v = tid <= stop ? (s & LB_VAL) : 0ull;
+    v = warp_sum(v);
+    if (lane == 0) sm.part[warp] = v;
+    __syncthreads();
+    unsigned long long tot = 0;
+#pragma unroll
+    for (int w = 0; w < NT / 32; ++w) tot += sm.part[w];
+    excl += tot;
+    __syncthreads();  // sm reused next step
+    if (found) break;
+    pred -= NT;
+  }
+  if (tid == 0) st_volatile_u64(&status[tile], LB_PRE | (excl + aggregate));
+  return excl;
+}
+
+}  // namespace wg

@@ -1,39 +1,52 @@
-// unique.cu -- Append Unique op with first-appearance numbering (A7).
+// unique.cu -- Append Unique op with first-appearance numbering (A7),
+// and its fusion with the sampling op for one whole hop (wg_sample_hop).
 //
 // Keys live in the open-addressing hash table of hash.cuh, which stays in L2.
 // Instead of the paper's per-bucket count of -1 values (whose order depends on the
 // insertion race), every key records the MINIMUM position at which it occurs in
-// the concatenated list [targets ; neighbours]; a neighbour position p is a "first
-// occurrence" iff that minimum equals nT + p, and the new ids are nT + exclusive
-// scan of the first-occurrence flags.  The result is deterministic and equals the
-// sequential definition.  Kernels:
-//   insert   all nT+nE keys; __match_any_sync elects one lane per distinct key in a
-//            warp; CAS claims a slot, atomicMin records the first position; every
-//            position remembers its slot (slot_of).  (Fused into the sampler by
-//            wg_sample_hop, sample.cu.)
-//   flag     single-pass scan over neighbour positions (decoupled look-back): reads
-//            the min position through slot_of (one dependent L2 read, no probing),
-//            writes U for first occurrences and the scan, and handles the targets
-//            (U[k] = T[k], duplicate-target check).  Its last block advances the
-//            table epoch.
+// the concatenated list [targets ; neighbours]; a neighbour position is a "first
+// occurrence" iff that minimum is its own position, and the new ids are nT +
+// exclusive scan of the first-occurrence flags.  The result is deterministic and
+// equals the sequential definition.  Kernels:
+//   insert   every key; __match_any_sync elects one lane per distinct key in a warp;
+//            CAS claims a slot, atomicMin records the first position; every position
+//            remembers its slot (slot_of).
+//   flag     single-pass scan (block-wide decoupled look-back) over the neighbour
+//            positions: reads the min position through slot_of (one dependent L2
+//            read, no probing), writes U for first occurrences, the scan, and handles
+//            the targets (U[k] = T[k], duplicate-target check).  Its last block
+//            advances the table epoch.
 //   relabel  sub_col[p] = id of nbrs[p]; optional duplicate counts (L186).  Nothing
-//            downstream in the batch needs it before the end, so it may run on a
-//            side stream.
+//            else in the batch reads it, so the fused hop runs it on a side stream.
+// PADDED = true is the fused hop: neighbours come from the sampler's padded slots
+// k*M + i (valid iff i < cnt[k]), positions are padded positions (same order as the
+// dense ones), and the flag pass scans "valid" and "first" together -- it also emits
+// the sampler's dense CSR (row_ptr, neighbours, positions), so no separate compaction
+// pass is needed.
 #include "hash.cuh"
+#include "scan.cuh"
 
 namespace wg {
 
 constexpr int UQ_THREADS = 256;
-constexpr int UQ_ITEMS = 4;
+constexpr int UQ_ITEMS = 8;
 constexpr int UQ_TILE = UQ_THREADS * UQ_ITEMS;  // neighbour positions per flag tile
+constexpr int CNT_BITS = 31;                    // packed scan value: (valid << 31) | first
 
 struct UniqueArgs {
   const int64_t* T;
   int64_t capT;
   const int64_t* d_nT;
-  const int64_t* nbrs;
-  int64_t capE;
-  const int64_t* d_nE;
+  const int64_t* nbrs;     // dense neighbours (standalone) or padded slots (PADDED)
+  int64_t capE;            // dense capacity (standalone) or capT * M (PADDED)
+  const int64_t* d_nE;     // dense count (standalone) or NULL (PADDED)
+  int M;                   // PADDED: fanout
+  const int32_t* cnt;      // PADDED: per-target sample counts
+  const int32_t* pos_pad;  // PADDED: adjacency positions of the padded slots (nullable)
+  int64_t* out_row_ptr;    // PADDED: dense CSR row pointer [nT+1]
+  int64_t* out_nbrs;       // PADDED: dense neighbours
+  int32_t* out_pos;        // PADDED: dense positions (nullable)
+  int64_t* d_num_edges;    // PADDED: dense neighbour count
   int64_t* U;
   int64_t* d_nU;
   int32_t* sub_col;
@@ -46,28 +59,26 @@ struct UniqueArgs {
   int64_t n;
 };
 
-__device__ __forceinline__ void load_counts(const UniqueArgs& a, int64_t& nT, int64_t& nE) {
-  nT = a.capT;
-  nE = a.capE;
-  if (a.d_nT) {
-    nT = *a.d_nT;
-    if (nT > a.capT || nT < 0) {
-      if (threadIdx.x == 0 && blockIdx.x == 0) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_CAPACITY);
-      nT = nT < 0 ? 0 : a.capT;
-    }
+__device__ __forceinline__ int64_t clamp_count(const int64_t* d, int64_t cap, unsigned* ctrl) {
+  if (!d) return cap;
+  int64_t v = *d;
+  if (v > cap || v < 0) {
+    if (threadIdx.x == 0 && blockIdx.x == 0) latch_error(&ctrl[CTRL_ERR], WG_DEVERR_CAPACITY);
+    v = v < 0 ? 0 : cap;
   }
-  if (a.d_nE) {
-    nE = *a.d_nE;
-    if (nE > a.capE || nE < 0) {
-      if (threadIdx.x == 0 && blockIdx.x == 0) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_CAPACITY);
-      nE = nE < 0 ? 0 : a.capE;
-    }
-  }
+  return v;
 }
 
+template <bool PADDED>
+__device__ __forceinline__ void load_counts(const UniqueArgs& a, int64_t& nT, int64_t& nE) {
+  nT = clamp_count(a.d_nT, a.capT, a.ctrl);
+  nE = PADDED ? nT * a.M : clamp_count(a.d_nE, a.capE, a.ctrl);
+}
+
+template <bool PADDED>
 __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueArgs a) {
   int64_t nT, nE;
-  load_counts(a, nT, nE);
+  load_counts<PADDED>(a, nT, nE);
   const unsigned epoch = a.ctrl[CTRL_EPOCH];
   const int64_t total = nT + nE;
   const int lane = threadIdx.x & 31;
@@ -78,8 +89,17 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueA
     bool valid = q < total;
     int64_t key = 0;
     if (valid) {
-      key = q < nT ? a.T[q] : a.nbrs[q - nT];
-      if (key < 0 || key >= a.n) {
+      if (q < nT) {
+        key = a.T[q];
+      } else if (PADDED) {
+        const int64_t j = q - nT;
+        const int64_t k = j / a.M;
+        valid = (int)(j - k * a.M) < a.cnt[k];
+        if (valid) key = a.nbrs[j];
+      } else {
+        key = a.nbrs[q - nT];
+      }
+      if (valid && (key < 0 || key >= a.n)) {
         latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_ID_RANGE);
         a.slot_of[q] = -1;
         valid = false;
@@ -100,17 +120,18 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueA
 
 __device__ __forceinline__ int64_t min_pos_at(const UniqueArgs& a, int32_t slot) {
   if (slot < 0) return -1;
-  return (int64_t)(a.ht.vals[slot] & KEY_MASK);
+  return (int64_t)(a.ht.slots[slot].val & KEY_MASK);
 }
 
+template <bool PADDED>
 __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArgs a) {
-  __shared__ int sm_wtot[UQ_THREADS / 32 + 1];
-  __shared__ unsigned long long sm_prefix;
+  __shared__ LookbackSmem<UQ_THREADS> lb;
+  __shared__ unsigned long long sm_wtot[UQ_THREADS / 32 + 1];
   __shared__ int sm_flag;
   int64_t nT, nE;
-  load_counts(a, nT, nE);
+  load_counts<PADDED>(a, nT, nE);
   const unsigned epoch = a.ctrl[CTRL_EPOCH];
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int tid = threadIdx.x;
 
   // targets: U[k] = T[k] (targets first, original order, L160); duplicate check (A8)
   for (int64_t k = (int64_t)blockIdx.x * UQ_THREADS + tid; k < nT; k += (int64_t)gridDim.x * UQ_THREADS) {
@@ -122,49 +143,91 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArg
 
   const int64_t tile_start = (int64_t)blockIdx.x * UQ_TILE;
   if (nE == 0) {
-    if (blockIdx.x == 0 && tid == 0 && a.d_nU) *a.d_nU = nT;
+    if (blockIdx.x == 0 && tid == 0) {
+      if (a.d_nU) *a.d_nU = nT;
+      if (PADDED) {
+        a.out_row_ptr[0] = 0;  // nT == 0 here (M >= 1)
+        if (a.d_num_edges) *a.d_num_edges = 0;
+      }
+    }
   } else if (tile_start < nE) {
+    const int64_t j0 = tile_start + (int64_t)tid * UQ_ITEMS;
     int32_t slots[UQ_ITEMS];
-    int64_t mps[UQ_ITEMS];
-    const int64_t p0 = tile_start + (int64_t)tid * UQ_ITEMS;
-    // coalesced 16-byte read of this thread's 4 slots when aligned (p0 is a multiple of 4)
-    if (p0 + UQ_ITEMS <= nE && (nT & 3) == 0) {
-      const int4 s4 = *reinterpret_cast<const int4*>(a.slot_of + nT + p0);
-      slots[0] = s4.x; slots[1] = s4.y; slots[2] = s4.z; slots[3] = s4.w;
+    bool valid[UQ_ITEMS];
+    int64_t k0 = 0;
+    int i0 = 0;
+    if (PADDED) {
+      k0 = j0 / a.M;
+      i0 = (int)(j0 - k0 * a.M);
+      int64_t k = k0;
+      int i = i0;
+      int c = k < nT ? a.cnt[k] : 0;
+#pragma unroll
+      for (int t = 0; t < UQ_ITEMS; ++t) {
+        valid[t] = (j0 + t < nE) && i < c;
+        if (++i == a.M) {
+          i = 0;
+          ++k;
+          c = (t + 1 < UQ_ITEMS && k < nT) ? a.cnt[k] : 0;
+        }
+      }
     } else {
 #pragma unroll
-      for (int j = 0; j < UQ_ITEMS; ++j) slots[j] = (p0 + j < nE) ? a.slot_of[nT + p0 + j] : -1;
+      for (int t = 0; t < UQ_ITEMS; ++t) valid[t] = j0 + t < nE;
     }
 #pragma unroll
-    for (int j = 0; j < UQ_ITEMS; ++j) mps[j] = min_pos_at(a, slots[j]);  // independent L2 reads
-    int cnt = 0;
-    int first[UQ_ITEMS];
+    for (int t = 0; t < UQ_ITEMS; ++t) slots[t] = valid[t] ? a.slot_of[nT + j0 + t] : -1;
+    int64_t mps[UQ_ITEMS];
 #pragma unroll
-    for (int j = 0; j < UQ_ITEMS; ++j) {
-      const int64_t p = p0 + j;
-      first[j] = (p < nE) && (mps[j] == nT + p);
-      if (p < nE) {
-        a.sub_col[p] = (int32_t)mps[j];  // temporary: min position (relabel turns it into an id)
-        if (a.dup) a.dup[nT + p] = 0;
+    for (int t = 0; t < UQ_ITEMS; ++t) mps[t] = min_pos_at(a, slots[t]);  // independent L2 reads
+    unsigned long long nv = 0, nf = 0;
+    bool first[UQ_ITEMS];
+#pragma unroll
+    for (int t = 0; t < UQ_ITEMS; ++t) {
+      first[t] = valid[t] && mps[t] == nT + j0 + t;
+      nv += valid[t];
+      nf += first[t];
+    }
+    unsigned long long agg;
+    const unsigned long long ex =
+        block_exclusive_sum<UQ_THREADS>((nv << CNT_BITS) | nf, sm_wtot, &agg);
+    const unsigned long long pre = block_lookback<UQ_THREADS>(a.status, (long)blockIdx.x, agg, lb);
+    const unsigned long long base = pre + ex;
+    int64_t ev = (int64_t)(base >> CNT_BITS);                   // dense position of the next valid slot
+    int64_t ef = (int64_t)(base & ((1ull << CNT_BITS) - 1));    // next new-node index
+    int64_t k = k0;
+    int i = i0;
+#pragma unroll
+    for (int t = 0; t < UQ_ITEMS; ++t) {
+      const int64_t j = j0 + t;
+      if (j < nE) {
+        if (PADDED && i == 0) a.out_row_ptr[k] = ev;
+        if (valid[t]) {
+          const int64_t p = PADDED ? ev : j;
+          if (PADDED) {
+            a.out_nbrs[p] = a.nbrs[j];
+            if (a.out_pos) a.out_pos[p] = a.pos_pad[j];
+          }
+          a.sub_col[p] = (int32_t)mps[t];  // temporary: min position (relabel turns it into an id)
+          if (first[t]) {
+            a.U[nT + ef] = a.nbrs[j];
+            if (a.dup) a.dup[nT + ef] = 0;
+            a.excl[j] = (int32_t)ef;
+          }
+          ev += 1;
+          ef += first[t];
+        }
+        if (j == nE - 1) {
+          if (a.d_nU) *a.d_nU = nT + ef;
+          if (PADDED) {
+            a.out_row_ptr[nT] = ev;
+            if (a.d_num_edges) *a.d_num_edges = ev;
+          }
+        }
       }
-      cnt += first[j];
-    }
-    int agg;
-    const int ex = block_exclusive_sum<UQ_THREADS>(cnt, sm_wtot, &agg);
-    if (warp == 0) {
-      const unsigned long long pre = tile_lookback(a.status, (long)blockIdx.x, (unsigned long long)agg);
-      if (lane == 0) sm_prefix = pre;
-    }
-    __syncthreads();
-    int64_t run = (int64_t)sm_prefix + ex;
-#pragma unroll
-    for (int j = 0; j < UQ_ITEMS; ++j) {
-      const int64_t p = p0 + j;
-      if (p < nE) {
-        a.excl[p] = (int32_t)run;
-        if (first[j]) a.U[nT + run] = a.nbrs[p];
-        run += first[j];
-        if (p == nE - 1 && a.d_nU) *a.d_nU = nT + run;
+      if (PADDED && ++i == a.M) {
+        i = 0;
+        ++k;
       }
     }
   }
@@ -182,9 +245,11 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArg
   }
 }
 
+// sub_col[p] = id of neighbour p; d_nE = the dense neighbour count.
 __global__ void __launch_bounds__(UQ_THREADS) unique_relabel_kernel(const UniqueArgs a) {
-  int64_t nT, nE;
-  load_counts(a, nT, nE);
+  const int64_t nT = clamp_count(a.d_nT, a.capT, a.ctrl);
+  int64_t nE = a.d_nE ? *a.d_nE : a.capE;
+  nE = nE < 0 ? 0 : (nE > a.capE ? a.capE : nE);
   for (int64_t p = (int64_t)blockIdx.x * UQ_THREADS + threadIdx.x; p < nE; p += (int64_t)gridDim.x * UQ_THREADS) {
     const int32_t mp = a.sub_col[p];
     int32_t id = -1;
@@ -194,39 +259,31 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_relabel_kernel(const Unique
   }
 }
 
-cudaError_t launch_append_unique(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t* d_nT,
-                                 const int64_t* nbrs, int64_t capE, const int64_t* d_nE, int64_t* U,
-                                 int64_t* d_nU, int32_t* sub_col, int32_t* dup, bool inserted, cudaStream_t st,
-                                 cudaStream_t side) {
-  UniqueArgs a;
-  a.T = T;
-  a.capT = capT;
-  a.d_nT = d_nT;
-  a.nbrs = nbrs;
-  a.capE = capE;
-  a.d_nE = d_nE;
-  a.U = U;
-  a.d_nU = d_nU;
-  a.sub_col = sub_col;
-  a.dup = dup;
+static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, cudaStream_t st, cudaStream_t side) {
   a.excl = h->ws.excl[h->excl_next];
   h->excl_next = (h->excl_next + 1) % EXCL_RING;
   a.slot_of = h->ws.slot_of;
-  a.ht = HashTable{h->ws.hkeys, h->ws.hvals, (unsigned long long)h->ws.hcap - 1};
+  a.ht = HashTable{h->ws.hslots, (unsigned long long)h->ws.hcap - 1};
   a.status = h->ws.status_unique;
   a.ctrl = h->ws.ctrl;
   a.n = h->n;
-  const int64_t total = capT + capE;
+  const int64_t total = a.capT + a.capE;
   const int64_t max_blocks = (int64_t)h->sm_count * 8;
-  if (!inserted) {
-    int64_t ib = (total + UQ_THREADS - 1) / UQ_THREADS;
-    ib = ib < 1 ? 1 : (ib > max_blocks ? max_blocks : ib);
-    unique_insert_kernel<<<(unsigned)ib, UQ_THREADS, 0, st>>>(a);
+  int64_t ib = (total + UQ_THREADS - 1) / UQ_THREADS;
+  ib = ib < 1 ? 1 : (ib > max_blocks ? max_blocks : ib);
+  const unsigned fb = (unsigned)(a.capE > 0 ? (a.capE + UQ_TILE - 1) / UQ_TILE : 1);
+  if (padded) {
+    unique_insert_kernel<true><<<(unsigned)ib, UQ_THREADS, 0, st>>>(a);
+    unique_flag_kernel<true><<<fb, UQ_THREADS, 0, st>>>(a);
+  } else {
+    unique_insert_kernel<false><<<(unsigned)ib, UQ_THREADS, 0, st>>>(a);
+    unique_flag_kernel<false><<<fb, UQ_THREADS, 0, st>>>(a);
   }
-  int64_t fb = capE > 0 ? (capE + UQ_TILE - 1) / UQ_TILE : 1;
-  unique_flag_kernel<<<(unsigned)fb, UQ_THREADS, 0, st>>>(a);
-  if (capE > 0) {
-    int64_t rb = (capE + UQ_THREADS - 1) / UQ_THREADS;
+  if (a.capE > 0) {
+    // relabel runs over the DENSE neighbours: count = num_edges (padded) or d_nE
+    UniqueArgs r = a;
+    if (padded) r.d_nE = a.d_num_edges;
+    int64_t rb = (a.capE + UQ_THREADS - 1) / UQ_THREADS;
     rb = rb > max_blocks ? max_blocks : rb;
     cudaStream_t rs = st;
     if (side && side != st) {
@@ -236,9 +293,57 @@ cudaError_t launch_append_unique(wg_dsm* h, const int64_t* T, int64_t capT, cons
       if (e != cudaSuccess) return e;
       rs = side;
     }
-    unique_relabel_kernel<<<(unsigned)rb, UQ_THREADS, 0, rs>>>(a);
+    unique_relabel_kernel<<<(unsigned)rb, UQ_THREADS, 0, rs>>>(r);
   }
   return cudaGetLastError();
+}
+
+cudaError_t launch_append_unique(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t* d_nT,
+                                 const int64_t* nbrs, int64_t capE, const int64_t* d_nE, int64_t* U,
+                                 int64_t* d_nU, int32_t* sub_col, int32_t* dup, cudaStream_t st) {
+  UniqueArgs a{};
+  a.T = T;
+  a.capT = capT;
+  a.d_nT = d_nT;
+  a.nbrs = nbrs;
+  a.capE = capE;
+  a.d_nE = d_nE;
+  a.M = 1;
+  a.U = U;
+  a.d_nU = d_nU;
+  a.sub_col = sub_col;
+  a.dup = dup;
+  return launch_unique_passes(h, a, false, st, nullptr);
+}
+
+cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap, const int64_t* d_n, int fanout,
+                                 uint64_t seed, const uint64_t* d_seed, int hop, bool want_pos, cudaStream_t st);
+
+cudaError_t launch_hop(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t* d_nT, int fanout, uint64_t seed,
+                       const uint64_t* d_seed, int hop, int64_t* out_row_ptr, int64_t* out_nbrs, int32_t* out_pos,
+                       int64_t* d_num_edges, int64_t* U, int64_t* d_nU, int32_t* sub_col, int32_t* dup,
+                       cudaStream_t st, cudaStream_t side) {
+  cudaError_t e = launch_sample_padded(h, T, capT, d_nT, fanout, seed, d_seed, hop, out_pos != nullptr, st);
+  if (e != cudaSuccess) return e;
+  UniqueArgs a{};
+  a.T = T;
+  a.capT = capT;
+  a.d_nT = d_nT;
+  a.nbrs = h->ws.nbrs_pad;
+  a.capE = capT * fanout;
+  a.d_nE = nullptr;
+  a.M = fanout;
+  a.cnt = h->ws.cnt;
+  a.pos_pad = h->ws.pos_pad;
+  a.out_row_ptr = out_row_ptr;
+  a.out_nbrs = out_nbrs;
+  a.out_pos = out_pos;
+  a.d_num_edges = d_num_edges;
+  a.U = U;
+  a.d_nU = d_nU;
+  a.sub_col = sub_col;
+  a.dup = dup;
+  return launch_unique_passes(h, a, true, st, side);
 }
 
 }  // namespace wg

@@ -49,9 +49,12 @@ __device__ __forceinline__ void owner_local(const ShardView& s, int64_t v, int& 
 // call is either epoch-tagged (hash table) or reset by the last block of the
 // kernel that used it (scan status + done counters), so no memset is needed per
 // call and every op is CUDA-graph capturable.
+struct __align__(16) HashSlot {
+  unsigned long long key;  // (epoch << 40) | node id
+  unsigned long long val;  // ((EPOCH_MAX - epoch) << 40) | first position
+};
 struct Workspace {
-  unsigned long long* hkeys = nullptr;   // [hcap] (epoch << 40) | node id
-  unsigned long long* hvals = nullptr;   // [hcap] ((EPOCH_MAX - epoch) << 40) | first position
+  HashSlot* hslots = nullptr;            // [hcap] append-unique hash table (hash.cuh)
   int64_t hcap = 0;                      // power of two
   unsigned long long* status_sample = nullptr;  // decoupled look-back tile status
   unsigned long long* status_unique = nullptr;
@@ -60,6 +63,9 @@ struct Workspace {
                                          // first-occurrence flags (a relabel on a side stream may
                                          // still read one while the next hops write the others)
   int32_t* slot_of = nullptr;            // [max_keys] hash slot of every position of the current call
+  int64_t* nbrs_pad = nullptr;           // [max_keys] sampler output, padded slots k*M + i
+  int32_t* pos_pad = nullptr;            // [max_keys] adjacency positions of the padded slots
+  int32_t* cnt = nullptr;                // [max_keys] per-target sample counts min(M, deg)
   unsigned* ctrl = nullptr;              // [16] control words (see CTRL_*)
   int64_t max_keys = 0;
 };
@@ -84,20 +90,24 @@ struct wg_dsm {
   wg_allgather_fn allgather = nullptr;
   void* ctx = nullptr;
   int sm_count = 148;
-  bool fuse_insert = false;             // wg_sample_hop: inserts inside the sampler (else a separate pass)
   int excl_next = 0;                    // next excl ring slot (host-side, per call)
   cudaEvent_t fork_event = nullptr;     // relabel fork onto a side stream
+  wg_dsm* parent = nullptr;             // set for a workspace fork (wg_dsm_fork): shards are the parent's
+  int live_forks = 0;                   // forks of this handle not yet destroyed
 };
 
 namespace wg {
 // launchers (stream-ordered); arguments already validated by the ABI layer
 cudaError_t launch_sample(wg_dsm* h, const int64_t* targets, int64_t cap, const int64_t* d_n, int fanout,
                           uint64_t seed, const uint64_t* d_seed, int hop, int64_t* out_row_ptr,
-                          int64_t* out_nbrs, int32_t* out_pos, int64_t* d_num_edges, bool fused, cudaStream_t st);
+                          int64_t* out_nbrs, int32_t* out_pos, int64_t* d_num_edges, cudaStream_t st);
 cudaError_t launch_append_unique(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t* d_nT,
                                  const int64_t* nbrs, int64_t capE, const int64_t* d_nE, int64_t* U,
-                                 int64_t* d_nU, int32_t* sub_col, int32_t* dup, bool inserted, cudaStream_t st,
-                                 cudaStream_t side);
+                                 int64_t* d_nU, int32_t* sub_col, int32_t* dup, cudaStream_t st);
+cudaError_t launch_hop(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t* d_nT, int fanout, uint64_t seed,
+                       const uint64_t* d_seed, int hop, int64_t* out_row_ptr, int64_t* out_nbrs, int32_t* out_pos,
+                       int64_t* d_num_edges, int64_t* U, int64_t* d_nU, int32_t* sub_col, int32_t* dup,
+                       cudaStream_t st, cudaStream_t side);
 cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int64_t* d_n, void* out,
                           cudaStream_t st);
 }  // namespace wg

@@ -152,6 +152,18 @@ class DSM:
             check(lib().wg_dsm_destroy(self.h))
         self.h = None
 
+    def fork(self, max_batch_keys=0):
+        """Another handle on the same shards with its own workspace (wg_dsm_fork), for
+        preparing independent batches concurrently on another stream."""
+        f = DSM.__new__(DSM)
+        f.__dict__.update({k: v for k, v in self.__dict__.items() if k != "h"})
+        if max_batch_keys:
+            f.max_batch_keys = max_batch_keys
+        h = ctypes.c_void_p()
+        check(lib().wg_dsm_fork(self.h, max_batch_keys, ctypes.byref(h)))
+        f.h = h
+        return f
+
     # --- the three ops --------------------------------------------------------
     def sample_neighbors(self, targets, fanout, seed, hop, n_targets_dev=None, seed_dev=None, out_row_ptr=None,
                          out_nbrs=None, out_pos=None, out_num_edges=None, cap=None, with_pos=False, stream=None):

@@ -179,3 +179,37 @@ def test_determinism_two_runs(tiny):
             assert np.array_equal(a[k], b[k])
     assert np.array_equal(outs[0][2], outs[1][2])
     dsm.destroy()
+
+
+def test_fork_concurrent_streams(tiny):
+    """wg_dsm_fork: two pipelines on the same shards, different workspaces, running
+    concurrently on two streams, both bit-exact."""
+    p, rp, col = tiny
+    dsm, _ = loader.build_dsm(p, on_device=False)
+    child = dsm.fork()
+    pipes = [pkg.MiniBatchPipeline(h, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
+             for h in (dsm, child)]
+    streams = [torch.cuda.Stream(), torch.cuda.Stream()]
+    rows = loader.host_row_provider(p.graph(), rp, col)
+    feats = loader.host_feat_provider(p)
+    for rnd in range(3):
+        Ss, rss = [], []
+        for j in range(2):
+            b = 100 + 2 * rnd + j
+            S = seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, b)
+            rs = seeds.rng_seed(presets.RNG_BASE, b)
+            Ss.append(S)
+            rss.append(rs)
+            st = streams[j]
+            st.wait_stream(torch.cuda.current_stream())
+            with torch.cuda.stream(st):
+                pipes[j].set_inputs(torch.from_numpy(S).cuda(), rs, stream=st)
+                pipes[j].enqueue(st)
+        torch.cuda.synchronize()
+        for j in range(2):
+            _check_batch(pipes[j], oracle.minibatch(rows, feats, Ss[j], p.fanouts, rss[j]), p.fanouts)
+    assert dsm.device_error() == 0 and child.device_error() == 0
+    with pytest.raises(pkg.WgError):
+        dsm.destroy()            # forks first
+    child.destroy()
+    dsm.destroy()
