@@ -202,7 +202,10 @@ def bench_wg(args):
     # P independent batch pipelines on P streams; pipeline j > 0 runs on a workspace fork of the DSM
     handles = [dsm] + [dsm.fork() for _ in range(P - 1)]
     pipes = [pkg.MiniBatchPipeline(h, p.fanouts, S) for h in handles]
-    streams = [torch.cuda.Stream(device=dev) for _ in range(P)]
+    # prep (latency-bound hops) on high-priority streams, gathers (bandwidth-bound) on low-priority ones,
+    # so the block scheduler interleaves the hops of one batch with the gather of another
+    streams = [torch.cuda.Stream(device=dev, priority=-1) for _ in range(P)]
+    gstreams = [torch.cuda.Stream(device=dev, priority=0) for _ in range(P)]
     n_single = args.warmup + args.steps
     n_conc = args.warmup + args.steps * P
     my_batches = [k * world + rank for k in range(n_single + n_conc)]
@@ -295,9 +298,10 @@ def bench_wg(args):
         for j in range(P):
             streams[j].wait_stream(main)
             launch(j, n_single + args.warmup + i * P + j, streams[j])
-            gather(j, streams[j])
+            gstreams[j].wait_stream(streams[j])
+            gather(j, gstreams[j])
         for j in range(P):
-            main.wait_stream(streams[j])
+            main.wait_stream(gstreams[j])
         evB[i][1].record(main)
     torch.cuda.synchronize()
     if world > 1:

@@ -10,13 +10,15 @@
 // ~8 x 256 threads per SM keeps ~0.5 MB in flight chip-wide -- enough to cover
 // local-HBM and NVLink latency.  Rows whose size is not a multiple of 16 use the
 // same scheme with 4- or 2-byte chunks.
+#include <algorithm>
+#include <cstdlib>
+
 #include "device_util.cuh"
 #include "wg_internal.cuh"
 
 namespace wg {
 
 constexpr int GATHER_THREADS = 256;
-constexpr int GATHER_UNROLL = 4;
 
 // n / d for n < 2^31 via multiply-high (Granlund-Montgomery; d >= 1).
 struct FastDiv {
@@ -55,7 +57,7 @@ struct GatherArgs {
   FastDiv cpr;  // chunks per row
 };
 
-template <typename V>
+template <typename V, int GATHER_UNROLL>
 __global__ void __launch_bounds__(GATHER_THREADS) gather_kernel(const GatherArgs a) {
   int64_t n = a.cap;
   if (a.d_n) {
@@ -97,34 +99,170 @@ __global__ void __launch_bounds__(GATHER_THREADS) gather_kernel(const GatherArgs
   }
 }
 
+// ---------------------------------------------------------------------------- TMA variant
+// One warp per block; the warp owns TMA_STAGES smem stages of R rows.  For each tile of
+// R consecutive output rows, lane r issues one bulk copy (cp.async.bulk, the TMA engine,
+// no registers involved) of row r from the owner shard into the stage, all signalling
+// one mbarrier with complete_tx; when the stage is full, lane 0 writes the whole tile
+// (R * row_bytes contiguous bytes of X) with ONE bulk smem->global store.  TMA_STAGES
+// tiles are in flight per warp.  Requires row_bytes % 16 == 0.
+constexpr int TMA_STAGES = 4;
+constexpr int TMA_STAGE_BYTES = 16 * 1024;
+
+__device__ __forceinline__ unsigned smem_u32(const void* p) {
+  return (unsigned)__cvta_generic_to_shared(p);
+}
+
+__global__ void __launch_bounds__(32) gather_tma_kernel(const GatherArgs a, int rows_per_tile, int row_bytes) {
+  extern __shared__ __align__(128) uint8_t smem[];
+  __shared__ __align__(8) unsigned long long mbar[TMA_STAGES];
+  const int lane = threadIdx.x;
+  int64_t n = a.cap;
+  if (a.d_n) {
+    n = *a.d_n;
+    if (n > a.cap || n < 0) {
+      if (lane == 0 && blockIdx.x == 0) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_CAPACITY);
+      n = n < 0 ? 0 : a.cap;
+    }
+  }
+  const int R = rows_per_tile;
+  const int64_t ntiles = (n + R - 1) / R;
+  if (lane == 0) {
+    for (int s = 0; s < TMA_STAGES; ++s)
+      asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&mbar[s])));
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncwarp();
+
+  auto issue = [&](int64_t tile, int s) {
+    const int64_t r0 = tile * R;
+    const int rows = (int)min((int64_t)R, n - r0);
+    uint8_t* stage = smem + (size_t)s * R * row_bytes;
+    bool ok = false;
+    const uint8_t* src = nullptr;
+    if (lane < rows) {
+      const int64_t v = a.ids[r0 + lane];
+      if (v >= 0 && v < a.s.n) {
+        int o;
+        int64_t l;
+        owner_local(a.s, v, o, l);
+        src = a.s.feat[o] + l * a.s.feat_stride;
+        ok = true;
+      } else {
+        latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_ID_RANGE);
+        uint4* z = reinterpret_cast<uint4*>(stage + (size_t)lane * row_bytes);
+        for (int c = 0; c < row_bytes / 16; ++c) z[c] = make_uint4(0, 0, 0, 0);
+      }
+    }
+    const unsigned nvalid = __popc(__ballot_sync(FULL_MASK, ok));
+    if (lane == 0) {
+      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // zero rows visible to the bulk store
+      asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(&mbar[s])),
+                   "r"(nvalid * (unsigned)row_bytes)
+                   : "memory");
+    }
+    __syncwarp();
+    if (ok)
+      asm volatile(
+          "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+              smem_u32(stage + (size_t)lane * row_bytes)),
+          "l"(src), "r"(row_bytes), "r"(smem_u32(&mbar[s]))
+          : "memory");
+  };
+
+  int64_t k = 0;
+  for (int s = 0; s < TMA_STAGES; ++s) {
+    const int64_t t = blockIdx.x + (int64_t)s * gridDim.x;
+    if (t < ntiles) issue(t, s);
+  }
+  for (int64_t t = blockIdx.x; t < ntiles; t += gridDim.x, ++k) {
+    const int s = (int)(k % TMA_STAGES);
+    const unsigned phase = (unsigned)((k / TMA_STAGES) & 1);
+    asm volatile(
+        "{\n .reg .pred p;\n WAIT_%=:\n mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1;\n @!p bra WAIT_%=;\n }" ::
+            "r"(smem_u32(&mbar[s])),
+        "r"(phase)
+        : "memory");
+    const int64_t r0 = t * R;
+    const int rows = (int)min((int64_t)R, n - r0);
+    uint8_t* stage = smem + (size_t)s * R * row_bytes;
+    if (lane == 0) {
+      asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(a.out + r0 * row_bytes),
+                   "r"(smem_u32(stage)), "r"((unsigned)(rows * row_bytes))
+                   : "memory");
+      asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+      asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // stage may be refilled
+    }
+    __syncwarp();
+    const int64_t tn = t + (int64_t)TMA_STAGES * gridDim.x;
+    if (tn < ntiles) issue(tn, s);
+  }
+  if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
+}
+
 cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int64_t* d_n, void* out,
                           cudaStream_t st) {
   const int64_t rb = h->row_bytes;
   int vb = (rb % 16 == 0 && ((uintptr_t)out % 16) == 0) ? 16 : (rb % 4 == 0 && ((uintptr_t)out % 4) == 0) ? 4 : 2;
   GatherArgs a{h->view, ids, cap, d_n, static_cast<uint8_t*>(out), h->ws.ctrl, FastDiv((unsigned)(rb / vb))};
   const int64_t total = cap * (rb / vb);
-  int64_t blocks = (total + GATHER_THREADS * GATHER_UNROLL - 1) / (GATHER_THREADS * GATHER_UNROLL);
-  // one full wave: resident blocks per SM (from the occupancy calculator) x SMs
-  static int occ[3] = {0, 0, 0};
-  const int which = vb == 16 ? 0 : (vb == 4 ? 1 : 2);
-  if (!occ[which]) {
-    int nb = 0;
-    if (vb == 16)
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<uint4>, GATHER_THREADS, 0);
-    else if (vb == 4)
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<unsigned>, GATHER_THREADS, 0);
-    else
-      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<unsigned short>, GATHER_THREADS, 0);
-    occ[which] = nb > 0 ? nb : 4;
+  // knobs (read once): WG_GATHER_UNROLL = independent 16 B loads in flight per thread (4 or 8),
+  // WG_GATHER_BPS = resident blocks per SM to use (0 = as many as fit: one full wave)
+  static int unroll = 0, bps = -1, use_tma = 0;
+  if (unroll == 0) {
+    const char* u = getenv("WG_GATHER_UNROLL");
+    unroll = (u && atoi(u) == 8) ? 8 : 4;
+    const char* b = getenv("WG_GATHER_BPS");
+    bps = b ? atoi(b) : 0;
+    const char* t = getenv("WG_GATHER_TMA");
+    use_tma = (t && t[0] == '1') ? 1 : 0;
   }
-  const int64_t max_blocks = (int64_t)h->sm_count * occ[which];
+  if (use_tma && vb == 16 && rb <= TMA_STAGE_BYTES) {
+    const int R = (int)std::min<int64_t>(32, TMA_STAGE_BYTES / rb);
+    const int smem = TMA_STAGES * R * (int)rb;
+    static int tma_bps = 0;
+    if (!tma_bps) {
+      cudaFuncSetAttribute(gather_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, TMA_STAGES * TMA_STAGE_BYTES);
+      int nb = 0;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_tma_kernel, 32, TMA_STAGES * TMA_STAGE_BYTES);
+      tma_bps = nb > 0 ? nb : 2;
+    }
+    const int64_t tiles = (cap + R - 1) / R;
+    int64_t gbk = (int64_t)h->sm_count * tma_bps;
+    gbk = std::max<int64_t>(1, std::min(gbk, tiles));
+    gather_tma_kernel<<<(unsigned)gbk, 32, smem, st>>>(a, R, (int)rb);
+    return cudaGetLastError();
+  }
+  int64_t blocks = (total + GATHER_THREADS * unroll - 1) / (GATHER_THREADS * unroll);
+  static int occ[2][3] = {{0, 0, 0}, {0, 0, 0}};
+  const int which = vb == 16 ? 0 : (vb == 4 ? 1 : 2);
+  const int ui = unroll == 8 ? 1 : 0;
+  if (!occ[ui][which]) {
+    int nb = 0;
+    if (unroll == 8) {
+      if (vb == 16) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<uint4, 8>, GATHER_THREADS, 0);
+      else if (vb == 4) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<unsigned, 8>, GATHER_THREADS, 0);
+      else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<unsigned short, 8>, GATHER_THREADS, 0);
+    } else {
+      if (vb == 16) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<uint4, 4>, GATHER_THREADS, 0);
+      else if (vb == 4) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<unsigned, 4>, GATHER_THREADS, 0);
+      else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<unsigned short, 4>, GATHER_THREADS, 0);
+    }
+    occ[ui][which] = nb > 0 ? nb : 4;
+  }
+  const int per_sm = (bps > 0 && bps < occ[ui][which]) ? bps : occ[ui][which];
+  const int64_t max_blocks = (int64_t)h->sm_count * per_sm;
   blocks = blocks < 1 ? 1 : (blocks > max_blocks ? max_blocks : blocks);
-  if (vb == 16)
-    gather_kernel<uint4><<<(unsigned)blocks, GATHER_THREADS, 0, st>>>(a);
-  else if (vb == 4)
-    gather_kernel<unsigned><<<(unsigned)blocks, GATHER_THREADS, 0, st>>>(a);
-  else
-    gather_kernel<unsigned short><<<(unsigned)blocks, GATHER_THREADS, 0, st>>>(a);
+  const unsigned gb = (unsigned)blocks;
+  if (unroll == 8) {
+    if (vb == 16) gather_kernel<uint4, 8><<<gb, GATHER_THREADS, 0, st>>>(a);
+    else if (vb == 4) gather_kernel<unsigned, 8><<<gb, GATHER_THREADS, 0, st>>>(a);
+    else gather_kernel<unsigned short, 8><<<gb, GATHER_THREADS, 0, st>>>(a);
+  } else {
+    if (vb == 16) gather_kernel<uint4, 4><<<gb, GATHER_THREADS, 0, st>>>(a);
+    else if (vb == 4) gather_kernel<unsigned, 4><<<gb, GATHER_THREADS, 0, st>>>(a);
+    else gather_kernel<unsigned short, 4><<<gb, GATHER_THREADS, 0, st>>>(a);
+  }
   return cudaGetLastError();
 }
 

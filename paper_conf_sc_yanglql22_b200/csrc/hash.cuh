@@ -63,4 +63,19 @@ __device__ __forceinline__ long long hash_insert_min(const HashTable& t, int64_t
   return slot;
 }
 
+// Target insert (position q < nT): returns the slot and sets *dup if another TARGET
+// with the same key was recorded first in this epoch (the returned old minimum is
+// then a target position).  Of two equal targets the later atomic always sees the
+// earlier one, so a duplicate target is always detected (reading A8).
+__device__ __forceinline__ long long hash_insert_target(const HashTable& t, int64_t key, int64_t q, int64_t nT,
+                                                        unsigned epoch, bool* dup) {
+  const long long slot = hash_insert(t, stored_key(epoch, key), epoch);
+  *dup = false;
+  if (slot >= 0) {
+    const unsigned long long old = atomicMin(&t.slots[slot].val, pack_pos(epoch, q));
+    *dup = (old >> 40) == (unsigned long long)(EPOCH_MAX - epoch) && (int64_t)(old & KEY_MASK) < nT;
+  }
+  return slot;
+}
+
 }  // namespace wg

@@ -11,11 +11,12 @@
 //   insert   every key; __match_any_sync elects one lane per distinct key in a warp;
 //            CAS claims a slot, atomicMin records the first position; every position
 //            remembers its slot (slot_of).
+//            It also copies the targets to U (targets first, L160) and detects
+//            duplicate targets from the atomicMin's old value (A8).
 //   flag     single-pass scan (block-wide decoupled look-back) over the neighbour
 //            positions: reads the min position through slot_of (one dependent L2
-//            read, no probing), writes U for first occurrences, the scan, and handles
-//            the targets (U[k] = T[k], duplicate-target check).  Its last block
-//            advances the table epoch.
+//            read, no probing), writes U for first occurrences and the scan.  Its last
+//            block advances the table epoch.
 //   relabel  sub_col[p] = id of nbrs[p]; optional duplicate counts (L186).  Nothing
 //            else in the batch reads it, so the fused hop runs it on a side stream.
 // PADDED = true is the fused hop: neighbours come from the sampler's padded slots
@@ -32,6 +33,8 @@ constexpr int UQ_THREADS = 256;
 constexpr int UQ_ITEMS = 8;
 constexpr int UQ_TILE = UQ_THREADS * UQ_ITEMS;  // neighbour positions per flag tile
 constexpr int CNT_BITS = 31;                    // packed scan value: (valid << 31) | first
+constexpr int32_t SLOT_EMPTY = -1;              // slot_of: padded slot without a sample
+constexpr int32_t SLOT_BADID = -2;              // slot_of: sample whose id is out of range
 
 struct UniqueArgs {
   const int64_t* T;
@@ -95,22 +98,40 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueA
         const int64_t j = q - nT;
         const int64_t k = j / a.M;
         valid = (int)(j - k * a.M) < a.cnt[k];
-        if (valid) key = a.nbrs[j];
+        if (valid)
+          key = a.nbrs[j];
+        else
+          a.slot_of[q] = SLOT_EMPTY;  // padding slot: no sample here
       } else {
         key = a.nbrs[q - nT];
       }
       if (valid && (key < 0 || key >= a.n)) {
         latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_ID_RANGE);
-        a.slot_of[q] = -1;
+        a.slot_of[q] = SLOT_BADID;  // a sample, but no key to number
         valid = false;
       }
     }
     const unsigned long long mk = valid ? (unsigned long long)key : (0x8000000000000000ull | (unsigned)lane);
     const unsigned same = __match_any_sync(FULL_MASK, mk);
     const int leader = __ffs(same) - 1;  // lowest lane = smallest position among equal keys
+    const bool is_target = q < nT;
+    if (is_target) {  // targets first, original order (L160)
+      a.U[q] = key;
+      if (a.dup) a.dup[q] = 0;
+    }
+    // two equal targets in this warp: duplicate target (A8)
+    const unsigned tmask = __ballot_sync(FULL_MASK, valid && is_target);
+    if (valid && is_target && leader == lane && __popc(same & tmask) > 1)
+      latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DUP_TARGET);
     long long slot = -1;
     if (valid && leader == lane) {
-      slot = hash_insert_min(a.ht, key, q, epoch);
+      if (is_target) {
+        bool dup = false;
+        slot = hash_insert_target(a.ht, key, q, nT, epoch, &dup);
+        if (dup) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DUP_TARGET);
+      } else {
+        slot = hash_insert_min(a.ht, key, q, epoch);
+      }
       if (slot < 0) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_CAPACITY);
     }
     slot = __shfl_sync(FULL_MASK, slot, leader);
@@ -133,14 +154,6 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArg
   const unsigned epoch = a.ctrl[CTRL_EPOCH];
   const int tid = threadIdx.x;
 
-  // targets: U[k] = T[k] (targets first, original order, L160); duplicate check (A8)
-  for (int64_t k = (int64_t)blockIdx.x * UQ_THREADS + tid; k < nT; k += (int64_t)gridDim.x * UQ_THREADS) {
-    a.U[k] = a.T[k];
-    if (a.dup) a.dup[k] = 0;
-    const int32_t slot = a.slot_of[k];
-    if (slot >= 0 && min_pos_at(a, slot) != k) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DUP_TARGET);
-  }
-
   const int64_t tile_start = (int64_t)blockIdx.x * UQ_TILE;
   if (nE == 0) {
     if (blockIdx.x == 0 && tid == 0) {
@@ -154,29 +167,42 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArg
     const int64_t j0 = tile_start + (int64_t)tid * UQ_ITEMS;
     int32_t slots[UQ_ITEMS];
     bool valid[UQ_ITEMS];
+    int64_t keys[UQ_ITEMS];
+    int32_t poss[UQ_ITEMS];
     int64_t k0 = 0;
     int i0 = 0;
     if (PADDED) {
       k0 = j0 / a.M;
       i0 = (int)(j0 - k0 * a.M);
-      int64_t k = k0;
-      int i = i0;
-      int c = k < nT ? a.cnt[k] : 0;
+    }
+    // every position's slot (the insert pass wrote SLOT_EMPTY for padding): no count read needed
+    const int32_t* sp = a.slot_of + nT + j0;
+    if (j0 + UQ_ITEMS <= nE && (nT & 3) == 0) {
+      const int4 s0 = *reinterpret_cast<const int4*>(sp);
+      const int4 s1 = *reinterpret_cast<const int4*>(sp + 4);
+      slots[0] = s0.x; slots[1] = s0.y; slots[2] = s0.z; slots[3] = s0.w;
+      slots[4] = s1.x; slots[5] = s1.y; slots[6] = s1.z; slots[7] = s1.w;
+    } else {
 #pragma unroll
-      for (int t = 0; t < UQ_ITEMS; ++t) {
-        valid[t] = (j0 + t < nE) && i < c;
-        if (++i == a.M) {
-          i = 0;
-          ++k;
-          c = (t + 1 < UQ_ITEMS && k < nT) ? a.cnt[k] : 0;
-        }
+      for (int t = 0; t < UQ_ITEMS; ++t) slots[t] = j0 + t < nE ? sp[t] : SLOT_EMPTY;
+    }
+    // the neighbour ids (and positions) are needed only after the scan: issue their loads now
+    if (j0 + UQ_ITEMS <= nE && ((uintptr_t)a.nbrs & 15) == 0) {
+#pragma unroll
+      for (int t = 0; t < UQ_ITEMS; t += 2) {
+        const longlong2 v2 = *reinterpret_cast<const longlong2*>(a.nbrs + j0 + t);
+        keys[t] = v2.x;
+        keys[t + 1] = v2.y;
       }
     } else {
 #pragma unroll
-      for (int t = 0; t < UQ_ITEMS; ++t) valid[t] = j0 + t < nE;
+      for (int t = 0; t < UQ_ITEMS; ++t) keys[t] = j0 + t < nE ? a.nbrs[j0 + t] : -1;
     }
 #pragma unroll
-    for (int t = 0; t < UQ_ITEMS; ++t) slots[t] = valid[t] ? a.slot_of[nT + j0 + t] : -1;
+    for (int t = 0; t < UQ_ITEMS; ++t) {
+      valid[t] = (j0 + t < nE) && (!PADDED || slots[t] != SLOT_EMPTY);
+      poss[t] = (PADDED && a.out_pos && valid[t]) ? a.pos_pad[j0 + t] : 0;
+    }
     int64_t mps[UQ_ITEMS];
 #pragma unroll
     for (int t = 0; t < UQ_ITEMS; ++t) mps[t] = min_pos_at(a, slots[t]);  // independent L2 reads
@@ -205,12 +231,12 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArg
         if (valid[t]) {
           const int64_t p = PADDED ? ev : j;
           if (PADDED) {
-            a.out_nbrs[p] = a.nbrs[j];
-            if (a.out_pos) a.out_pos[p] = a.pos_pad[j];
+            a.out_nbrs[p] = keys[t];
+            if (a.out_pos) a.out_pos[p] = poss[t];
           }
           a.sub_col[p] = (int32_t)mps[t];  // temporary: min position (relabel turns it into an id)
           if (first[t]) {
-            a.U[nT + ef] = a.nbrs[j];
+            a.U[nT + ef] = keys[t];
             if (a.dup) a.dup[nT + ef] = 0;
             a.excl[j] = (int32_t)ef;
           }

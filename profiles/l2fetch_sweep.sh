@@ -1,0 +1,10 @@
+#!/bin/bash
+mkdir -p gpurun_out
+timeout 900 python -m pytest tests -m gpu -q -x > gpurun_out/pytest_gpu.log 2>&1; echo pytest=$?; tail -3 gpurun_out/pytest_gpu.log
+for G in 0 32 64; do for P in 1 4; do
+WG_L2_FETCH=$G timeout 600 python bench.py --steps 50 --warmup 5 --cpu-sample-s 0 --concurrency $P > gpurun_out/bench_g${G}_p$P.log 2>&1
+python -c "import json;d=json.loads(open('gpurun_out/bench_g${G}_p$P.log').read().strip().splitlines()[-1]);print('L2fetch',$G,'P',$P,round(d['value']),round(d['ms_per_step'],4),round(d['single_batch']['ms_per_batch'],4),round(d['roofline']['frac'],3),round(d['roofline']['gather_ms_per_launch'],4))"
+done; done
+WG_L2_FETCH=32 timeout 300 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv --log-file gpurun_out/launches_g32.csv python bench.py --steps 2 --warmup 3 --cpu-sample-s 0 --e2e-steps 1 --concurrency 1 > /dev/null 2>&1
+timeout 300 ncu --metrics gpu__time_duration.sum,dram__bytes_read.sum,dram__bytes_write.sum --clock-control none --csv --log-file gpurun_out/launches_g0.csv python bench.py --steps 2 --warmup 3 --cpu-sample-s 0 --e2e-steps 1 --concurrency 1 > /dev/null 2>&1
+echo done

@@ -213,3 +213,35 @@ def test_fork_concurrent_streams(tiny):
         dsm.destroy()            # forks first
     child.destroy()
     dsm.destroy()
+
+
+def test_gather_tma_variant_subprocess():
+    """The TMA bulk-copy gather (WG_GATHER_TMA=1, chosen once per process) is bit-exact too."""
+    import os
+    import subprocess
+    import sys
+    code = r'''
+import sys, numpy as np, torch
+sys.path.insert(0, "tests")
+from gpu_helpers import make_dsm
+import oracle
+from synth import features, presets
+for dim, dtype in ((100, "fp32"), (4, "fp32"), (768, "fp16"), (1024, "fp32"), (3, "fp32")):
+    n = 5000
+    rp = np.zeros(n + 1, dtype=np.int64)
+    feat = features.feature_bytes(presets.FEAT_SEED, np.arange(n), dim, dtype)
+    dsm = make_dsm(rp, np.zeros(0, np.int64), feat, dim, dtype)
+    rng = np.random.default_rng(dim)
+    for ids in (rng.integers(0, n, 7777), np.arange(n)[::-1], np.full(33, 7), np.zeros(0)):
+        ids = np.ascontiguousarray(ids, dtype=np.int64)
+        X = dsm.gather(torch.from_numpy(ids).cuda())
+        torch.cuda.synchronize()
+        assert np.array_equal(X[:len(ids)].cpu().numpy(), oracle.gather(feat, np.arange(n), ids)), (dim, dtype)
+    assert dsm.device_error() == 0
+    dsm.destroy()
+print("TMA OK")
+'''
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", code], cwd=root, env=dict(os.environ, WG_GATHER_TMA="1"),
+                       capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0 and "TMA OK" in r.stdout, r.stdout + r.stderr
