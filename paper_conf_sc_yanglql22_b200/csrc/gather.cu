@@ -20,24 +20,6 @@ namespace wg {
 
 constexpr int GATHER_THREADS = 256;
 
-// n / d for n < 2^31 via multiply-high (Granlund-Montgomery; d >= 1).
-struct FastDiv {
-  unsigned d, mul, shift;
-  __host__ explicit FastDiv(unsigned d_) : d(d_) {
-    shift = 0;
-    while ((1u << shift) < d) ++shift;
-    unsigned long long m = ((1ull << (32 + shift)) + d - 1) / d;
-    mul = (unsigned)m;  // the implicit bit 2^32 is added back in div()
-    if (d == 1) { mul = 0; shift = 0; }
-  }
-  __device__ __forceinline__ unsigned div(unsigned n) const {
-    if (d == 1) return n;
-    // q = floor((n * (2^32 + mul)) / 2^(32+shift)) computed without overflow
-    const unsigned t = __umulhi(n, mul);
-    return (unsigned)(((unsigned long long)t + n) >> shift);
-  }
-};
-
 template <typename V>
 __device__ __forceinline__ V ld_feat(const void* p);
 template <>

@@ -29,9 +29,10 @@
 namespace wg {
 
 constexpr int SAMPLE_THREADS = 256;
-constexpr int SAMPLE_UNR = 4;  // rounds per warp, all in flight at once
-template <int G>
-constexpr int sample_tile() { return (SAMPLE_THREADS / G) * SAMPLE_UNR; }  // 128 / 64 / 32 targets per block
+// SAMPLE_UNR = rounds per warp, all in flight at once (1, 2 or 4; chosen per launch: small hops use
+// fewer rounds per warp and therefore more blocks / SMs)
+template <int G, int SAMPLE_UNR>
+constexpr int sample_tile() { return (SAMPLE_THREADS / G) * SAMPLE_UNR; }  // targets per block
 
 struct SampleArgs {
   ShardView s;
@@ -48,7 +49,7 @@ struct SampleArgs {
   unsigned* ctrl;
 };
 
-template <int G>
+template <int G, int SAMPLE_UNR>
 __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs a) {
   __shared__ unsigned sm_chain[SAMPLE_THREADS / 32][32];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -231,14 +232,20 @@ cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap,
   a.pos_pad = want_pos ? h->ws.pos_pad : nullptr;
   a.cnt = h->ws.cnt;
   a.ctrl = h->ws.ctrl;
-  const int tile = fanout <= 8 ? sample_tile<8>() : fanout <= 16 ? sample_tile<16>() : sample_tile<32>();
+  const int G = fanout <= 8 ? 8 : fanout <= 16 ? 16 : 32;
+  int unr = 4;  // largest of 4/2/1 that still gives >= 2 blocks per SM
+  while (unr > 1 && cap < (int64_t)(SAMPLE_THREADS / G) * unr * 2 * h->sm_count) unr >>= 1;
+  const int tile = (SAMPLE_THREADS / G) * unr;
   const unsigned blocks = (unsigned)(cap > 0 ? (cap + tile - 1) / tile : 1);
-  if (fanout <= 8)
-    sample_kernel<8><<<blocks, SAMPLE_THREADS, 0, st>>>(a);
-  else if (fanout <= 16)
-    sample_kernel<16><<<blocks, SAMPLE_THREADS, 0, st>>>(a);
-  else
-    sample_kernel<32><<<blocks, SAMPLE_THREADS, 0, st>>>(a);
+#define WG_SAMPLE_LAUNCH(GG, UU) sample_kernel<GG, UU><<<blocks, SAMPLE_THREADS, 0, st>>>(a)
+  if (G == 8) {
+    if (unr == 4) WG_SAMPLE_LAUNCH(8, 4); else if (unr == 2) WG_SAMPLE_LAUNCH(8, 2); else WG_SAMPLE_LAUNCH(8, 1);
+  } else if (G == 16) {
+    if (unr == 4) WG_SAMPLE_LAUNCH(16, 4); else if (unr == 2) WG_SAMPLE_LAUNCH(16, 2); else WG_SAMPLE_LAUNCH(16, 1);
+  } else {
+    if (unr == 4) WG_SAMPLE_LAUNCH(32, 4); else if (unr == 2) WG_SAMPLE_LAUNCH(32, 2); else WG_SAMPLE_LAUNCH(32, 1);
+  }
+#undef WG_SAMPLE_LAUNCH
   return cudaGetLastError();
 }
 

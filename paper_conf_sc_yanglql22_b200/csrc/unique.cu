@@ -30,8 +30,8 @@
 namespace wg {
 
 constexpr int UQ_THREADS = 256;
-constexpr int UQ_ITEMS = 8;
-constexpr int UQ_TILE = UQ_THREADS * UQ_ITEMS;  // neighbour positions per flag tile
+// neighbour positions per thread of the flag scan: 1..8, chosen per launch so that small hops
+// spread over many SMs (latency-bound) and large hops keep several loads in flight per thread
 constexpr int CNT_BITS = 31;                    // packed scan value: (valid << 31) | first
 constexpr int32_t SLOT_EMPTY = -1;              // slot_of: padded slot without a sample
 constexpr int32_t SLOT_BADID = -2;              // slot_of: sample whose id is out of range
@@ -44,6 +44,7 @@ struct UniqueArgs {
   int64_t capE;            // dense capacity (standalone) or capT * M (PADDED)
   const int64_t* d_nE;     // dense count (standalone) or NULL (PADDED)
   int M;                   // PADDED: fanout
+  FastDiv Mdiv;            // PADDED: division by M
   const int32_t* cnt;      // PADDED: per-target sample counts
   const int32_t* pos_pad;  // PADDED: adjacency positions of the padded slots (nullable)
   int64_t* out_row_ptr;    // PADDED: dense CSR row pointer [nT+1]
@@ -144,15 +145,20 @@ __device__ __forceinline__ int64_t min_pos_at(const UniqueArgs& a, int32_t slot)
   return (int64_t)(a.ht.slots[slot].val & KEY_MASK);
 }
 
-template <bool PADDED>
+template <bool PADDED, int UQ_ITEMS>
 __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArgs a) {
+  // warp-striped: warp w of the tile covers 32 * UQ_ITEMS consecutive positions, lane l the
+  // positions l, l+32, ...; every load and store instruction touches 32 consecutive elements,
+  // and the in-warp scans are ballots + popc.
+  constexpr int UQ_TILE = UQ_THREADS * UQ_ITEMS;
   __shared__ LookbackSmem<UQ_THREADS> lb;
   __shared__ unsigned long long sm_wtot[UQ_THREADS / 32 + 1];
   __shared__ int sm_flag;
   int64_t nT, nE;
   load_counts<PADDED>(a, nT, nE);
   const unsigned epoch = a.ctrl[CTRL_EPOCH];
-  const int tid = threadIdx.x;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const unsigned lt = (1u << lane) - 1u;
 
   const int64_t tile_start = (int64_t)blockIdx.x * UQ_TILE;
   if (nE == 0) {
@@ -164,97 +170,76 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArg
       }
     }
   } else if (tile_start < nE) {
-    const int64_t j0 = tile_start + (int64_t)tid * UQ_ITEMS;
+    const int64_t wbase = tile_start + (int64_t)warp * 32 * UQ_ITEMS + lane;
     int32_t slots[UQ_ITEMS];
-    bool valid[UQ_ITEMS];
     int64_t keys[UQ_ITEMS];
     int32_t poss[UQ_ITEMS];
-    int64_t k0 = 0;
-    int i0 = 0;
-    if (PADDED) {
-      k0 = j0 / a.M;
-      i0 = (int)(j0 - k0 * a.M);
-    }
-    // every position's slot (the insert pass wrote SLOT_EMPTY for padding): no count read needed
-    const int32_t* sp = a.slot_of + nT + j0;
-    if (j0 + UQ_ITEMS <= nE && (nT & 3) == 0) {
-      const int4 s0 = *reinterpret_cast<const int4*>(sp);
-      const int4 s1 = *reinterpret_cast<const int4*>(sp + 4);
-      slots[0] = s0.x; slots[1] = s0.y; slots[2] = s0.z; slots[3] = s0.w;
-      slots[4] = s1.x; slots[5] = s1.y; slots[6] = s1.z; slots[7] = s1.w;
-    } else {
-#pragma unroll
-      for (int t = 0; t < UQ_ITEMS; ++t) slots[t] = j0 + t < nE ? sp[t] : SLOT_EMPTY;
-    }
-    // the neighbour ids (and positions) are needed only after the scan: issue their loads now
-    if (j0 + UQ_ITEMS <= nE && ((uintptr_t)a.nbrs & 15) == 0) {
-#pragma unroll
-      for (int t = 0; t < UQ_ITEMS; t += 2) {
-        const longlong2 v2 = *reinterpret_cast<const longlong2*>(a.nbrs + j0 + t);
-        keys[t] = v2.x;
-        keys[t + 1] = v2.y;
-      }
-    } else {
-#pragma unroll
-      for (int t = 0; t < UQ_ITEMS; ++t) keys[t] = j0 + t < nE ? a.nbrs[j0 + t] : -1;
-    }
-#pragma unroll
-    for (int t = 0; t < UQ_ITEMS; ++t) {
-      valid[t] = (j0 + t < nE) && (!PADDED || slots[t] != SLOT_EMPTY);
-      poss[t] = (PADDED && a.out_pos && valid[t]) ? a.pos_pad[j0 + t] : 0;
-    }
     int64_t mps[UQ_ITEMS];
-#pragma unroll
-    for (int t = 0; t < UQ_ITEMS; ++t) mps[t] = min_pos_at(a, slots[t]);  // independent L2 reads
-    unsigned long long nv = 0, nf = 0;
-    bool first[UQ_ITEMS];
+    unsigned vm[UQ_ITEMS], fm[UQ_ITEMS];
 #pragma unroll
     for (int t = 0; t < UQ_ITEMS; ++t) {
-      first[t] = valid[t] && mps[t] == nT + j0 + t;
-      nv += valid[t];
-      nf += first[t];
+      const int64_t j = wbase + 32 * t;
+      const bool in = j < nE;
+      // every position's slot (the insert pass wrote SLOT_EMPTY for padding): no count read needed
+      slots[t] = in ? a.slot_of[nT + j] : SLOT_EMPTY;
+      keys[t] = in ? a.nbrs[j] : -1;  // needed only after the scan: issued now
+    }
+    unsigned long long wv = 0, wf = 0;
+#pragma unroll
+    for (int t = 0; t < UQ_ITEMS; ++t) {
+      const int64_t j = wbase + 32 * t;
+      const bool valid = j < nE && (!PADDED || slots[t] != SLOT_EMPTY);
+      poss[t] = (PADDED && a.out_pos && valid) ? a.pos_pad[j] : 0;
+      mps[t] = min_pos_at(a, slots[t]);  // independent L2 reads
+      vm[t] = __ballot_sync(FULL_MASK, valid);
+    }
+#pragma unroll
+    for (int t = 0; t < UQ_ITEMS; ++t) {
+      const int64_t j = wbase + 32 * t;
+      fm[t] = __ballot_sync(FULL_MASK, ((vm[t] >> lane) & 1u) && mps[t] == nT + j);
+      wv += __popc(vm[t]);
+      wf += __popc(fm[t]);
     }
     unsigned long long agg;
-    const unsigned long long ex =
-        block_exclusive_sum<UQ_THREADS>((nv << CNT_BITS) | nf, sm_wtot, &agg);
+    unsigned long long ex =
+        block_exclusive_sum<UQ_THREADS>(lane == 0 ? ((wv << CNT_BITS) | wf) : 0ull, sm_wtot, &agg);
+    ex = __shfl_sync(FULL_MASK, ex, 0);  // this warp's offset inside the tile
     const unsigned long long pre = block_lookback<UQ_THREADS>(a.status, (long)blockIdx.x, agg, lb);
     const unsigned long long base = pre + ex;
-    int64_t ev = (int64_t)(base >> CNT_BITS);                   // dense position of the next valid slot
-    int64_t ef = (int64_t)(base & ((1ull << CNT_BITS) - 1));    // next new-node index
-    int64_t k = k0;
-    int i = i0;
+    int64_t ev = (int64_t)(base >> CNT_BITS);                 // dense position of this warp's next valid slot
+    int64_t ef = (int64_t)(base & ((1ull << CNT_BITS) - 1));  // next new-node index
 #pragma unroll
     for (int t = 0; t < UQ_ITEMS; ++t) {
-      const int64_t j = j0 + t;
-      if (j < nE) {
-        if (PADDED && i == 0) a.out_row_ptr[k] = ev;
-        if (valid[t]) {
-          const int64_t p = PADDED ? ev : j;
-          if (PADDED) {
-            a.out_nbrs[p] = keys[t];
-            if (a.out_pos) a.out_pos[p] = poss[t];
-          }
-          a.sub_col[p] = (int32_t)mps[t];  // temporary: min position (relabel turns it into an id)
-          if (first[t]) {
-            a.U[nT + ef] = keys[t];
-            if (a.dup) a.dup[nT + ef] = 0;
-            a.excl[j] = (int32_t)ef;
-          }
-          ev += 1;
-          ef += first[t];
+      const int64_t j = wbase + 32 * t;
+      const bool valid = (vm[t] >> lane) & 1u;
+      const bool first = (fm[t] >> lane) & 1u;
+      const int64_t p = PADDED ? ev + __popc(vm[t] & lt) : j;
+      const int64_t f = ef + __popc(fm[t] & lt);
+      if (PADDED && j < nE) {
+        const unsigned k = a.Mdiv.div((unsigned)j);
+        if ((unsigned)j == k * (unsigned)a.M) a.out_row_ptr[k] = p;  // first slot of target k
+      }
+      if (valid) {
+        if (PADDED) {
+          a.out_nbrs[p] = keys[t];
+          if (a.out_pos) a.out_pos[p] = poss[t];
         }
-        if (j == nE - 1) {
-          if (a.d_nU) *a.d_nU = nT + ef;
-          if (PADDED) {
-            a.out_row_ptr[nT] = ev;
-            if (a.d_num_edges) *a.d_num_edges = ev;
-          }
+        a.sub_col[p] = (int32_t)mps[t];  // temporary: min position (relabel turns it into an id)
+      }
+      if (first) {
+        a.U[nT + f] = keys[t];
+        if (a.dup) a.dup[nT + f] = 0;
+        a.excl[j] = (int32_t)f;
+      }
+      if (j == nE - 1) {
+        if (a.d_nU) *a.d_nU = nT + f + first;
+        if (PADDED) {
+          a.out_row_ptr[nT] = p + valid;
+          if (a.d_num_edges) *a.d_num_edges = p + valid;
         }
       }
-      if (PADDED && ++i == a.M) {
-        i = 0;
-        ++k;
-      }
+      ev += __popc(vm[t]);
+      ef += __popc(fm[t]);
     }
   }
 
@@ -297,13 +282,27 @@ static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, c
   const int64_t max_blocks = (int64_t)h->sm_count * 8;
   int64_t ib = (total + UQ_THREADS - 1) / UQ_THREADS;
   ib = ib < 1 ? 1 : (ib > max_blocks ? max_blocks : ib);
-  const unsigned fb = (unsigned)(a.capE > 0 ? (a.capE + UQ_TILE - 1) / UQ_TILE : 1);
+  // items per thread: the largest of 8/4/2/1 that still gives >= 2 tiles per SM
+  int items = 8;
+  while (items > 1 && a.capE < (int64_t)items * UQ_THREADS * 2 * h->sm_count) items >>= 1;
+  const int64_t tile = (int64_t)items * UQ_THREADS;
+  const unsigned fb = (unsigned)(a.capE > 0 ? (a.capE + tile - 1) / tile : 1);
   if (padded) {
     unique_insert_kernel<true><<<(unsigned)ib, UQ_THREADS, 0, st>>>(a);
-    unique_flag_kernel<true><<<fb, UQ_THREADS, 0, st>>>(a);
+    switch (items) {
+      case 8: unique_flag_kernel<true, 8><<<fb, UQ_THREADS, 0, st>>>(a); break;
+      case 4: unique_flag_kernel<true, 4><<<fb, UQ_THREADS, 0, st>>>(a); break;
+      case 2: unique_flag_kernel<true, 2><<<fb, UQ_THREADS, 0, st>>>(a); break;
+      default: unique_flag_kernel<true, 1><<<fb, UQ_THREADS, 0, st>>>(a); break;
+    }
   } else {
     unique_insert_kernel<false><<<(unsigned)ib, UQ_THREADS, 0, st>>>(a);
-    unique_flag_kernel<false><<<fb, UQ_THREADS, 0, st>>>(a);
+    switch (items) {
+      case 8: unique_flag_kernel<false, 8><<<fb, UQ_THREADS, 0, st>>>(a); break;
+      case 4: unique_flag_kernel<false, 4><<<fb, UQ_THREADS, 0, st>>>(a); break;
+      case 2: unique_flag_kernel<false, 2><<<fb, UQ_THREADS, 0, st>>>(a); break;
+      default: unique_flag_kernel<false, 1><<<fb, UQ_THREADS, 0, st>>>(a); break;
+    }
   }
   if (a.capE > 0) {
     // relabel runs over the DENSE neighbours: count = num_edges (padded) or d_nE
@@ -335,6 +334,7 @@ cudaError_t launch_append_unique(wg_dsm* h, const int64_t* T, int64_t capT, cons
   a.capE = capE;
   a.d_nE = d_nE;
   a.M = 1;
+  a.Mdiv = FastDiv(1u);
   a.U = U;
   a.d_nU = d_nU;
   a.sub_col = sub_col;
@@ -359,6 +359,7 @@ cudaError_t launch_hop(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t*
   a.capE = capT * fanout;
   a.d_nE = nullptr;
   a.M = fanout;
+  a.Mdiv = FastDiv((unsigned)fanout);
   a.cnt = h->ws.cnt;
   a.pos_pad = h->ws.pos_pad;
   a.out_row_ptr = out_row_ptr;
