@@ -74,8 +74,11 @@ static void free_workspace(wg_dsm* h) {
 static wg_status alloc_workspace(wg_dsm* h, int64_t max_keys) {
   Workspace& w = h->ws;
   if (max_keys < 1) max_keys = 1;
+  // Load factor <= 1/4 at the capacity bound (~0.07 for typical batches): a warp inserts up to 32
+  // keys at once and waits for its LONGEST linear probe, so short probe tails matter more than
+  // table size (only touched slots occupy L2).
   int64_t cap = 1024;
-  while (cap < max_keys + max_keys / 2) cap <<= 1;  // worst-case load <= 2/3 (typical batches: ~0.3)
+  while (cap < 4 * max_keys) cap <<= 1;
   w.hcap = cap;
   w.max_keys = max_keys;
   w.status_cap = max_keys / 32 + 2;  // sampler tiles hold >= 32 targets, flag tiles 1024 positions

@@ -5,7 +5,7 @@
 // sector): key = (epoch << 40) | node id, val = ((EPOCH_MAX - epoch) << 40) | first
 // position.  A key from an older epoch reads as an empty slot and an older
 // value always loses an atomicMin against the current epoch, so the table is never
-// cleared between calls.  Linear probing, fmix64 hash, worst-case load <= 2/3.
+// cleared between calls.  Linear probing, fmix64 hash, load factor <= 1/4.
 #pragma once
 
 #include "device_util.cuh"
@@ -29,15 +29,29 @@ __device__ __forceinline__ unsigned long long pack_pos(unsigned epoch, int64_t q
 }
 
 // Returns the slot holding `stored` (claiming an empty one if needed), or -1 if full.
-__device__ __forceinline__ long long hash_insert(const HashTable& t, unsigned long long stored, unsigned epoch) {
+// *seen receives the slot's value as read together with its key (one 16 B load) when the
+// key was already present, or ~0 when this call claimed the slot.
+__device__ __forceinline__ long long hash_insert(const HashTable& t, unsigned long long stored, unsigned epoch,
+                                                 unsigned long long* seen) {
   unsigned long long slot = fmix64(stored & KEY_MASK) & t.mask;
   for (unsigned long long probe = 0; probe <= t.mask; ++probe) {
-    unsigned long long cur = ld_volatile_u64(&t.slots[slot].key);
+    unsigned long long cur, val;
+    asm volatile("ld.volatile.global.v2.u64 {%0, %1}, [%2];" : "=l"(cur), "=l"(val) : "l"(&t.slots[slot]));
     for (;;) {
-      if (cur == stored) return (long long)slot;
+      if (cur == stored) {
+        *seen = val;
+        return (long long)slot;
+      }
       if ((unsigned)(cur >> 40) == epoch) break;  // occupied by another key this epoch
       const unsigned long long prev = atomicCAS(&t.slots[slot].key, cur, stored);
-      if (prev == cur || prev == stored) return (long long)slot;
+      if (prev == cur) {
+        *seen = ~0ull;
+        return (long long)slot;
+      }
+      if (prev == stored) {
+        *seen = ~0ull;  // claimed by another thread a moment ago: its minimum may not be there yet
+        return (long long)slot;
+      }
       cur = prev;
     }
     slot = (slot + 1) & t.mask;
@@ -57,9 +71,14 @@ __device__ __forceinline__ long long hash_find(const HashTable& t, unsigned long
 }
 
 // Insert `key` at position q, recording the minimum position.  Returns the slot or -1.
+// The atomicMin is skipped when the value read with the key already holds a smaller
+// position of this epoch: hub ids occur thousands of times per hop, and this removes
+// most of the same-address atomics they would otherwise serialise on.
 __device__ __forceinline__ long long hash_insert_min(const HashTable& t, int64_t key, int64_t q, unsigned epoch) {
-  const long long slot = hash_insert(t, stored_key(epoch, key), epoch);
-  if (slot >= 0) atomicMin(&t.slots[slot].val, pack_pos(epoch, q));
+  unsigned long long seen;
+  const long long slot = hash_insert(t, stored_key(epoch, key), epoch, &seen);
+  const unsigned long long mine = pack_pos(epoch, q);
+  if (slot >= 0 && seen > mine) atomicMin(&t.slots[slot].val, mine);
   return slot;
 }
 
@@ -69,7 +88,8 @@ __device__ __forceinline__ long long hash_insert_min(const HashTable& t, int64_t
 // earlier one, so a duplicate target is always detected (reading A8).
 __device__ __forceinline__ long long hash_insert_target(const HashTable& t, int64_t key, int64_t q, int64_t nT,
                                                         unsigned epoch, bool* dup) {
-  const long long slot = hash_insert(t, stored_key(epoch, key), epoch);
+  unsigned long long seen;
+  const long long slot = hash_insert(t, stored_key(epoch, key), epoch, &seen);
   *dup = false;
   if (slot >= 0) {
     const unsigned long long old = atomicMin(&t.slots[slot].val, pack_pos(epoch, q));

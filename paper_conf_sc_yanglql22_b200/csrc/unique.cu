@@ -24,6 +24,11 @@
 // dense ones), and the flag pass scans "valid" and "first" together -- it also emits
 // the sampler's dense CSR (row_ptr, neighbours, positions), so no separate compaction
 // pass is needed.
+#include <climits>
+#include <cstdlib>
+
+#include <algorithm>
+
 #include "hash.cuh"
 #include "scan.cuh"
 
