@@ -40,6 +40,9 @@ def parse():
     ap.add_argument("--e2e-steps", type=int, default=20)
     ap.add_argument("--concurrency", type=int, default=4, help="independent batches in flight per GPU (streams)")
     ap.add_argument("--out", default=None, help="also append the JSON line to this file")
+    ap.add_argument("--sweep", action="store_true", help="config 4: feature-gather sweep over row sizes")
+    ap.add_argument("--sweep-rows", type=int, default=100_000_000)
+    ap.add_argument("--sweep-ids", type=int, default=1_000_000)
     return ap.parse_args()
 
 
@@ -418,9 +421,75 @@ def gather_traffic():
     return d.get("dram_bytes_per_launch")
 
 
+def bench_sweep(args):
+    """Config 4 (BASELINE.json configs[3]): feature-gather sweep over row sizes on a
+    100M-row table (the paper's Fig. 8 random-segment experiment, L240/L266): 1M
+    uniform random ids per rank, dims 64..1024 x fp16/fp32.  Cells whose table does not
+    fit one GPU are reported as skipped (they need W >= 2)."""
+    import torch
+
+    import paper_conf_sc_yanglql22_b200 as pkg
+    from synth import features as sfeat
+    from synth import gpu as sgpu
+    from synth import presets, seeds
+    torch.cuda.set_device(0)
+    dev = torch.device("cuda", 0)
+    n = args.sweep_rows
+    R = args.sweep_ids
+    peak, peak_src = peaks()
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    ids = torch.from_numpy(seeds.gather_ids(n, R, presets.SEED_BASE, 0)).to(dev)
+    cells = []
+    for dtype in ("fp16", "fp32"):
+        for dim in (64, 128, 256, 512, 768, 1024):
+            rb = dim * sfeat.elt_bytes(dtype)
+            pitch = (rb + 63) // 64 * 64
+            need = n * pitch + n * 8 + R * rb
+            free, _ = torch.cuda.mem_get_info()
+            if need > 0.9 * free:
+                cells.append({"dtype": dtype, "dim": dim, "row_bytes": rb, "skipped": f"table {n * pitch / 1e9:.0f} GB "
+                              "does not fit one GPU (needs W >= 2)"})
+                continue
+            dsm = pkg.DSM(n, 0, dim, dtype, 1, device=0)
+            _, _, fv = dsm.local_view()
+            sgpu.fill_features_gpu(fv, presets.FEAT_SEED, 0, 1, dim, sfeat.WG_DTYPE_CODE[dtype])
+            out = torch.empty((R, rb), dtype=torch.uint8, device=dev)
+            for _ in range(3):
+                dsm.gather(ids, out=out)
+            torch.cuda.synchronize()
+            ts = []
+            for i in range(args.steps):
+                flush.fill_(i & 0xFF)
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                dsm.gather(ids, out=out)
+                e1.record()
+                torch.cuda.synchronize()
+                ts.append(e0.elapsed_time(e1) / 1e3)
+            assert dsm.device_error() == 0
+            t = statistics.median(ts)
+            algo = R * rb / t / 1e9
+            cells.append({"dtype": dtype, "dim": dim, "row_bytes": rb, "ms": t * 1e3, "algo_gbs": algo,
+                          "hbm_gbs_read_plus_write": 2 * algo, "frac_of_hbm_roofline": 2 * algo / peak})
+            del out, fv
+            dsm.destroy()
+            torch.cuda.empty_cache()
+    best = max((c for c in cells if "ms" in c), key=lambda c: c["frac_of_hbm_roofline"])
+    line = {"metric": "feature gather GB/s vs HBM roofline (config 4 sweep, W=1)", "value": best["hbm_gbs_read_plus_write"],
+            "unit": "GB/s", "n_gpus": 1, "steps": args.steps, "warmup": 3, "higher_is_better": True,
+            "config": {"workload": "gather-sweep", "rows": n, "ids_per_rank": R, "ids": "uniform with replacement",
+                       "l2": "flushed between gathers"},
+            "roofline": {"bound": "hbm", "peak": peak, "unit": "GB/s", "peak_source": peak_src,
+                         "frac": best["frac_of_hbm_roofline"]},
+            "cells": cells}
+    emit(line, args)
+
+
 def main():
     args = parse()
-    if args.impl == "reference":
+    if args.sweep:
+        bench_sweep(args)
+    elif args.impl == "reference":
         bench_reference(args)
     else:
         bench_wg(args)

@@ -38,6 +38,8 @@ def build_dsm(preset, rank=0, world=1, device=None, allgather=None, max_seeds=No
         g_rp, g_col = sgraph.csr(spec)
         e_local = local_num_edges(g_rp, rank, world)
     info["gen_s"] = time.perf_counter() - t0
+    if on_device:
+        torch.cuda.empty_cache()  # return the generator's temporaries to the driver before the big slab
     t1 = time.perf_counter()
     dsm = DSM(spec.n, e_local, fd, fdt, keys, rank=rank, world_size=world, device=device.index, allgather=allgather)
     torch.cuda.synchronize(device)

@@ -61,3 +61,32 @@ def test_products_batches_bit_exact(products):
                 assert np.array_equal(got[k], exp[k]), (b, h, k)
         assert np.array_equal(pipe.features(), ref["X"])
     assert dsm.device_error() == 0
+
+
+@pytest.mark.slow
+def test_papers100m_shaped_batch_bit_exact():
+    """configs[2] shape on ONE GPU (111M nodes, ~3.2B CSR entries, 128 x fp32 = 57 GB of
+    features; 83 GB of shards): one whole [15,10,5] batch of 1024 seeds, every array
+    compared with the oracle (rows regenerated on the host for the touched nodes)."""
+    p = presets.get("papers100m")
+    free, _ = torch.cuda.mem_get_info()
+    if free < 150e9:
+        pytest.skip("needs a whole B200")
+    dsm, info = loader.build_dsm(p, on_device=True)
+    try:
+        rp, col, _ = dsm.local_view()
+        assert abs(int(rp[-1].item()) - p.target_e) / p.target_e < 0.03
+        pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
+        S = seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 7)
+        rs = seeds.rng_seed(presets.RNG_BASE, 7)
+        pipe.run(torch.from_numpy(S).cuda(), rs)
+        torch.cuda.synchronize()
+        ref = oracle.minibatch(loader.host_row_provider(p.graph()), loader.host_feat_provider(p), S, p.fanouts, rs)
+        for h in range(len(p.fanouts)):
+            got, exp = pipe.result(h), ref["hops"][h]
+            for k in ("row_ptr", "nbrs", "pos", "unique", "sub_col", "dup"):
+                assert np.array_equal(got[k], exp[k]), (h, k)
+        assert np.array_equal(pipe.features(), ref["X"])
+        assert dsm.device_error() == 0
+    finally:
+        dsm.destroy()
