@@ -190,12 +190,21 @@ def bench_wg(args):
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    ndev = torch.cuda.device_count()
+    torch.cuda.set_device(local % ndev)
+    dev = torch.device("cuda", local % ndev)
     ag = None
+    backend = None
     if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
+        # one rank per GPU over NCCL; if ranks share a GPU (a test box with fewer GPUs than ranks)
+        # NCCL refuses, so the setup-time handle exchange falls back to gloo (never on the hot path)
+        backend = "nccl" if ndev >= int(os.environ.get("LOCAL_WORLD_SIZE", world)) else "gloo"
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
         ag = pkg.TorchDistAllgather(device=dev)
+    local = local % ndev
     p = presets.get(args.config)
     S = p.seeds_per_batch
     P = max(1, args.concurrency)
@@ -273,7 +282,8 @@ def bench_wg(args):
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize()
-    clocks.start()
+    if rank == 0 or world == 1:
+        clocks.start()
     wall0 = time.perf_counter()
     for i in range(args.steps):
         k = args.warmup + i
@@ -319,7 +329,7 @@ def bench_wg(args):
     def max_over_ranks(x):
         if world == 1:
             return x
-        t = torch.tensor([x], dtype=torch.float64, device=dev)
+        t = torch.tensor([x], dtype=torch.float64, device=dev if backend == "nccl" else "cpu")
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
     dev_s_single = max_over_ranks(sum(step_ms) / 1e3)
@@ -330,13 +340,20 @@ def bench_wg(args):
     rows = rows_gathered.cpu().numpy()
     hc = hop_counts.cpu().numpy()
     gather_s = sum(gather_ms) / 1e3
-    alg_bytes = float(2 * rows.sum() * rb)           # read + write per gathered row (W=1: all local HBM)
+    # roofline of the gather: t_roof = max(2RB / HBM, (W-1)/W * RB / NVLink); at W=1 every
+    # byte is local HBM (read + write); at W>1 the (W-1)/W remote share crosses NVLink (770 GB/s measured
+    # peer bandwidth per direction, B200_PROFILING.md; 900 nominal) and bounds the kernel.
     peak, peak_src = peaks()
+    hbm_bytes = float(2 * rows.sum() * rb)
+    nvl_bytes = float((world - 1) / world * rows.sum() * rb)
+    t_hbm = hbm_bytes / (peak * 1e9)
+    t_nvl = nvl_bytes / 770e9
+    if t_nvl > t_hbm:
+        bound, alg_bytes, peak_used, peak_src_used = "nvlink", nvl_bytes, 770.0, \
+            "measured peer copy BW per direction (B200_PROFILING.md; 900 nominal)"
+    else:
+        bound, alg_bytes, peak_used, peak_src_used = "hbm", hbm_bytes, peak, peak_src
     achieved = alg_bytes / gather_s / 1e9
-    bound = "hbm"
-    if world > 1:
-        remote = (world - 1) / world
-        bound = "nvlink" if remote * rows.mean() * rb / 770e9 > 2 * rows.mean() * rb / (peak * 1e9) else "hbm"
 
     # ---- e2e through the public API with pinned host buffers (H2D seeds, D2H counts)
     e2e_times = []
@@ -379,9 +396,10 @@ def bench_wg(args):
             "config": cfg,
             "single_batch": {"value": value_single, "unit": UNIT, "ms_per_batch": 1e3 * dev_s_single / args.steps,
                              "ms_per_batch_median": statistics.median(step_ms)},
-            "roofline": {"kernel": "wg::gather_kernel", "bound": bound, "achieved": achieved, "peak": peak,
-                         "unit": "GB/s", "frac": achieved / peak, "traffic": gather_traffic(),
-                         "peak_source": peak_src,
+            "roofline": {"kernel": "wg::gather_kernel", "bound": bound, "achieved": achieved, "peak": peak_used,
+                         "unit": "GB/s", "frac": achieved / peak_used,
+                         "traffic": gather_traffic() if world == 1 else None,
+                         "peak_source": peak_src_used,
                          "algorithmic_bytes_per_launch": alg_bytes / args.steps,
                          "gather_ms_per_launch": 1e3 * gather_s / args.steps,
                          "gather_share_of_single_batch": gather_s / (sum(step_ms) / 1e3),
