@@ -24,6 +24,8 @@ template <typename V>
 __device__ __forceinline__ V ld_feat(const void* p);
 template <>
 __device__ __forceinline__ uint4 ld_feat<uint4>(const void* p) { return ld_nc_na_v4(p); }
+
+
 template <>
 __device__ __forceinline__ unsigned ld_feat<unsigned>(const void* p) { return ld_nc_na_u32(p); }
 template <>
