@@ -462,8 +462,10 @@ def bench_sweep(args):
     flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
     ids = torch.from_numpy(seeds.gather_ids(n, R, presets.SEED_BASE, 0)).to(dev)
     cells = []
-    for dtype in ("fp16", "fp32"):
-        for dim in (64, 128, 256, 512, 768, 1024):
+    grid = [("fp16", d) for d in (2, 4, 8, 16, 32)]  # 4-64 B segments (Fig. 8's small sizes, NEXT #3)
+    grid += [(t, d) for t in ("fp16", "fp32") for d in (64, 128, 256, 512, 768, 1024)]
+    for dtype, dim in grid:
+        if True:
             rb = dim * sfeat.elt_bytes(dtype)
             pitch = (rb + 63) // 64 * 64
             need = n * pitch + n * 8 + R * rb

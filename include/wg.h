@@ -41,6 +41,7 @@ extern "C" {
 #endif
 
 #define WG_MAX_WORLD 8          /* ranks (GPUs) per DSM: one HGX B200 box */
+#define WG_MAX_FANOUT 1024      /* largest M: <= 32 uses the warp sampler, above a block per target */
 
 typedef struct wg_dsm* wg_dsm_t; /* opaque host handle, one per rank process */
 typedef void* wg_stream_t;       /* a cudaStream_t */
@@ -52,7 +53,7 @@ typedef enum {
   WG_ERR_OOM = 3,          /* device allocation failed */
   WG_ERR_PEER_ACCESS = 4,  /* IPC export/import of a peer shard failed */
   WG_ERR_CAPACITY = 5,     /* request exceeds the workspace sized at create */
-  WG_ERR_UNSUPPORTED = 6,  /* device below sm_100, or fanout > 32 */
+  WG_ERR_UNSUPPORTED = 6,  /* device below sm_100, or fanout > WG_MAX_FANOUT */
   WG_ERR_COLLECTIVE = 7    /* the allgather callback returned non-zero */
 } wg_status;
 
@@ -140,8 +141,11 @@ wg_status wg_dsm_destroy(wg_dsm_t h);
  * adjacency list; d_out_num_edges (nullable) = device int64 total.
  * seed: the per-batch rng_seed; if d_seed is non-NULL the seed is read from that
  * device uint64 instead (so a captured CUDA graph can be replayed with new seeds).
- * Requires 1 <= fanout <= 32 (WG_ERR_UNSUPPORTED above 32) and n_targets * fanout <=
- * max_batch_keys (the padded per-target slots live in the workspace). */
+ * Requires 1 <= fanout <= WG_MAX_FANOUT (WG_ERR_UNSUPPORTED above) and n_targets * fanout
+ * <= max_batch_keys (the padded per-target slots live in the workspace).  fanout <= 32:
+ * a warp lane group per target with a sort-free form of Algorithm 1; fanout > 32: a
+ * block of next_pow2(fanout) threads per target running Algorithm 1 as listed, with
+ * a bitonic block sort as parallel_sort (L118-120).  Both give identical results. */
 wg_status wg_sample_neighbors(wg_dsm_t h, const int64_t* d_targets, int64_t n_targets,
                               const int64_t* d_n_targets, int32_t fanout, uint64_t seed,
                               const uint64_t* d_seed, int32_t hop, int64_t* d_out_row_ptr,

@@ -343,7 +343,7 @@ wg_status wg_sample_neighbors(wg_dsm_t h, const int64_t* d_targets, int64_t n_ta
                               int64_t* d_out_num_edges, wg_stream_t stream) {
   if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
   if (fanout < 1) return fail(WG_ERR_INVALID_ARG, "fanout must be >= 1");
-  if (fanout > 32) return fail(WG_ERR_UNSUPPORTED, "fanout > 32 (warp path only)");
+  if (fanout > WG_MAX_FANOUT) return fail(WG_ERR_UNSUPPORTED, "fanout > 1024");
   if (n_targets < 0 || (n_targets > 0 && !d_targets) || !d_out_row_ptr || (n_targets > 0 && !d_out_nbrs))
     return fail(WG_ERR_INVALID_ARG, "null pointer or negative size");
   if (hop < 0) return fail(WG_ERR_INVALID_ARG, "hop must be >= 0");
@@ -382,7 +382,7 @@ wg_status wg_sample_hop(wg_dsm_t h, const int64_t* d_targets, int64_t n_targets,
                         wg_stream_t stream, wg_stream_t side_stream) {
   if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
   if (fanout < 1) return fail(WG_ERR_INVALID_ARG, "fanout must be >= 1");
-  if (fanout > 32) return fail(WG_ERR_UNSUPPORTED, "fanout > 32 (warp path only)");
+  if (fanout > WG_MAX_FANOUT) return fail(WG_ERR_UNSUPPORTED, "fanout > 1024");
   if (n_targets < 0 || hop < 0 || !d_out_row_ptr || !d_out_num_edges ||
       (n_targets > 0 && (!d_targets || !d_out_nbrs || !d_out_unique || !d_out_sub_col)))
     return fail(WG_ERR_INVALID_ARG, "null pointer or negative size");

@@ -154,6 +154,127 @@ __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs
   }
 }
 
+// ---------------------------------------------------------------- fanout > 32
+// One block of BT = next_pow2(M) threads per target, "M threads in the thread block of
+// CUDA are grouped together to generate the sampled neighbors for one target node"
+// (L118): Algorithm 1 exactly as listed (L122-158), with parallel_sort = a block bitonic
+// sort of the packed 64-bit keys (r << 32 | i) (L118-120) in shared memory, chain / q /
+// last in shared memory and path doubling as ceil(log2 M) synchronous rounds.
+template <int BT>
+__global__ void __launch_bounds__(BT) sample_block_kernel(const SampleArgs a) {
+  __shared__ unsigned long long s_key[BT];
+  __shared__ unsigned s_r[BT], s_chain[BT], s_q[BT], s_last[BT];
+  __shared__ int64_t s_v, s_start;
+  __shared__ unsigned s_n;
+  int64_t nT = a.cap;
+  if (a.d_n) {
+    nT = *a.d_n;
+    nT = nT < 0 ? 0 : (nT > a.cap ? a.cap : nT);
+  }
+  const int64_t k = blockIdx.x;
+  if (k >= nT) return;
+  const int i = threadIdx.x;
+  const int M = a.M;
+  if (i == 0) {
+    int64_t v = a.targets[k], start = 0;
+    unsigned n = 0;
+    if (v < 0 || v >= a.s.n) {
+      latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_ID_RANGE);
+      v = -1;
+    } else {
+      int o;
+      int64_t l;
+      owner_local(a.s, v, o, l);
+      const int64_t* rp = a.s.row_ptr[o] + l;
+      start = rp[0];
+      const int64_t d = rp[1] - start;
+      if (d >= (int64_t(1) << 32) || d < 0)
+        latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DEGREE);
+      else
+        n = (unsigned)d;
+    }
+    s_v = v;
+    s_start = start;
+    s_n = n;
+    a.cnt[k] = v >= 0 ? (int32_t)min(n, (unsigned)M) : 0;
+  }
+  __syncthreads();
+  const int64_t v = s_v;
+  if (v < 0) return;
+  const unsigned N = s_n;
+  int o;
+  int64_t l;
+  owner_local(a.s, v, o, l);
+  const int64_t* col = a.s.col[o] + s_start;
+  if (N <= (unsigned)M) {  // L118: all of N neighbours, CSR order (A5)
+    for (unsigned j = i; j < N; j += BT) {
+      a.nbrs_pad[k * M + j] = col[j];
+      if (a.pos_pad) a.pos_pad[k * M + j] = (int32_t)j;
+    }
+    return;
+  }
+  // line 1-4: r[i] = random(N-1-i); chain[i] = i
+  const unsigned long long seed = a.d_seed ? *a.d_seed : a.seed;
+  unsigned r = 0;
+  if (i < M) {
+    const uint4 x = philox4x32_10(make_uint4((unsigned)(i >> 2), (unsigned)a.hop, (unsigned)((uint64_t)v & 0xffffffffu),
+                                             (unsigned)((uint64_t)v >> 32)),
+                                  make_uint2((unsigned)(seed & 0xffffffffu), (unsigned)(seed >> 32)));
+    const unsigned xi = (i & 3) == 0 ? x.x : (i & 3) == 1 ? x.y : (i & 3) == 2 ? x.z : x.w;
+    r = __umulhi(xi, N - (unsigned)i);
+  }
+  s_r[i] = r;
+  s_chain[i] = (unsigned)i;
+  s_key[i] = i < M ? (((unsigned long long)r << 32) | (unsigned)i) : ~0ull;
+  __syncthreads();
+  // line 5: s, p = parallel_sort(r) -- bitonic sort of the packed keys
+  for (int size = 2; size <= BT; size <<= 1) {
+    for (int stride = size >> 1; stride > 0; stride >>= 1) {
+      const int partner = i ^ stride;
+      if (partner > i) {
+        const unsigned long long x = s_key[i], y = s_key[partner];
+        const bool up = (i & size) == 0;
+        if ((x > y) == up) {
+          s_key[i] = y;
+          s_key[partner] = x;
+        }
+      }
+      __syncthreads();
+    }
+  }
+  // lines 6-11
+  unsigned si = 0, pi = 0;
+  if (i < M) {
+    si = (unsigned)(s_key[i] >> 32);
+    pi = (unsigned)(s_key[i] & 0xffffffffu);
+    s_q[pi] = (unsigned)i;
+    const bool run_end = (i == M - 1) || si != (unsigned)(s_key[i + 1] >> 32);
+    if (run_end && si >= N - (unsigned)M) s_chain[N - si - 1] = pi;
+  }
+  __syncthreads();
+  // line 12: path doubling
+  for (int step = 1; step < M; step <<= 1) {
+    const unsigned c = i < M ? s_chain[s_chain[i]] : 0u;
+    __syncthreads();
+    if (i < M) s_chain[i] = c;
+    __syncthreads();
+  }
+  // lines 13-15
+  if (i < M) s_last[i] = N - s_chain[i] - 1;
+  __syncthreads();
+  // lines 16-22
+  if (i < M) {
+    const unsigned qi = s_q[i];
+    unsigned res;
+    if (i == 0 || qi == 0 || (unsigned)(s_key[qi] >> 32) != (unsigned)(s_key[qi - 1] >> 32))
+      res = s_r[i];
+    else
+      res = s_last[(unsigned)(s_key[qi - 1] & 0xffffffffu)];
+    a.nbrs_pad[k * M + i] = col[res];
+    if (a.pos_pad) a.pos_pad[k * M + i] = (int32_t)res;
+  }
+}
+
 // ---------------------------------------------------------------- compaction
 // out_row_ptr = exclusive scan of cnt; out_nbrs / out_pos = the valid padded slots in
 // order.  Single pass, decoupled look-back over tiles of COMPACT_TILE targets.
@@ -232,6 +353,15 @@ cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap,
   a.pos_pad = want_pos ? h->ws.pos_pad : nullptr;
   a.cnt = h->ws.cnt;
   a.ctrl = h->ws.ctrl;
+  if (fanout > 32) {  // block per target (Algorithm 1 with a block sort)
+    const unsigned blocks = (unsigned)(cap > 0 ? cap : 1);
+    if (fanout <= 64) sample_block_kernel<64><<<blocks, 64, 0, st>>>(a);
+    else if (fanout <= 128) sample_block_kernel<128><<<blocks, 128, 0, st>>>(a);
+    else if (fanout <= 256) sample_block_kernel<256><<<blocks, 256, 0, st>>>(a);
+    else if (fanout <= 512) sample_block_kernel<512><<<blocks, 512, 0, st>>>(a);
+    else sample_block_kernel<1024><<<blocks, 1024, 0, st>>>(a);
+    return cudaGetLastError();
+  }
   const int G = fanout <= 8 ? 8 : fanout <= 16 ? 16 : 32;
   int unr = 4;  // largest of 4/2/1 that still gives >= 2 blocks per SM
   while (unr > 1 && cap < (int64_t)(SAMPLE_THREADS / G) * unr * 2 * h->sm_count) unr >>= 1;

@@ -245,3 +245,38 @@ print("TMA OK")
     r = subprocess.run([sys.executable, "-c", code], cwd=root, env=dict(os.environ, WG_GATHER_TMA="1"),
                        capture_output=True, text=True, timeout=600)
     assert r.returncode == 0 and "TMA OK" in r.stdout, r.stdout + r.stderr
+
+
+@pytest.mark.parametrize("M", [33, 64, 100, 257, 1024])
+def test_sample_large_fanout_block_kernel(M):
+    """fanout > 32: block per target running Algorithm 1 with a block bitonic sort (NEXT #4)."""
+    rng = np.random.default_rng(M)
+    n = 3000
+    degs = [0, 1, 32, 33, M - 1, M, M + 1, 2 * M, 5000]
+    rows = [np.sort(rng.choice(n, size=min(degs[v % len(degs)], n), replace=False)) if degs[v % len(degs)] <= n
+            else rng.integers(0, n, degs[v % len(degs)]) for v in range(n)]
+    rp, col = csr_from_rows(rows)
+    dsm = make_dsm(rp, col, max_keys=1 << 20)
+    T = np.arange(0, 400, dtype=np.int64)
+    for hop, seed in ((0, 99), (2, 0xDEADBEEF12345678)):
+        g = gpu_hop(dsm, T, M, seed, hop)
+        o = oracle_hop(rp, col, T, M, seed, hop)
+        for a, b in zip(g, o):
+            assert np.array_equal(a, b)
+    assert dsm.device_error() == 0
+    dsm.destroy()
+
+
+def test_pipeline_large_fanout(tiny):
+    p, rp, col = tiny
+    dsm, _ = loader.build_dsm(p, on_device=False, max_seeds=64, extra_keys=64 * 60 * 41 + 64 * 60)
+    fan = [60, 40]
+    pipe = pkg.MiniBatchPipeline(dsm, fan, 64, with_pos=True, with_dup=True)
+    S = seeds.seed_nodes(p.n, 64, presets.SEED_BASE, 3)
+    rs = seeds.rng_seed(presets.RNG_BASE, 3)
+    pipe.run(torch.from_numpy(S).cuda(), rs)
+    torch.cuda.synchronize()
+    ref = oracle.minibatch(loader.host_row_provider(p.graph(), rp, col), loader.host_feat_provider(p), S, fan, rs)
+    _check_batch(pipe, ref, fan)
+    assert dsm.device_error() == 0
+    dsm.destroy()
