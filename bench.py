@@ -43,6 +43,8 @@ def parse():
     ap.add_argument("--sweep", action="store_true", help="config 4: feature-gather sweep over row sizes")
     ap.add_argument("--sweep-rows", type=int, default=100_000_000)
     ap.add_argument("--sweep-ids", type=int, default=1_000_000)
+    ap.add_argument("--latency", action="store_true", help="Table I analogue: dependent-load latency vs span")
+    ap.add_argument("--chase-accesses", type=int, default=100_000)
     return ap.parse_args()
 
 
@@ -509,9 +511,43 @@ def bench_sweep(args):
     emit(line, args)
 
 
+def bench_latency(args):
+    """NEXT #3 / PAPER.md Table I (L66-80): dependent 8 B load latency vs span (8..128 GB) of a
+    DSM shard, one thread, `accesses` chained loads.  W=1: local HBM (the P2P column needs W>1)."""
+    import torch
+
+    import paper_conf_sc_yanglql22_b200 as pkg
+    torch.cuda.set_device(0)
+    free, _ = torch.cuda.mem_get_info()
+    gib = 1 << 30
+    spans = [s * gib for s in (1, 8, 16, 32, 64, 128) if s * gib < 0.85 * free]
+    rows = max(spans) // 512
+    dsm = pkg.DSM(rows, 0, 128, "fp32", 1, device=0)   # 512 B rows, filled with generator bits
+    from synth import gpu as sgpu
+    from synth import presets
+    _, _, fv = dsm.local_view()
+    sgpu.fill_features_gpu(fv, presets.FEAT_SEED, 0, 1, 128, 0)
+    torch.cuda.synchronize()
+    del fv
+    res = []
+    for sp in spans:
+        dsm.chase(0, sp, 2000)                            # warm-up (TLB, clocks)
+        ns = statistics.median(dsm.chase(0, sp, args.chase_accesses) for _ in range(3))
+        res.append({"span_gb": sp / gib, "ns_per_access": ns})
+    dsm.destroy()
+    line = {"metric": "dependent-load latency through a DSM shard (Table I analogue, local HBM, W=1)",
+            "value": res[-1]["ns_per_access"], "unit": "ns", "higher_is_better": False,
+            "config": {"accesses": args.chase_accesses, "threads": 1, "paper_A100_p2p_us": [1.35, 1.37, 1.43, 1.51, 1.56],
+                       "paper_A100_um_us": [20.8, 29.6, 32.5, 35.3, 35.8]},
+            "spans": res}
+    emit(line, args)
+
+
 def main():
     args = parse()
-    if args.sweep:
+    if args.latency:
+        bench_latency(args)
+    elif args.sweep:
         bench_sweep(args)
     elif args.impl == "reference":
         bench_reference(args)

@@ -197,6 +197,16 @@ wg_status wg_sample_hop(wg_dsm_t h, const int64_t* d_targets, int64_t n_targets,
 wg_status wg_gather(wg_dsm_t h, const int64_t* d_ids, int64_t n_ids, const int64_t* d_n_ids,
                     void* d_out, wg_stream_t stream);
 
+/* DSM characterisation, the analogue of PAPER.md Table I (L66-80): one GPU thread
+ * performs `accesses` dependent 8 B loads at random 64 B-aligned offsets within the
+ * first span_bytes of rank `rank`'s feature shard (local HBM when rank is this rank,
+ * a peer's HBM over NVLink otherwise); each address is a hash of the previously loaded
+ * value.  The caller times the launch (e.g. with CUDA events) and divides by
+ * `accesses`.  d_sink: one device uint64 receiving a checksum (keeps the loads live).
+ * Errors: WG_ERR_INVALID_ARG if span_bytes exceeds that shard. */
+wg_status wg_dsm_chase(wg_dsm_t h, int32_t rank, int64_t span_bytes, int64_t accesses, uint64_t* d_sink,
+                       wg_stream_t stream);
+
 /* Read (and optionally clear) the latched device error word.  Synchronises the
  * handle's device. */
 wg_status wg_device_error(wg_dsm_t h, uint32_t* code, int32_t clear);

@@ -144,6 +144,17 @@ class DSM:
         check(lib().wg_device_error(self.h, ctypes.byref(c), 1 if clear else 0))
         return c.value
 
+    def chase(self, rank, span_bytes, accesses, stream=None):
+        """Table-I-style dependent-load latency through rank's feature shard; returns ns/access."""
+        sink = torch.zeros(1, dtype=torch.int64, device=self.device)
+        s = stream or torch.cuda.current_stream(self.device)
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(s)
+        check(lib().wg_dsm_chase(self.h, rank, span_bytes, accesses, _ptr(sink), _stream(s)))
+        e1.record(s)
+        e1.synchronize()
+        return e0.elapsed_time(e1) * 1e6 / accesses
+
     def reset_workspace(self, stream=None):
         check(lib().wg_dsm_reset_workspace(self.h, _stream(stream)))
 

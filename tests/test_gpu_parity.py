@@ -280,3 +280,15 @@ def test_pipeline_large_fanout(tiny):
     _check_batch(pipe, ref, fan)
     assert dsm.device_error() == 0
     dsm.destroy()
+
+
+def test_dsm_chase_latency_runs():
+    """wg_dsm_chase (Table I analogue): a positive, plausible per-access latency; span checks."""
+    n = 1 << 16
+    rp = np.zeros(n + 1, dtype=np.int64)
+    dsm = pkg.DSM(n, 0, 16, "fp32", 16)
+    ns = dsm.chase(0, n * 64, 20000)
+    assert 20 < ns < 5000
+    with pytest.raises(pkg.WgError):
+        dsm.chase(0, n * 64 * 2, 10)
+    dsm.destroy()
