@@ -197,6 +197,25 @@ wg_status wg_sample_hop(wg_dsm_t h, const int64_t* d_targets, int64_t n_targets,
 wg_status wg_gather(wg_dsm_t h, const int64_t* d_ids, int64_t n_ids, const int64_t* d_n_ids,
                     void* d_out, wg_stream_t stream);
 
+/* ---- GNN layer op consuming the prepared mini-batch (III-C4) ----
+ * g-SpMM with mean aggregation (GraphSAGE-mean message passing, Eq. (1)) on the
+ * sub-graph CSR produced by one hop: rows = targets (d_row_ptr int64[n_rows+1], e.g.
+ * wg_sample_hop's d_out_row_ptr), columns = sub-graph ids (d_sub_col int32), features
+ * d_x float32 [*, dim] row-major (e.g. the gathered X viewed as float32; dim % 4 == 0).
+ * forward:  d_y[t, :] = mean over the row's edges of d_x[sub_col[e], :] (0 for an empty
+ *           row), fp32 accumulation in edge order.
+ * backward: d_dx[c, :] = sum over edges t->c of d_dy[t, :] / deg(t), computed on the same
+ *           CSR with atomic adds (no transpose, L186); rows with d_dup_count == 1 (the
+ *           Append Unique duplicate count; nullable) are written with a plain store
+ *           (L186-192).  d_dx [n_x_rows, dim] is zeroed by the call.
+ * d_n_rows: optional device count (as for the other ops). */
+wg_status wg_spmm_mean_forward(const int64_t* d_row_ptr, int64_t n_rows, const int64_t* d_n_rows,
+                               const int32_t* d_sub_col, const float* d_x, int64_t dim, float* d_y,
+                               wg_stream_t stream);
+wg_status wg_spmm_mean_backward(const int64_t* d_row_ptr, int64_t n_rows, const int64_t* d_n_rows,
+                                const int32_t* d_sub_col, const int32_t* d_dup_count, const float* d_dy,
+                                int64_t dim, float* d_dx, int64_t n_x_rows, wg_stream_t stream);
+
 /* DSM characterisation, the analogue of PAPER.md Table I (L66-80): one GPU thread
  * performs `accesses` dependent 8 B loads at random 64 B-aligned offsets within the
  * first span_bytes of rank `rank`'s feature shard (local HBM when rank is this rank,

@@ -51,6 +51,10 @@ def lib():
         L.orc_append_unique.restype = ctypes.c_int
         L.orc_gather.argtypes = [P, P, ctypes.c_int64, ctypes.c_int64, P, ctypes.c_int64, P]
         L.orc_gather.restype = ctypes.c_int
+        L.orc_spmm_mean_forward.argtypes = [P, ctypes.c_int64, P, P, ctypes.c_int64, P]
+        L.orc_spmm_mean_forward.restype = None
+        L.orc_spmm_mean_backward.argtypes = [P, ctypes.c_int64, P, P, ctypes.c_int64, P, ctypes.c_int64]
+        L.orc_spmm_mean_backward.restype = None
         _lib = L
     return _lib
 
@@ -135,6 +139,29 @@ def gather(table_rows, table_ids, ids):
     if rc != 0:
         raise ValueError("gather: id without a table row")
     return out
+
+
+def spmm_mean_forward(row_ptr, col, x):
+    """g-SpMM mean aggregation forward, float64."""
+    row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
+    col = np.ascontiguousarray(col, dtype=np.int32)
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    n = len(row_ptr) - 1
+    y = np.zeros((n, x.shape[1]), dtype=np.float64)
+    lib().orc_spmm_mean_forward(_p(row_ptr), n, _p(col if len(col) else np.zeros(1, np.int32)), _p(x), x.shape[1], _p(y))
+    return y
+
+
+def spmm_mean_backward(row_ptr, col, dy, n_x_rows):
+    """g-SpMM mean aggregation backward (gradient w.r.t. x), float64."""
+    row_ptr = np.ascontiguousarray(row_ptr, dtype=np.int64)
+    col = np.ascontiguousarray(col, dtype=np.int32)
+    dy = np.ascontiguousarray(dy, dtype=np.float64)
+    n = len(row_ptr) - 1
+    dx = np.zeros((n_x_rows, dy.shape[1]), dtype=np.float64)
+    lib().orc_spmm_mean_backward(_p(row_ptr), n, _p(col if len(col) else np.zeros(1, np.int32)), _p(dy), dy.shape[1],
+                                 _p(dx), n_x_rows)
+    return dx
 
 
 def minibatch(row_provider, feat_provider, seeds, fanouts, rng_seed: int, timer=None):

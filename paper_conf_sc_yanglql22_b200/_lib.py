@@ -52,10 +52,14 @@ def lib():
     L.wg_sample_hop.argtypes = [P, P, I64, P, I32, U64, P, I32, P, P, P, P, P, P, P, P, P, P]
     L.wg_gather.argtypes = [P, P, I64, P, P, P]
     L.wg_dsm_chase.argtypes = [P, I32, I64, I64, P, P]
+    L.wg_spmm_mean_forward.argtypes = [P, I64, P, P, P, I64, P, P]
+    L.wg_spmm_mean_backward.argtypes = [P, I64, P, P, P, P, I64, P, I64, P]
     L.wg_device_error.argtypes = [P, P, I32]
     L.wg_dsm_reset_workspace.argtypes = [P, P]
     for f in ("wg_dsm_create", "wg_dsm_fork", "wg_dsm_local_view", "wg_dsm_shard_info", "wg_dsm_destroy", "wg_sample_neighbors",
-              "wg_append_unique", "wg_sample_hop", "wg_gather", "wg_dsm_chase", "wg_dsm_chase", "wg_device_error", "wg_dsm_reset_workspace"):
+              "wg_append_unique", "wg_sample_hop", "wg_gather", "wg_dsm_chase", "wg_spmm_mean_forward",
+           "wg_spmm_mean_backward", "wg_spmm_mean_forward",
+              "wg_spmm_mean_backward", "wg_dsm_chase", "wg_device_error", "wg_dsm_reset_workspace"):
         getattr(L, f).restype = ctypes.c_int
     L.wg_last_error.restype = ctypes.c_char_p
     L.wg_last_error.argtypes = []
@@ -71,5 +75,6 @@ def check(status):
 
 
 EXPORTS = ["wg_dsm_create", "wg_dsm_fork", "wg_dsm_local_view", "wg_dsm_shard_info", "wg_dsm_destroy", "wg_sample_neighbors",
-           "wg_append_unique", "wg_sample_hop", "wg_gather", "wg_dsm_chase", "wg_device_error", "wg_dsm_reset_workspace", "wg_last_error",
+           "wg_append_unique", "wg_sample_hop", "wg_gather", "wg_dsm_chase", "wg_spmm_mean_forward",
+           "wg_spmm_mean_backward", "wg_device_error", "wg_dsm_reset_workspace", "wg_last_error",
            "wg_version"]

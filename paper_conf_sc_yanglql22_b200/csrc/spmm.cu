@@ -1,0 +1,121 @@
+// spmm.cu -- g-SpMM on the sampled sub-graph CSR (section III-C4;
+// SURVEY.md 8(f) NEXT #2): the GraphSAGE-mean message passing of Eq. (1) that consumes
+// the hot path's outputs (row_ptr, sub_col, X).
+//
+// forward   Y[t, :] = 1/deg(t) * sum_{e in row t} X[sub_col[e], :]   ("the forward of
+//           g-SpMM can be done directly on the CSR matrix", L186)
+// backward  dX[c, :] += dY[t, :] / deg(t) for every edge t -> c, computed on the same CSR
+//           with atomic adds instead of a transpose (L186); sub-graph nodes sampled exactly
+//           once (duplicate count 1, produced by Append Unique) receive a plain store
+//           instead of an atomic (L186-192).
+// One warp per target row, lanes over 16 B slices of the feature row; fp32 accumulate in
+// edge order (deterministic forward).
+#include "device_util.cuh"
+#include "wg_internal.cuh"
+
+namespace wg {
+
+constexpr int SPMM_THREADS = 256;
+
+__device__ __forceinline__ int64_t count_or_cap(const int64_t* d, int64_t cap) {
+  if (!d) return cap;
+  const int64_t v = *d;
+  return v < 0 ? 0 : (v > cap ? cap : v);
+}
+
+// D4 = feature columns / 4 (float4 slices per row)
+__global__ void __launch_bounds__(SPMM_THREADS) spmm_mean_fwd_kernel(const int64_t* row_ptr, int64_t cap_rows,
+                                                                     const int64_t* d_rows, const int32_t* col,
+                                                                     const float4* X, int D4, float4* Y) {
+  const int64_t n = count_or_cap(d_rows, cap_rows);
+  const int lane = threadIdx.x & 31;
+  const int64_t warps = (int64_t)gridDim.x * (SPMM_THREADS / 32);
+  for (int64_t t = ((int64_t)blockIdx.x * SPMM_THREADS + threadIdx.x) / 32; t < n; t += warps) {
+    const int64_t b = row_ptr[t], e = row_ptr[t + 1];
+    const float inv = e > b ? 1.0f / (float)(e - b) : 0.0f;
+    for (int c = lane; c < D4; c += 32) {
+      float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int64_t k = b; k < e; ++k) {
+        const float4 x = __ldg(&X[(int64_t)col[k] * D4 + c]);
+        acc.x += x.x;
+        acc.y += x.y;
+        acc.z += x.z;
+        acc.w += x.w;
+      }
+      Y[t * D4 + c] = make_float4(acc.x * inv, acc.y * inv, acc.z * inv, acc.w * inv);
+    }
+  }
+}
+
+__global__ void __launch_bounds__(SPMM_THREADS) spmm_mean_bwd_kernel(const int64_t* row_ptr, int64_t cap_rows,
+                                                                     const int64_t* d_rows, const int32_t* col,
+                                                                     const int32_t* dup, const float4* dY, int D4,
+                                                                     float4* dX) {
+  const int64_t n = count_or_cap(d_rows, cap_rows);
+  const int lane = threadIdx.x & 31;
+  const int64_t warps = (int64_t)gridDim.x * (SPMM_THREADS / 32);
+  for (int64_t t = ((int64_t)blockIdx.x * SPMM_THREADS + threadIdx.x) / 32; t < n; t += warps) {
+    const int64_t b = row_ptr[t], e = row_ptr[t + 1];
+    if (e == b) continue;
+    const float inv = 1.0f / (float)(e - b);
+    for (int c = lane; c < D4; c += 32) {
+      float4 g = dY[t * D4 + c];
+      g = make_float4(g.x * inv, g.y * inv, g.z * inv, g.w * inv);
+      for (int64_t k = b; k < e; ++k) {
+        const int64_t r = col[k];
+        if (dup && dup[r] == 1)
+          dX[r * D4 + c] = g;  // the only contribution this row receives
+        else
+          atomicAdd(&dX[r * D4 + c], g);
+      }
+    }
+  }
+}
+
+}  // namespace wg
+
+using namespace wg;
+
+extern "C" {
+
+wg_status wg_spmm_mean_forward(const int64_t* d_row_ptr, int64_t n_rows, const int64_t* d_n_rows,
+                               const int32_t* d_sub_col, const float* d_x, int64_t dim, float* d_y,
+                               wg_stream_t stream) {
+  if (n_rows < 0 || dim <= 0 || dim % 4 != 0 || (n_rows > 0 && (!d_row_ptr || !d_sub_col || !d_x || !d_y)))
+    return fail(WG_ERR_INVALID_ARG, "bad arguments (dim must be a positive multiple of 4)");
+  if (n_rows == 0) return WG_OK;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  int64_t blocks = (n_rows * 32 + SPMM_THREADS - 1) / SPMM_THREADS;
+  blocks = blocks > (int64_t)sms * 8 ? (int64_t)sms * 8 : blocks;
+  spmm_mean_fwd_kernel<<<(unsigned)blocks, SPMM_THREADS, 0, (cudaStream_t)stream>>>(
+      d_row_ptr, n_rows, d_n_rows, d_sub_col, reinterpret_cast<const float4*>(d_x), (int)(dim / 4),
+      reinterpret_cast<float4*>(d_y));
+  cudaError_t e = cudaGetLastError();
+  return e == cudaSuccess ? WG_OK : fail(WG_ERR_CUDA, cudaGetErrorString(e));
+}
+
+wg_status wg_spmm_mean_backward(const int64_t* d_row_ptr, int64_t n_rows, const int64_t* d_n_rows,
+                                const int32_t* d_sub_col, const int32_t* d_dup_count, const float* d_dy,
+                                int64_t dim, float* d_dx, int64_t n_x_rows, wg_stream_t stream) {
+  if (n_rows < 0 || n_x_rows < 0 || dim <= 0 || dim % 4 != 0 ||
+      (n_rows > 0 && (!d_row_ptr || !d_sub_col || !d_dy || !d_dx)))
+    return fail(WG_ERR_INVALID_ARG, "bad arguments (dim must be a positive multiple of 4)");
+  cudaStream_t st = (cudaStream_t)stream;
+  cudaError_t e = cudaMemsetAsync(d_dx, 0, (size_t)n_x_rows * dim * sizeof(float), st);
+  if (e != cudaSuccess) return fail(WG_ERR_CUDA, cudaGetErrorString(e));
+  if (n_rows == 0) return WG_OK;
+  int dev = 0, sms = 148;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  int64_t blocks = (n_rows * 32 + SPMM_THREADS - 1) / SPMM_THREADS;
+  blocks = blocks > (int64_t)sms * 8 ? (int64_t)sms * 8 : blocks;
+  spmm_mean_bwd_kernel<<<(unsigned)blocks, SPMM_THREADS, 0, st>>>(
+      d_row_ptr, n_rows, d_n_rows, d_sub_col, d_dup_count, reinterpret_cast<const float4*>(d_dy), (int)(dim / 4),
+      reinterpret_cast<float4*>(d_dx));
+  e = cudaGetLastError();
+  return e == cudaSuccess ? WG_OK : fail(WG_ERR_CUDA, cudaGetErrorString(e));
+}
+
+}  // extern "C"

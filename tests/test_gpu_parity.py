@@ -292,3 +292,39 @@ def test_dsm_chase_latency_runs():
     with pytest.raises(pkg.WgError):
         dsm.chase(0, n * 64 * 2, 10)
     dsm.destroy()
+
+
+def test_spmm_mean_forward_backward_vs_oracle(tiny):
+    """NEXT #2: g-SpMM mean aggregation on the last hop's sub-graph CSR with the gathered
+    features (float32), forward and backward (atomics + duplicate-count stores) against the
+    float64 oracle; fp32 tolerance: <= 16-term sums in forward, atomics order in backward."""
+    from paper_conf_sc_yanglql22_b200 import layers
+    p, rp, col = tiny
+    dsm, _ = loader.build_dsm(p, on_device=False)
+    pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_dup=True)
+    S = seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 11)
+    pipe.run(torch.from_numpy(S).cuda(), seeds.rng_seed(presets.RNG_BASE, 11))
+    torch.cuda.synchronize()
+    h = pipe.result(1)
+    nT = len(pipe.result(0)["unique"])
+    U = len(h["unique"])
+    X = torch.from_numpy(pipe.features().view(np.float32).reshape(U, p.feat_dim).copy()).cuda()
+    row_ptr = torch.from_numpy(h["row_ptr"]).cuda()
+    sub_col = torch.from_numpy(h["sub_col"]).cuda()
+    dup = torch.from_numpy(h["dup"]).cuda()
+    Y = layers.spmm_mean_forward(row_ptr, sub_col, X)
+    Yo = oracle.spmm_mean_forward(h["row_ptr"], h["sub_col"], X.cpu().double().numpy())
+    assert Y.shape == (nT, p.feat_dim)
+    assert np.allclose(Y.cpu().numpy(), Yo, rtol=0, atol=1e-5)
+    dY = torch.from_numpy(np.random.default_rng(1).uniform(-1, 1, (nT, p.feat_dim)).astype(np.float32)).cuda()
+    dX = layers.spmm_mean_backward(row_ptr, sub_col, dup, dY, U)
+    dX_nodup = layers.spmm_mean_backward(row_ptr, sub_col, None, dY, U)
+    dXo = oracle.spmm_mean_backward(h["row_ptr"], h["sub_col"], dY.cpu().double().numpy(), U)
+    assert np.allclose(dX.cpu().numpy(), dXo, rtol=1e-5, atol=1e-5)
+    assert np.allclose(dX.cpu().numpy(), dX_nodup.cpu().numpy(), rtol=1e-5, atol=1e-5)
+    # autograd wrapper
+    Xg = X.clone().requires_grad_(True)
+    out = layers.SpMMMean.apply(Xg, row_ptr, sub_col, dup)
+    (out * dY).sum().backward()
+    assert np.allclose(Xg.grad.cpu().numpy(), dXo, rtol=1e-5, atol=1e-5)
+    dsm.destroy()

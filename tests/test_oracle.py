@@ -288,3 +288,27 @@ def test_minibatch_tiny_invariants():
         check_append_unique(T, hop["nbrs"], hop["unique"], hop["sub_col"], hop["dup"])
         prevU = hop["unique"]
     assert np.array_equal(out["X"], features.feature_bytes(presets.FEAT_SEED, prevU, p.feat_dim, p.feat_dtype))
+
+
+# ---------------------------------------------------------------- g-SpMM (NEXT #2)
+def test_spmm_mean_pins():
+    """orc_spmm_mean_*: mean of constant rows is the constant, empty rows give 0,
+    linearity, and the adjoint identity <dy, A x> = <A^T dy, x> ties backward to forward."""
+    rng = np.random.default_rng(2)
+    nx, d = 50, 8
+    deg = rng.integers(0, 6, size=30)
+    rp = np.concatenate(([0], np.cumsum(deg)))
+    col = rng.integers(0, nx, size=rp[-1]).astype(np.int32)
+    x = np.ones((nx, d)) * 3.5
+    y = oracle.spmm_mean_forward(rp, col, x)
+    assert np.allclose(y[deg > 0], 3.5) and np.all(y[deg == 0] == 0)
+    x1, x2 = rng.standard_normal((nx, d)), rng.standard_normal((nx, d))
+    assert np.allclose(oracle.spmm_mean_forward(rp, col, 2 * x1 - x2),
+                       2 * oracle.spmm_mean_forward(rp, col, x1) - oracle.spmm_mean_forward(rp, col, x2))
+    dy = rng.standard_normal((30, d))
+    lhs = np.sum(dy * oracle.spmm_mean_forward(rp, col, x1))
+    rhs = np.sum(oracle.spmm_mean_backward(rp, col, dy, nx) * x1)
+    assert abs(lhs - rhs) < 1e-9 * max(1, abs(lhs))
+    # one row, explicit: mean of rows 1 and 3
+    y = oracle.spmm_mean_forward([0, 2], np.array([1, 3], np.int32), x1)
+    assert np.allclose(y[0], (x1[1] + x1[3]) / 2)
