@@ -44,6 +44,7 @@ def parse():
     ap.add_argument("--sweep-rows", type=int, default=100_000_000)
     ap.add_argument("--sweep-ids", type=int, default=1_000_000)
     ap.add_argument("--latency", action="store_true", help="Table I analogue: dependent-load latency vs span")
+    ap.add_argument("--layer", action="store_true", help="NEXT #2: g-SpMM mean aggregation on a prepared batch")
     ap.add_argument("--chase-accesses", type=int, default=100_000)
     return ap.parse_args()
 
@@ -543,9 +544,61 @@ def bench_latency(args):
     emit(line, args)
 
 
+def bench_layer(args):
+    """NEXT #2 measurement: g-SpMM mean aggregation (GraphSAGE layer input) on a prepared
+    products-shaped batch -- the last hop's CSR and the gathered features."""
+    import torch
+
+    import paper_conf_sc_yanglql22_b200 as pkg
+    from paper_conf_sc_yanglql22_b200 import layers, loader
+    from synth import presets, seeds
+    torch.cuda.set_device(0)
+    p = presets.get(args.config)
+    dsm, _ = loader.build_dsm(p)
+    pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_dup=True)
+    S = torch.from_numpy(seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 5)).cuda()
+    pipe.run(S, seeds.rng_seed(presets.RNG_BASE, 5))
+    torch.cuda.synchronize()
+    last, prev = pipe.hops[-1], pipe.hops[-2]
+    T = int(prev["num_unique"].item())
+    E = int(last["num_edges"].item())
+    U = int(last["num_unique"].item())
+    D = p.feat_dim
+    X = pipe.X[:U].view(torch.float32).reshape(U, D) if p.feat_dtype == "fp32" else torch.rand(U, D, device="cuda")
+    row_ptr, sub_col, dup = last["row_ptr"][:T + 1], last["sub_col"][:E], last["dup"][:U]
+    dY = torch.rand(T, D, device="cuda")
+    peak, peak_src = peaks()
+    res = {}
+    for name, fn, alg in (
+            ("forward", lambda: layers.spmm_mean_forward(row_ptr, sub_col, X), (E + T) * D * 4 + E * 4 + T * 8),
+            ("backward", lambda: layers.spmm_mean_backward(row_ptr, sub_col, dup, dY, U),
+             (T + E) * D * 4 + U * D * 4 + E * 4 + T * 8)):
+        for _ in range(3):
+            fn()
+        ts = []
+        for _ in range(args.steps):
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            fn()
+            e1.record()
+            torch.cuda.synchronize()
+            ts.append(e0.elapsed_time(e1) / 1e3)
+        t = statistics.median(ts)
+        res[name] = {"ms": t * 1e3, "algorithmic_bytes": alg, "achieved_gbs": alg / t / 1e9,
+                     "frac_of_hbm_roofline": alg / t / 1e9 / peak}
+    dsm.destroy()
+    line = {"metric": "g-SpMM mean aggregation on the prepared batch (NEXT #2)", "value": res["forward"]["achieved_gbs"],
+            "unit": "GB/s", "higher_is_better": True, "n_gpus": 1, "steps": args.steps,
+            "config": {"workload": p.name, "rows": T, "edges": E, "x_rows": U, "dim": D, "dtype": "fp32"},
+            "roofline": {"bound": "hbm", "peak": peak, "peak_source": peak_src}, "results": res}
+    emit(line, args)
+
+
 def main():
     args = parse()
-    if args.latency:
+    if args.layer:
+        bench_layer(args)
+    elif args.latency:
         bench_latency(args)
     elif args.sweep:
         bench_sweep(args)
