@@ -45,6 +45,7 @@ def parse():
     ap.add_argument("--sweep-ids", type=int, default=1_000_000)
     ap.add_argument("--latency", action="store_true", help="Table I analogue: dependent-load latency vs span")
     ap.add_argument("--layer", action="store_true", help="NEXT #2: g-SpMM mean aggregation on a prepared batch")
+    ap.add_argument("--compare-gather", action="store_true", help="NEXT #1: P2P vs distributed-memory gather")
     ap.add_argument("--chase-accesses", type=int, default=100_000)
     return ap.parse_args()
 
@@ -594,9 +595,79 @@ def bench_layer(args):
     emit(line, args)
 
 
+def bench_compare_gather(args):
+    """NEXT #1 / PAPER.md Fig. 10 (L297-305): the P2P global gather (one kernel, L182) vs the
+    distributed-memory five-step gather (bucket, all-to-all ids, local gather, all-to-all rows,
+    reorder, L178-180) on the same ids.  Under torchrun (W>1) the all-to-alls run on NCCL; at
+    W=1 they are local copies, so the ratio shows the extra memory passes only."""
+    import torch
+    import torch.distributed as dist
+
+    import paper_conf_sc_yanglql22_b200 as pkg
+    from paper_conf_sc_yanglql22_b200 import loader
+    from paper_conf_sc_yanglql22_b200.nccl_gather import DistributedGather
+    from synth import presets, seeds
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0")) % torch.cuda.device_count()
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    ag = None
+    if world > 1:
+        if torch.cuda.device_count() >= world:
+            dist.init_process_group("nccl", device_id=dev)
+        else:
+            dist.init_process_group("gloo")
+        ag = pkg.TorchDistAllgather(device=dev)
+    p = presets.get(args.config)
+    dsm, _ = loader.build_dsm(p, rank=rank, world=world, device=local, allgather=ag)
+    dg = DistributedGather(dsm)
+    ids = torch.from_numpy(seeds.gather_ids(p.n, args.sweep_ids, presets.SEED_BASE, rank)).to(dev)
+    out = torch.empty((ids.numel(), dsm.row_bytes), dtype=torch.uint8, device=dev)
+    flush = torch.empty(512 << 20, dtype=torch.uint8, device=dev)
+    res = {}
+    for name, fn in (("p2p_one_kernel", lambda: dsm.gather(ids, out=out)), ("distributed_five_step", lambda: dg.gather(ids, out=out))):
+        for _ in range(3):
+            fn()
+        ts = []
+        for i in range(args.steps):
+            flush.fill_(i & 0xFF)
+            if world > 1:
+                dist.barrier()
+            torch.cuda.synchronize()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record()
+            fn()
+            e1.record()
+            torch.cuda.synchronize()
+            ts.append(e0.elapsed_time(e1) / 1e3)
+        t = statistics.median(ts)
+        if world > 1:
+            tt = torch.tensor([t], dtype=torch.float64)
+            dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+            t = float(tt.item())
+        res[name] = {"ms": t * 1e3, "algo_gbs_per_gpu": ids.numel() * dsm.row_bytes / t / 1e9}
+    assert dsm.device_error() == 0
+    if rank == 0:
+        line = {"metric": "global gather: P2P (DSM, one kernel) vs distributed-memory five-step (Fig. 10 analogue)",
+                "value": res["distributed_five_step"]["ms"] / res["p2p_one_kernel"]["ms"], "unit": "x (time ratio)",
+                "higher_is_better": True, "n_gpus": world, "steps": args.steps,
+                "config": {"workload": p.name, "ids_per_rank": int(ids.numel()), "row_bytes": dsm.row_bytes,
+                           "exchange": "NCCL" if world > 1 and torch.cuda.device_count() >= world else
+                           ("gloo via host" if world > 1 else "local copy (W=1)")},
+                "results": res}
+        emit(line, args)
+    torch.cuda.synchronize()
+    dsm.destroy()
+    if world > 1:
+        dist.destroy_process_group()
+
+
 def main():
     args = parse()
-    if args.layer:
+    if args.compare_gather:
+        bench_compare_gather(args)
+    elif args.layer:
         bench_layer(args)
     elif args.latency:
         bench_latency(args)

@@ -197,6 +197,20 @@ wg_status wg_sample_hop(wg_dsm_t h, const int64_t* d_targets, int64_t n_targets,
 wg_status wg_gather(wg_dsm_t h, const int64_t* d_ids, int64_t n_ids, const int64_t* d_n_ids,
                     void* d_out, wg_stream_t stream);
 
+/* ---- Distributed-memory global gather: the comparison baseline (PAPER.md L178-180,
+ * Fig. 4 left, Fig. 10).  The caller drives the five steps with NCCL all-to-alls:
+ *   1 wg_bucket_by_owner  2 all-to-all counts + ids  3 wg_gather on the received ids
+ *   (all owned by this rank)  4 all-to-all features  5 wg_rows_permute.
+ * wg_bucket_by_owner: d_counts int64[2*W] (first W = ids per owner rank; the rest is
+ * scratch), d_bucketed_ids int64[n_ids] = the ids grouped by owner (rank 0's first; order
+ * within a group unspecified), d_perm int64[n_ids] = position of input i in the grouped
+ * array (-1 for an invalid id, which also latches WG_DEVERR_ID_RANGE).
+ * wg_rows_permute: d_dst[i] = d_src[d_perm[i]] for rows of row_bytes (zeros for -1). */
+wg_status wg_bucket_by_owner(wg_dsm_t h, const int64_t* d_ids, int64_t n_ids, const int64_t* d_n_ids,
+                             int64_t* d_counts, int64_t* d_bucketed_ids, int64_t* d_perm, wg_stream_t stream);
+wg_status wg_rows_permute(const void* d_src, void* d_dst, const int64_t* d_perm, int64_t n, int64_t row_bytes,
+                          wg_stream_t stream);
+
 /* ---- GNN layer op consuming the prepared mini-batch (III-C4) ----
  * g-SpMM with mean aggregation (GraphSAGE-mean message passing, Eq. (1)) on the
  * sub-graph CSR produced by one hop: rows = targets (d_row_ptr int64[n_rows+1], e.g.

@@ -56,6 +56,25 @@ def main():
         assert dsm.device_error() == 0
         dsm.destroy()
         print("PARITY OK", flush=True)
+    elif mode == "ncclgather":
+        import oracle
+        import paper_conf_sc_yanglql22_b200 as pkg
+        from paper_conf_sc_yanglql22_b200 import loader
+        from paper_conf_sc_yanglql22_b200.nccl_gather import DistributedGather
+        from synth import features, presets
+        torch.cuda.set_device(0)
+        p = presets.get("tiny")
+        ag = pkg.TorchDistAllgather()
+        dsm, _ = loader.build_dsm(p, rank=rank, world=world, allgather=ag, on_device=False)
+        ids = np.random.default_rng(rank).integers(0, p.n, 7000).astype(np.int64)
+        out = DistributedGather(dsm).gather(torch.from_numpy(ids).cuda())
+        direct = dsm.gather(torch.from_numpy(ids).cuda())
+        torch.cuda.synchronize()
+        exp = features.feature_bytes(presets.FEAT_SEED, ids, p.feat_dim, p.feat_dtype)
+        assert np.array_equal(out[:len(ids)].cpu().numpy(), exp)
+        assert np.array_equal(direct[:len(ids)].cpu().numpy(), exp)
+        dsm.destroy()
+        print("PARITY OK", flush=True)
     dist.destroy_process_group()
 
 

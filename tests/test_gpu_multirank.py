@@ -68,14 +68,16 @@ def test_virtual_ranks_w_invariance(W):
     _destroy_all(dsms)
 
 
-def test_two_processes_cuda_ipc():
+@pytest.mark.parametrize("mode", ["ipc", "ncclgather"])
+def test_two_processes_cuda_ipc(mode):
     """torchrun-style 2 ranks (gloo for the handle allgather) on the SAME GPU: rank 1
     reads rank 0's shard through cudaIpcOpenMemHandle and vice versa."""
-    env = dict(os.environ, MASTER_ADDR="127.0.0.1", MASTER_PORT=str(29500 + os.getpid() % 1000), WORLD_SIZE="2")
+    port = 29500 + os.getpid() % 1000 + (7 if mode != "ipc" else 0)
+    env = dict(os.environ, MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), WORLD_SIZE="2")
     procs = []
     for r in range(2):
         e = dict(env, RANK=str(r), LOCAL_RANK=str(r))
-        procs.append(subprocess.Popen([sys.executable, os.path.join(ROOT, "tests", "mp_worker.py"), "ipc"],
+        procs.append(subprocess.Popen([sys.executable, os.path.join(ROOT, "tests", "mp_worker.py"), mode],
                                       env=e, stdout=subprocess.PIPE, stderr=subprocess.STDOUT))
     outs = [p.communicate(timeout=600)[0].decode() for p in procs]
     for p, o in zip(procs, outs):

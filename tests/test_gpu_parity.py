@@ -328,3 +328,19 @@ def test_spmm_mean_forward_backward_vs_oracle(tiny):
     (out * dY).sum().backward()
     assert np.allclose(Xg.grad.cpu().numpy(), dXo, rtol=1e-5, atol=1e-5)
     dsm.destroy()
+
+
+def test_distributed_memory_gather_w1():
+    """NEXT #1 baseline (NCCL-style five-step gather) equals the P2P gather byte for byte."""
+    from paper_conf_sc_yanglql22_b200.nccl_gather import DistributedGather
+    n, dim = 5000, 100
+    rp = np.zeros(n + 1, dtype=np.int64)
+    feat = features.feature_bytes(presets.FEAT_SEED, np.arange(n), dim, "fp32")
+    dsm = make_dsm(rp, np.zeros(0, np.int64), feat, dim, "fp32")
+    ids = torch.from_numpy(np.random.default_rng(3).integers(0, n, 20000)).cuda()
+    a = dsm.gather(ids)
+    b = DistributedGather(dsm).gather(ids)
+    torch.cuda.synchronize()
+    assert torch.equal(a[:20000], b[:20000])
+    assert dsm.device_error() == 0
+    dsm.destroy()
