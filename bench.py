@@ -45,6 +45,8 @@ def parse():
     ap.add_argument("--sweep-ids", type=int, default=1_000_000)
     ap.add_argument("--latency", action="store_true", help="Table I analogue: dependent-load latency vs span")
     ap.add_argument("--layer", action="store_true", help="NEXT #2: g-SpMM mean aggregation on a prepared batch")
+    ap.add_argument("--pass-b", default="both", choices=["both", "prep", "gather"],
+                    help="diagnostics: run only the prep or only the gather in the throughput pass")
     ap.add_argument("--compare-gather", action="store_true", help="NEXT #1: P2P vs distributed-memory gather")
     ap.add_argument("--chase-accesses", type=int, default=100_000)
     return ap.parse_args()
@@ -317,8 +319,10 @@ def bench_wg(args):
         streams[j].wait_stream(main)
     for i in range(args.steps):
         for j in range(P):
-            launch(j, n_single + args.warmup + i * P + j, streams[j])
-            gather(j, streams[j])
+            if args.pass_b != "gather":
+                launch(j, n_single + args.warmup + i * P + j, streams[j])
+            if args.pass_b != "prep":
+                gather(j, streams[j])
     for j in range(P):
         main.wait_stream(streams[j])
     evB[1].record(main)
