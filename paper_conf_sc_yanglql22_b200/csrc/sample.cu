@@ -1,8 +1,8 @@
 // sample.cu -- multi-GPU sampling op (Algorithm 1).
 //
-// sample_kernel (no scan, no inter-block dependency): a group of G lanes (G = next
-// power of two >= M, 8..32) handles one target; each warp handles SAMPLE_UNR rounds
-// of 32/G targets at once, so every lane keeps SAMPLE_UNR independent neighbour loads
+// sample_kernel (no scan, no inter-block dependency): a group of G = max(M, 4) lanes
+// (fanout M <= 32) handles one target; each warp handles SAMPLE_UNR rounds
+// of floor(32/G) targets at once, so every lane keeps SAMPLE_UNR independent neighbour loads
 // in flight (the op is latency-bound: random 16 B row_ptr and 8 B col reads, local or
 // over NVLink).  Per target:
 //   - lane u of the group loads the (row_ptr[l], row_ptr[l+1]) pair of round u's
@@ -29,10 +29,12 @@
 namespace wg {
 
 constexpr int SAMPLE_THREADS = 256;
+constexpr int SAMPLE_UNR_MAX = 4;
 // SAMPLE_UNR = rounds per warp, all in flight at once (1, 2 or 4; chosen per launch: small hops use
 // fewer rounds per warp and therefore more blocks / SMs)
-template <int G, int SAMPLE_UNR>
-constexpr int sample_tile() { return (SAMPLE_THREADS / G) * SAMPLE_UNR; }  // targets per block
+// Lane groups are G = max(M, SAMPLE_UNR) lanes (not a power of two), so a warp holds
+// floor(32 / G) targets per round: e.g. 6 targets for M = 5, 3 for M = 10.
+__host__ __device__ inline int sample_group(int M) { return M > SAMPLE_UNR_MAX ? M : SAMPLE_UNR_MAX; }
 
 struct SampleArgs {
   ShardView s;
@@ -49,7 +51,7 @@ struct SampleArgs {
   unsigned* ctrl;
 };
 
-template <int G, int SAMPLE_UNR>
+template <int SAMPLE_UNR>
 __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs a) {
   __shared__ unsigned sm_chain[SAMPLE_THREADS / 32][32];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -61,17 +63,18 @@ __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs
       nT = nT < 0 ? 0 : a.cap;
     }
   }
-  constexpr int TPW = 32 / G;  // targets per warp per round
-  const int g = lane / G;      // target slot within the warp
-  const int i = lane % G;      // draw index
   const int M = a.M;
+  const int G = sample_group(M);
+  const int TPW = 32 / G;      // targets per warp per round
+  const int g = lane / G;      // target slot within the warp (g == TPW: leftover lanes, idle)
+  const int i = lane - g * G;  // draw index
   const int64_t warp_base = ((int64_t)blockIdx.x * (SAMPLE_THREADS / 32) + warp) * (TPW * SAMPLE_UNR);
   if (warp_base >= nT) return;  // warp-uniform
 
   // ---- row_ptr pairs: lane u of each group fetches round u's target (all in flight)
   int64_t my_v = -1, my_start = 0;
   unsigned my_deg = 0;
-  if (i < SAMPLE_UNR) {
+  if (i < SAMPLE_UNR && g < TPW) {
     const int64_t k = warp_base + (int64_t)i * TPW + g;
     if (k < nT) {
       my_v = a.targets[k];
@@ -106,7 +109,7 @@ __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs
     const int64_t tv = __shfl_sync(FULL_MASK, my_v, from);
     const int64_t tstart = __shfl_sync(FULL_MASK, my_start, from);
     const unsigned N = __shfl_sync(FULL_MASK, my_deg, from);
-    const bool active = k < nT && tv >= 0;
+    const bool active = g < TPW && k < nT && tv >= 0;
     const bool full = N <= (unsigned)M;
     const bool draw = active && !full && i < M;
     unsigned r = 0;
@@ -140,7 +143,7 @@ __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs
     if (ok[u]) owner_local(a.s, tv, o, l);
     src[u] = a.s.col[o] + tstart + pos[u];
     dst[u] = k * M + i;
-    if (i == 0 && k < nT) a.cnt[k] = active ? (int32_t)min(N, (unsigned)M) : 0;
+    if (i == 0 && g < TPW && k < nT) a.cnt[k] = active ? (int32_t)min(N, (unsigned)M) : 0;
   }
   int64_t nb[SAMPLE_UNR];
 #pragma unroll
@@ -362,19 +365,14 @@ cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap,
     else sample_block_kernel<1024><<<blocks, 1024, 0, st>>>(a);
     return cudaGetLastError();
   }
-  const int G = fanout <= 8 ? 8 : fanout <= 16 ? 16 : 32;
+  const int G = sample_group(fanout);
+  const int tpw = 32 / G;
   int unr = 4;  // largest of 4/2/1 that still gives >= 2 blocks per SM
-  while (unr > 1 && cap < (int64_t)(SAMPLE_THREADS / G) * unr * 2 * h->sm_count) unr >>= 1;
-  const int tile = (SAMPLE_THREADS / G) * unr;
+  while (unr > 1 && cap < (int64_t)(SAMPLE_THREADS / 32) * tpw * unr * 2 * h->sm_count) unr >>= 1;
+  const int64_t tile = (int64_t)(SAMPLE_THREADS / 32) * tpw * unr;
   const unsigned blocks = (unsigned)(cap > 0 ? (cap + tile - 1) / tile : 1);
-#define WG_SAMPLE_LAUNCH(GG, UU) sample_kernel<GG, UU><<<blocks, SAMPLE_THREADS, 0, st>>>(a)
-  if (G == 8) {
-    if (unr == 4) WG_SAMPLE_LAUNCH(8, 4); else if (unr == 2) WG_SAMPLE_LAUNCH(8, 2); else WG_SAMPLE_LAUNCH(8, 1);
-  } else if (G == 16) {
-    if (unr == 4) WG_SAMPLE_LAUNCH(16, 4); else if (unr == 2) WG_SAMPLE_LAUNCH(16, 2); else WG_SAMPLE_LAUNCH(16, 1);
-  } else {
-    if (unr == 4) WG_SAMPLE_LAUNCH(32, 4); else if (unr == 2) WG_SAMPLE_LAUNCH(32, 2); else WG_SAMPLE_LAUNCH(32, 1);
-  }
+#define WG_SAMPLE_LAUNCH(UU) sample_kernel<UU><<<blocks, SAMPLE_THREADS, 0, st>>>(a)
+  if (unr == 4) WG_SAMPLE_LAUNCH(4); else if (unr == 2) WG_SAMPLE_LAUNCH(2); else WG_SAMPLE_LAUNCH(1);
 #undef WG_SAMPLE_LAUNCH
   return cudaGetLastError();
 }
