@@ -102,12 +102,10 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueA
         key = a.T[q];
       } else if (PADDED) {
         const int64_t j = q - nT;
-        const int64_t k = j / a.M;
-        valid = (int)(j - k * a.M) < a.cnt[k];
-        if (valid)
-          key = a.nbrs[j];
-        else
-          a.slot_of[q] = SLOT_EMPTY;  // padding slot: no sample here
+        const unsigned k = a.Mdiv.div((unsigned)j);
+        key = a.nbrs[j];  // loaded together with the count (ignored for a padding slot)
+        valid = (int)((unsigned)j - k * (unsigned)a.M) < a.cnt[k];
+        if (!valid) a.slot_of[q] = SLOT_EMPTY;  // padding slot: no sample here
       } else {
         key = a.nbrs[q - nT];
       }
