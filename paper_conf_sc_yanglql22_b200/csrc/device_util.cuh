@@ -1,5 +1,5 @@
 // device_util.cuh -- device helpers of the CUDA path: Philox, warp/block scans,
-// single-pass decoupled look-back, cache-hinted vector loads.
+// look-back status format, last-block cleanup, cache-hinted vector loads, fast division.
 #pragma once
 
 #include <cuda_runtime.h>
@@ -90,39 +90,8 @@ __device__ __forceinline__ T block_exclusive_sum(T v, T* warp_tot, T* total) {
 // ---------------------------------------------------------------- decoupled look-back
 // Tile status word: bits 63..62 = flag (0 none, 1 aggregate, 2 inclusive prefix),
 // bits 61..0 = value.  Flag and value share one 64-bit word, so publication needs
-// no fence.  Called by ALL 32 lanes of one warp; returns the tile's exclusive
-// prefix in every lane and publishes the inclusive prefix.
+// no fence.  The block-wide look-back itself is in scan.cuh.
 constexpr unsigned long long LB_AGG = 1ull << 62, LB_PRE = 2ull << 62, LB_VAL = (1ull << 62) - 1;
-
-__device__ __forceinline__ unsigned long long tile_lookback(unsigned long long* status, long tile,
-                                                            unsigned long long aggregate) {
-  const int lane = threadIdx.x & 31;
-  if (tile == 0) {
-    if (lane == 0) st_volatile_u64(&status[0], LB_PRE | aggregate);
-    return 0;
-  }
-  if (lane == 0) st_volatile_u64(&status[tile], LB_AGG | aggregate);
-  unsigned long long excl = 0;
-  long pred = tile - 1;
-  for (;;) {
-    const long idx = pred - lane;
-    unsigned long long s = idx >= 0 ? ld_volatile_u64(&status[idx]) : LB_PRE;
-    while (__any_sync(FULL_MASK, (s >> 62) == 0)) {
-      if ((s >> 62) == 0) {
-        __nanosleep(20);
-        s = ld_volatile_u64(&status[idx]);
-      }
-    }
-    const unsigned pmask = __ballot_sync(FULL_MASK, (s >> 62) == 2);
-    const int stop = pmask ? __ffs(pmask) - 1 : 31;
-    unsigned long long v = lane <= stop ? (s & LB_VAL) : 0ull;
-    excl += warp_sum(v);
-    if (pmask) break;
-    pred -= 32;
-  }
-  if (lane == 0) st_volatile_u64(&status[tile], LB_PRE | (excl + aggregate));
-  return excl;
-}
 
 // Last-block cleanup: every block calls this once at its very end (all threads).
 // Returns true (in every thread of the block) for the block that finished last;

@@ -59,18 +59,6 @@ __device__ __forceinline__ long long hash_insert(const HashTable& t, unsigned lo
   return -1;
 }
 
-__device__ __forceinline__ long long hash_find(const HashTable& t, unsigned long long stored, unsigned epoch) {
-  unsigned long long slot = fmix64(stored & KEY_MASK) & t.mask;
-  for (unsigned long long probe = 0; probe <= t.mask; ++probe) {
-    const unsigned long long cur = t.slots[slot].key;
-    if (cur == stored) return (long long)slot;
-    if ((unsigned)(cur >> 40) != epoch) return -1;  // empty: not present
-    slot = (slot + 1) & t.mask;
-  }
-  return -1;
-}
-
-// Insert `key` at position q, recording the minimum position.  Returns the slot or -1.
 // The atomicMin is skipped when the value read with the key already holds a smaller
 // position of this epoch: hub ids occur thousands of times per hop, and this removes
 // most of the same-address atomics they would otherwise serialise on.
