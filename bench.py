@@ -38,7 +38,7 @@ def parse():
     ap.add_argument("--no-graph", action="store_true", help="launch ops eagerly instead of graph replay")
     ap.add_argument("--cpu-sample-s", type=float, default=12.0, help="target seconds of oracle work (cpu_baseline)")
     ap.add_argument("--e2e-steps", type=int, default=20)
-    ap.add_argument("--concurrency", type=int, default=4, help="independent batches in flight per GPU (streams)")
+    ap.add_argument("--concurrency", type=int, default=8, help="independent batches in flight per GPU (streams)")
     ap.add_argument("--out", default=None, help="also append the JSON line to this file")
     ap.add_argument("--sweep", action="store_true", help="config 4: feature-gather sweep over row sizes")
     ap.add_argument("--sweep-rows", type=int, default=100_000_000)

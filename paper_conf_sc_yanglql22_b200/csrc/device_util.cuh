@@ -9,6 +9,15 @@ namespace wg {
 
 constexpr unsigned FULL_MASK = 0xffffffffu;
 
+// Programmatic dependent launch: wait for the previous kernel of the stream (no-op when
+// the kernel was launched without the PDL attribute), then let the next one start.
+__device__ __forceinline__ void pdl_wait() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" :::); }
+__device__ __forceinline__ void pdl_enter() {
+  pdl_wait();
+  pdl_trigger();
+}
+
 // Philox4x32-10 (Salmon et al. SC'11), the counter-based generator of reading A3.
 __device__ __forceinline__ uint4 philox4x32_10(uint4 c, uint2 k) {
 #pragma unroll

@@ -24,6 +24,15 @@ namespace wg {
 
 static thread_local std::string g_last_error;
 
+bool pdl_enabled() {
+  static int on = -1;
+  if (on < 0) {
+    const char* e = getenv("WG_PDL");
+    on = (e && e[0] == '0') ? 0 : 1;
+  }
+  return on != 0;
+}
+
 void set_error(const std::string& msg) { g_last_error = msg; }
 wg_status fail(wg_status s, const std::string& msg) {
   g_last_error = msg;

@@ -43,6 +43,7 @@ struct GatherArgs {
 
 template <typename V, int GATHER_UNROLL>
 __global__ void __launch_bounds__(GATHER_THREADS) gather_kernel(const GatherArgs a) {
+  pdl_enter();
   int64_t n = a.cap;
   if (a.d_n) {
     n = *a.d_n;
@@ -98,6 +99,7 @@ __device__ __forceinline__ unsigned smem_u32(const void* p) {
 }
 
 __global__ void __launch_bounds__(32) gather_tma_kernel(const GatherArgs a, int rows_per_tile, int row_bytes) {
+  pdl_enter();
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ __align__(8) unsigned long long mbar[TMA_STAGES];
   const int lane = threadIdx.x;
@@ -239,14 +241,13 @@ cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int6
   blocks = blocks < 1 ? 1 : (blocks > max_blocks ? max_blocks : blocks);
   const unsigned gb = (unsigned)blocks;
   if (unroll == 8) {
-    if (vb == 16) gather_kernel<uint4, 8><<<gb, GATHER_THREADS, 0, st>>>(a);
-    else if (vb == 4) gather_kernel<unsigned, 8><<<gb, GATHER_THREADS, 0, st>>>(a);
-    else gather_kernel<unsigned short, 8><<<gb, GATHER_THREADS, 0, st>>>(a);
-  } else {
-    if (vb == 16) gather_kernel<uint4, 4><<<gb, GATHER_THREADS, 0, st>>>(a);
-    else if (vb == 4) gather_kernel<unsigned, 4><<<gb, GATHER_THREADS, 0, st>>>(a);
-    else gather_kernel<unsigned short, 4><<<gb, GATHER_THREADS, 0, st>>>(a);
+    if (vb == 16) return launch_pdl(gather_kernel<uint4, 8>, gb, GATHER_THREADS, 0, st, a);
+    if (vb == 4) return launch_pdl(gather_kernel<unsigned, 8>, gb, GATHER_THREADS, 0, st, a);
+    return launch_pdl(gather_kernel<unsigned short, 8>, gb, GATHER_THREADS, 0, st, a);
   }
+  if (vb == 16) return launch_pdl(gather_kernel<uint4, 4>, gb, GATHER_THREADS, 0, st, a);
+  if (vb == 4) return launch_pdl(gather_kernel<unsigned, 4>, gb, GATHER_THREADS, 0, st, a);
+  return launch_pdl(gather_kernel<unsigned short, 4>, gb, GATHER_THREADS, 0, st, a);
   return cudaGetLastError();
 }
 

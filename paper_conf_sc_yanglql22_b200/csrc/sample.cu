@@ -53,6 +53,7 @@ struct SampleArgs {
 
 template <int SAMPLE_UNR>
 __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs a) {
+  pdl_enter();
   __shared__ unsigned sm_chain[SAMPLE_THREADS / 32][32];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   int64_t nT = a.cap;
@@ -165,6 +166,7 @@ __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs
 // last in shared memory and path doubling as ceil(log2 M) synchronous rounds.
 template <int BT>
 __global__ void __launch_bounds__(BT) sample_block_kernel(const SampleArgs a) {
+  pdl_enter();
   __shared__ unsigned long long s_key[BT];
   __shared__ unsigned s_r[BT], s_chain[BT], s_q[BT], s_last[BT];
   __shared__ int64_t s_v, s_start;
@@ -300,6 +302,7 @@ struct CompactArgs {
 };
 
 __global__ void __launch_bounds__(COMPACT_THREADS) sample_compact_kernel(const CompactArgs a) {
+  pdl_enter();
   __shared__ LookbackSmem<COMPACT_THREADS> lb;
   __shared__ int sm_wtot[COMPACT_THREADS / 32 + 1];
   __shared__ int sm_flag;
@@ -358,12 +361,11 @@ cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap,
   a.ctrl = h->ws.ctrl;
   if (fanout > 32) {  // block per target (Algorithm 1 with a block sort)
     const unsigned blocks = (unsigned)(cap > 0 ? cap : 1);
-    if (fanout <= 64) sample_block_kernel<64><<<blocks, 64, 0, st>>>(a);
-    else if (fanout <= 128) sample_block_kernel<128><<<blocks, 128, 0, st>>>(a);
-    else if (fanout <= 256) sample_block_kernel<256><<<blocks, 256, 0, st>>>(a);
-    else if (fanout <= 512) sample_block_kernel<512><<<blocks, 512, 0, st>>>(a);
-    else sample_block_kernel<1024><<<blocks, 1024, 0, st>>>(a);
-    return cudaGetLastError();
+    if (fanout <= 64) return launch_pdl(sample_block_kernel<64>, blocks, 64, 0, st, a);
+    if (fanout <= 128) return launch_pdl(sample_block_kernel<128>, blocks, 128, 0, st, a);
+    if (fanout <= 256) return launch_pdl(sample_block_kernel<256>, blocks, 256, 0, st, a);
+    if (fanout <= 512) return launch_pdl(sample_block_kernel<512>, blocks, 512, 0, st, a);
+    return launch_pdl(sample_block_kernel<1024>, blocks, 1024, 0, st, a);
   }
   const int G = sample_group(fanout);
   const int tpw = 32 / G;
@@ -371,10 +373,9 @@ cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap,
   while (unr > 1 && cap < (int64_t)(SAMPLE_THREADS / 32) * tpw * unr * 2 * h->sm_count) unr >>= 1;
   const int64_t tile = (int64_t)(SAMPLE_THREADS / 32) * tpw * unr;
   const unsigned blocks = (unsigned)(cap > 0 ? (cap + tile - 1) / tile : 1);
-#define WG_SAMPLE_LAUNCH(UU) sample_kernel<UU><<<blocks, SAMPLE_THREADS, 0, st>>>(a)
-  if (unr == 4) WG_SAMPLE_LAUNCH(4); else if (unr == 2) WG_SAMPLE_LAUNCH(2); else WG_SAMPLE_LAUNCH(1);
-#undef WG_SAMPLE_LAUNCH
-  return cudaGetLastError();
+  if (unr == 4) return launch_pdl(sample_kernel<4>, blocks, SAMPLE_THREADS, 0, st, a);
+  if (unr == 2) return launch_pdl(sample_kernel<2>, blocks, SAMPLE_THREADS, 0, st, a);
+  return launch_pdl(sample_kernel<1>, blocks, SAMPLE_THREADS, 0, st, a);
 }
 
 cudaError_t launch_sample(wg_dsm* h, const int64_t* targets, int64_t cap, const int64_t* d_n, int fanout,
@@ -385,8 +386,7 @@ cudaError_t launch_sample(wg_dsm* h, const int64_t* targets, int64_t cap, const 
   CompactArgs c{cap, d_n, fanout, h->ws.nbrs_pad, h->ws.pos_pad, h->ws.cnt, out_row_ptr, out_nbrs, out_pos,
                 d_num_edges, h->ws.status_sample, h->ws.ctrl};
   const unsigned blocks = (unsigned)(cap > 0 ? (cap + COMPACT_TILE - 1) / COMPACT_TILE : 1);
-  sample_compact_kernel<<<blocks, COMPACT_THREADS, 0, st>>>(c);
-  return cudaGetLastError();
+  return launch_pdl(sample_compact_kernel, blocks, COMPACT_THREADS, 0, st, c);
 }
 
 }  // namespace wg

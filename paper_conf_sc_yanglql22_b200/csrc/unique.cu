@@ -86,6 +86,7 @@ __device__ __forceinline__ void load_counts(const UniqueArgs& a, int64_t& nT, in
 
 template <bool PADDED>
 __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueArgs a) {
+  pdl_enter();
   int64_t nT, nE;
   load_counts<PADDED>(a, nT, nE);
   const unsigned epoch = a.ctrl[CTRL_EPOCH];
@@ -150,6 +151,7 @@ __device__ __forceinline__ int64_t min_pos_at(const UniqueArgs& a, int32_t slot)
 
 template <bool PADDED, int UQ_ITEMS>
 __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArgs a) {
+  pdl_enter();
   // warp-striped: warp w of the tile covers 32 * UQ_ITEMS consecutive positions, lane l the
   // positions l, l+32, ...; every load and store instruction touches 32 consecutive elements,
   // and the in-warp scans are ballots + popc.
@@ -261,6 +263,7 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArg
 
 // sub_col[p] = id of neighbour p; d_nE = the dense neighbour count.
 __global__ void __launch_bounds__(UQ_THREADS) unique_relabel_kernel(const UniqueArgs a) {
+  pdl_enter();
   const int64_t nT = clamp_count(a.d_nT, a.capT, a.ctrl);
   int64_t nE = a.d_nE ? *a.d_nE : a.capE;
   nE = nE < 0 ? 0 : (nE > a.capE ? a.capE : nE);
@@ -290,23 +293,27 @@ static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, c
   while (items > 1 && a.capE < (int64_t)items * UQ_THREADS * 2 * h->sm_count) items >>= 1;
   const int64_t tile = (int64_t)items * UQ_THREADS;
   const unsigned fb = (unsigned)(a.capE > 0 ? (a.capE + tile - 1) / tile : 1);
+  cudaError_t e;
   if (padded) {
-    unique_insert_kernel<true><<<(unsigned)ib, UQ_THREADS, 0, st>>>(a);
+    e = launch_pdl(unique_insert_kernel<true>, (unsigned)ib, UQ_THREADS, 0, st, a);
+    if (e != cudaSuccess) return e;
     switch (items) {
-      case 8: unique_flag_kernel<true, 8><<<fb, UQ_THREADS, 0, st>>>(a); break;
-      case 4: unique_flag_kernel<true, 4><<<fb, UQ_THREADS, 0, st>>>(a); break;
-      case 2: unique_flag_kernel<true, 2><<<fb, UQ_THREADS, 0, st>>>(a); break;
-      default: unique_flag_kernel<true, 1><<<fb, UQ_THREADS, 0, st>>>(a); break;
+      case 8: e = launch_pdl(unique_flag_kernel<true, 8>, fb, UQ_THREADS, 0, st, a); break;
+      case 4: e = launch_pdl(unique_flag_kernel<true, 4>, fb, UQ_THREADS, 0, st, a); break;
+      case 2: e = launch_pdl(unique_flag_kernel<true, 2>, fb, UQ_THREADS, 0, st, a); break;
+      default: e = launch_pdl(unique_flag_kernel<true, 1>, fb, UQ_THREADS, 0, st, a); break;
     }
   } else {
-    unique_insert_kernel<false><<<(unsigned)ib, UQ_THREADS, 0, st>>>(a);
+    e = launch_pdl(unique_insert_kernel<false>, (unsigned)ib, UQ_THREADS, 0, st, a);
+    if (e != cudaSuccess) return e;
     switch (items) {
-      case 8: unique_flag_kernel<false, 8><<<fb, UQ_THREADS, 0, st>>>(a); break;
-      case 4: unique_flag_kernel<false, 4><<<fb, UQ_THREADS, 0, st>>>(a); break;
-      case 2: unique_flag_kernel<false, 2><<<fb, UQ_THREADS, 0, st>>>(a); break;
-      default: unique_flag_kernel<false, 1><<<fb, UQ_THREADS, 0, st>>>(a); break;
+      case 8: e = launch_pdl(unique_flag_kernel<false, 8>, fb, UQ_THREADS, 0, st, a); break;
+      case 4: e = launch_pdl(unique_flag_kernel<false, 4>, fb, UQ_THREADS, 0, st, a); break;
+      case 2: e = launch_pdl(unique_flag_kernel<false, 2>, fb, UQ_THREADS, 0, st, a); break;
+      default: e = launch_pdl(unique_flag_kernel<false, 1>, fb, UQ_THREADS, 0, st, a); break;
     }
   }
+  if (e != cudaSuccess) return e;
   if (a.capE > 0) {
     // relabel runs over the DENSE neighbours: count = num_edges (padded) or d_nE
     UniqueArgs r = a;

@@ -97,6 +97,27 @@ struct wg_dsm {
 };
 
 namespace wg {
+// Programmatic dependent launch (sm_90+): kernels of one op chain are launched with
+// ProgrammaticStreamSerialization, start their blocks while the previous kernel drains and
+// wait for its results with griddepcontrol.wait (pdl_wait) before touching memory.
+// WG_PDL=0 disables it (A/B switch); correctness never depends on it.
+bool pdl_enabled();
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                              Args... args) {
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = grid;
+  cfg.blockDim = block;
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
+}
+
 // launchers (stream-ordered); arguments already validated by the ABI layer
 cudaError_t launch_sample(wg_dsm* h, const int64_t* targets, int64_t cap, const int64_t* d_n, int fanout,
                           uint64_t seed, const uint64_t* d_seed, int hop, int64_t* out_row_ptr,
