@@ -109,6 +109,10 @@ static wg_status alloc_workspace(wg_dsm* h, int64_t max_keys) {
   WG_CUDA_TRY(cudaMemset(w.status_unique, 0, w.status_cap * 8));
   unsigned ctrl[CTRL_WORDS] = {0};
   ctrl[CTRL_EPOCH] = 1;
+  if (const char* e = getenv("WG_EPOCH_START")) {  // test hook: start near the end of the epoch space
+    const long v = atol(e);
+    if (v >= 1 && v < (long)EPOCH_MAX) ctrl[CTRL_EPOCH] = (unsigned)v;
+  }
   WG_CUDA_TRY(cudaMemcpy(w.ctrl, ctrl, sizeof(ctrl), cudaMemcpyHostToDevice));
   return WG_OK;
 }

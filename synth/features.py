@@ -37,7 +37,7 @@ def feature_bits(feat_seed: int, v, dim: int, dtype: str) -> np.ndarray:
 def feature_bytes(feat_seed: int, v, dim: int, dtype: str) -> np.ndarray:
     """Row bytes [len(v), dim*elt] (uint8) of nodes v."""
     b = feature_bits(feat_seed, v, dim, dtype)
-    return b.view(np.uint8).reshape(b.shape[0], -1)
+    return b.view(np.uint8).reshape(b.shape[0], dim * DTYPES[dtype][0])
 
 
 def feature_bytes_native(feat_seed: int, v, dim: int, dtype: str) -> np.ndarray:

@@ -344,3 +344,66 @@ def test_distributed_memory_gather_w1():
     assert torch.equal(a[:20000], b[:20000])
     assert dsm.device_error() == 0
     dsm.destroy()
+
+
+def test_pipeline_degenerate_batches(tiny):
+    """Empty seed list, a single seed, seeds whose rows are empty: device counts of 0 flow
+    through every kernel of the captured graph."""
+    p, rp, col = tiny
+    n = 64
+    rows = [[] for _ in range(n)]
+    rows[5] = [6, 7]
+    rows[6] = [5]
+    g_rp, g_col = csr_from_rows(rows)
+    feat = features.feature_bytes(presets.FEAT_SEED, np.arange(n), 8, "fp32")
+    dsm = make_dsm(g_rp, g_col, feat, 8, "fp32", max_keys=4096)
+    pipe = pkg.MiniBatchPipeline(dsm, [3, 2], 16, with_pos=True, with_dup=True)
+    rowsf = loader.host_row_provider(None, g_rp, g_col)
+
+    def feats(ids):
+        u = np.unique(np.asarray(ids, dtype=np.int64))
+        return u, features.feature_bytes(presets.FEAT_SEED, u, 8, "fp32")
+    pipe.run(torch.from_numpy(np.array([1], np.int64)).cuda(), 3)
+    torch.cuda.synchronize()
+    pipe.capture()
+    for S in (np.zeros(0, np.int64), np.array([0, 1, 2], np.int64), np.array([5], np.int64), np.array([9, 5, 6], np.int64)):
+        pipe.run(torch.from_numpy(S).cuda() if len(S) else torch.zeros(0, dtype=torch.int64, device="cuda"), 11)
+        torch.cuda.synchronize()
+        ref = oracle.minibatch(rowsf, feats, S, [3, 2], 11)
+        _check_batch(pipe, ref, [3, 2])
+    assert dsm.device_error() == 0
+    dsm.destroy()
+
+
+def test_epoch_exhaustion_and_reset(tiny):
+    """The hash-table epoch space: near its end an op latches WG_DEVERR_EPOCH;
+    wg_dsm_reset_workspace restores correct operation (test hook WG_EPOCH_START)."""
+    import os
+    import subprocess
+    import sys
+    code = r'''
+import sys, numpy as np, torch
+sys.path.insert(0, "tests")
+import oracle
+from gpu_helpers import make_dsm, gpu_unique
+T = np.array([4, 9], np.int64); nb = np.array([1, 4, 1, 7], np.int64)
+rp = np.zeros(11, np.int64)
+dsm = make_dsm(rp, np.zeros(0, np.int64), max_keys=64)
+U, sc, dup = gpu_unique(dsm, T, nb)          # uses epoch EPOCH_MAX-2 -> bumps to EPOCH_MAX-1
+assert list(U) == [4, 9, 1, 7] and dsm.device_error() == 0
+gpu_unique(dsm, T, nb)                       # epoch + 1 would reach EPOCH_MAX: latched
+assert dsm.device_error() & 0x10
+dsm.reset_workspace(); torch.cuda.synchronize()
+for _ in range(3):
+    U, sc, dup = gpu_unique(dsm, T, nb)
+    Uo, sco, dupo = oracle.append_unique(T, nb)
+    assert np.array_equal(U, Uo) and np.array_equal(sc, sco) and np.array_equal(dup, dupo)
+assert dsm.device_error() == 0
+dsm.destroy()
+print("EPOCH OK")
+'''
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", code], cwd=root,
+                       env=dict(os.environ, WG_EPOCH_START=str((1 << 23) - 3)), capture_output=True, text=True,
+                       timeout=600)
+    assert r.returncode == 0 and "EPOCH OK" in r.stdout, r.stdout + r.stderr
