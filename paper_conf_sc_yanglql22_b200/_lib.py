@@ -51,6 +51,7 @@ def lib():
     L.wg_append_unique.argtypes = [P, P, I64, P, P, I64, P, P, P, P, P, P]
     L.wg_sample_hop.argtypes = [P, P, I64, P, I32, U64, P, I32, P, P, P, P, P, P, P, P, P, P]
     L.wg_gather.argtypes = [P, P, I64, P, P, P]
+    L.wg_gather_rows.argtypes = [P, P, I64, P, P, P, P]
     L.wg_dsm_chase.argtypes = [P, I32, I64, I64, P, P]
     L.wg_bucket_by_owner.argtypes = [P, P, I64, P, P, P, P, P]
     L.wg_rows_permute.argtypes = [P, P, P, I64, I64, P]
@@ -59,7 +60,7 @@ def lib():
     L.wg_device_error.argtypes = [P, P, I32]
     L.wg_dsm_reset_workspace.argtypes = [P, P]
     for f in ("wg_dsm_create", "wg_dsm_fork", "wg_dsm_local_view", "wg_dsm_shard_info", "wg_dsm_destroy", "wg_sample_neighbors",
-              "wg_append_unique", "wg_sample_hop", "wg_gather", "wg_dsm_chase", "wg_spmm_mean_forward",
+              "wg_append_unique", "wg_sample_hop", "wg_gather", "wg_gather_rows", "wg_dsm_chase", "wg_spmm_mean_forward",
            "wg_spmm_mean_backward", "wg_bucket_by_owner", "wg_rows_permute", "wg_spmm_mean_forward",
               "wg_spmm_mean_backward", "wg_bucket_by_owner", "wg_rows_permute", "wg_dsm_chase", "wg_device_error", "wg_dsm_reset_workspace"):
         getattr(L, f).restype = ctypes.c_int
@@ -77,6 +78,6 @@ def check(status):
 
 
 EXPORTS = ["wg_dsm_create", "wg_dsm_fork", "wg_dsm_local_view", "wg_dsm_shard_info", "wg_dsm_destroy", "wg_sample_neighbors",
-           "wg_append_unique", "wg_sample_hop", "wg_gather", "wg_dsm_chase", "wg_spmm_mean_forward",
+           "wg_append_unique", "wg_sample_hop", "wg_gather", "wg_gather_rows", "wg_dsm_chase", "wg_spmm_mean_forward",
            "wg_spmm_mean_backward", "wg_bucket_by_owner", "wg_rows_permute", "wg_device_error", "wg_dsm_reset_workspace", "wg_last_error",
            "wg_version"]

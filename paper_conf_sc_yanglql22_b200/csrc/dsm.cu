@@ -416,8 +416,8 @@ wg_status wg_sample_hop(wg_dsm_t h, const int64_t* d_targets, int64_t n_targets,
   return WG_OK;
 }
 
-wg_status wg_gather(wg_dsm_t h, const int64_t* d_ids, int64_t n_ids, const int64_t* d_n_ids, void* d_out,
-                    wg_stream_t stream) {
+wg_status wg_gather_rows(wg_dsm_t h, const int64_t* d_ids, int64_t n_ids, const int64_t* d_begin,
+                         const int64_t* d_end, void* d_out, wg_stream_t stream) {
   if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
   if (n_ids < 0 || (n_ids > 0 && (!d_ids || !d_out))) return fail(WG_ERR_INVALID_ARG, "null pointer or negative size");
   if (h->row_bytes == 0) return fail(WG_ERR_INVALID_ARG, "DSM has no feature table");
@@ -426,10 +426,15 @@ wg_status wg_gather(wg_dsm_t h, const int64_t* d_ids, int64_t n_ids, const int64
   if (n_ids * (h->row_bytes / 2) >= (int64_t(1) << 31) || n_ids * (h->row_bytes / vb) >= (int64_t(1) << 31))
     return fail(WG_ERR_UNSUPPORTED, "gather too large for one launch (split the id list)");
   cudaSetDevice(h->device);
-  if (n_ids == 0 && !d_n_ids) return WG_OK;
-  cudaError_t e = launch_gather(h, d_ids, n_ids, d_n_ids, d_out, (cudaStream_t)stream);
+  if (n_ids == 0 && !d_end) return WG_OK;
+  cudaError_t e = launch_gather(h, d_ids, n_ids, d_end, d_begin, d_out, (cudaStream_t)stream);
   if (e != cudaSuccess) return fail(WG_ERR_CUDA, std::string("gather launch: ") + cudaGetErrorString(e));
   return WG_OK;
+}
+
+wg_status wg_gather(wg_dsm_t h, const int64_t* d_ids, int64_t n_ids, const int64_t* d_n_ids, void* d_out,
+                    wg_stream_t stream) {
+  return wg_gather_rows(h, d_ids, n_ids, nullptr, d_n_ids, d_out, stream);
 }
 
 wg_status wg_device_error(wg_dsm_t h, uint32_t* code, int32_t clear) {

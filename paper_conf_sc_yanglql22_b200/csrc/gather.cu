@@ -36,6 +36,7 @@ struct GatherArgs {
   const int64_t* ids;
   int64_t cap;
   const int64_t* d_n;
+  const int64_t* d_begin;  // nullable: first row (rows [begin, n) of ids / out are processed)
   uint8_t* out;
   unsigned* ctrl;
   FastDiv cpr;  // chunks per row
@@ -52,10 +53,14 @@ __global__ void __launch_bounds__(GATHER_THREADS) gather_kernel(const GatherArgs
       n = n < 0 ? 0 : a.cap;
     }
   }
+  int64_t begin = a.d_begin ? *a.d_begin : 0;
+  begin = begin < 0 ? 0 : (begin > n ? n : begin);
+  const int64_t* __restrict__ ids = a.ids + begin;
+  n -= begin;
   const unsigned cpr = a.cpr.d;
   const unsigned total = (unsigned)(n * cpr);  // < 2^31 (checked on the host)
   const unsigned stride = gridDim.x * GATHER_THREADS;
-  V* __restrict__ out = reinterpret_cast<V*>(a.out);
+  V* __restrict__ out = reinterpret_cast<V*>(a.out + begin * (int64_t)cpr * (int64_t)sizeof(V));
   for (unsigned c0 = blockIdx.x * GATHER_THREADS + threadIdx.x; c0 < total; c0 += stride * GATHER_UNROLL) {
     V val[GATHER_UNROLL];
     unsigned dst[GATHER_UNROLL];
@@ -66,7 +71,7 @@ __global__ void __launch_bounds__(GATHER_THREADS) gather_kernel(const GatherArgs
       if (c < total) {
         const unsigned row = a.cpr.div(c);
         const unsigned colc = c - row * cpr;
-        const int64_t v = a.ids[row];
+        const int64_t v = ids[row];
         if (v >= 0 && v < a.s.n) {
           int o;
           int64_t l;
@@ -111,6 +116,11 @@ __global__ void __launch_bounds__(32) gather_tma_kernel(const GatherArgs a, int 
       n = n < 0 ? 0 : a.cap;
     }
   }
+  int64_t begin = a.d_begin ? *a.d_begin : 0;
+  begin = begin < 0 ? 0 : (begin > n ? n : begin);
+  const int64_t* ids = a.ids + begin;
+  uint8_t* outp = a.out + begin * (int64_t)row_bytes;
+  n -= begin;
   const int R = rows_per_tile;
   const int64_t ntiles = (n + R - 1) / R;
   if (lane == 0) {
@@ -127,7 +137,7 @@ __global__ void __launch_bounds__(32) gather_tma_kernel(const GatherArgs a, int 
     bool ok = false;
     const uint8_t* src = nullptr;
     if (lane < rows) {
-      const int64_t v = a.ids[r0 + lane];
+      const int64_t v = ids[r0 + lane];
       if (v >= 0 && v < a.s.n) {
         int o;
         int64_t l;
@@ -173,7 +183,7 @@ __global__ void __launch_bounds__(32) gather_tma_kernel(const GatherArgs a, int 
     const int rows = (int)min((int64_t)R, n - r0);
     uint8_t* stage = smem + (size_t)s * R * row_bytes;
     if (lane == 0) {
-      asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(a.out + r0 * row_bytes),
+      asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(outp + r0 * row_bytes),
                    "r"(smem_u32(stage)), "r"((unsigned)(rows * row_bytes))
                    : "memory");
       asm volatile("cp.async.bulk.commit_group;" ::: "memory");
@@ -186,11 +196,11 @@ __global__ void __launch_bounds__(32) gather_tma_kernel(const GatherArgs a, int 
   if (lane == 0) asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
 }
 
-cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int64_t* d_n, void* out,
-                          cudaStream_t st) {
+cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int64_t* d_n, const int64_t* d_begin,
+                          void* out, cudaStream_t st) {
   const int64_t rb = h->row_bytes;
   int vb = (rb % 16 == 0 && ((uintptr_t)out % 16) == 0) ? 16 : (rb % 4 == 0 && ((uintptr_t)out % 4) == 0) ? 4 : 2;
-  GatherArgs a{h->view, ids, cap, d_n, static_cast<uint8_t*>(out), h->ws.ctrl, FastDiv((unsigned)(rb / vb))};
+  GatherArgs a{h->view, ids, cap, d_n, d_begin, static_cast<uint8_t*>(out), h->ws.ctrl, FastDiv((unsigned)(rb / vb))};
   const int64_t total = cap * (rb / vb);
   // knobs (read once): WG_GATHER_UNROLL = independent 16 B loads in flight per thread (4 or 8),
   // WG_GATHER_BPS = resident blocks per SM to use (0 = as many as fit: one full wave)

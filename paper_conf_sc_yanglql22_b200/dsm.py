@@ -244,6 +244,12 @@ class DSM:
                                   _stream(side_stream) if side_stream is not None else None))
         return o
 
+    def gather_rows(self, ids, cap, begin_dev, end_dev, out, stream=None):
+        """Rows [*begin_dev, *end_dev) of ids -> the same rows of out (wg_gather_rows)."""
+        check(lib().wg_gather_rows(self.h, _ptr(ids), cap, _ptr(begin_dev), _ptr(end_dev), _ptr(out),
+                                   _stream(stream)))
+        return out
+
     def gather(self, ids, n_ids=None, n_ids_dev=None, out=None, stream=None):
         """Global gather: out[i] = feature row of ids[i] (uint8 rows)."""
         n = ids.numel() if n_ids is None else n_ids

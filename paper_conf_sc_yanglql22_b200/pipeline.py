@@ -31,10 +31,15 @@ def required_keys(n, fanouts, max_seeds):
 
 
 class MiniBatchPipeline:
-    def __init__(self, dsm: DSM, fanouts, max_seeds, with_pos=False, with_dup=False, fused=True):
+    def __init__(self, dsm: DSM, fanouts, max_seeds, with_pos=False, with_dup=False, fused=True,
+                 incremental_gather=True):
         self.dsm, self.fanouts, self.max_seeds = dsm, list(fanouts), max_seeds
         self.fused = fused
         self.side = torch.cuda.Stream(device=dsm.device) if fused else None
+        # incremental gather: U_{h-1} is a prefix of U_h, so the feature rows of hop h's new nodes
+        # are gathered on gside while hop h+1 samples; only the last hop's new rows remain at the end
+        self.incremental = incremental_gather
+        self.gside = torch.cuda.Stream(device=dsm.device) if incremental_gather else None
         self.with_pos, self.with_dup = with_pos, with_dup
         dev = dsm.device
         self.T_cap, self.E_cap, self.U_cap = capacities(dsm.num_nodes, fanouts, max_seeds)
@@ -68,6 +73,8 @@ class MiniBatchPipeline:
         if self.fused:
             self.side.wait_stream(main)
         tgt, tcap, tn = self.seeds, self.max_seeds, self.n_seeds
+        incr = gather and self.incremental and self.X is not None
+        prev_nu = None
         for h, m in enumerate(self.fanouts):
             b = self.hops[h]
             if self.fused:
@@ -80,11 +87,17 @@ class MiniBatchPipeline:
                 d.append_unique(tgt, b["nbrs"], n_targets=tcap, n_nbrs=self.E_cap[h], n_targets_dev=tn,
                                 n_nbrs_dev=b["num_edges"], out_unique=b["unique"], out_num_unique=b["num_unique"],
                                 out_sub_col=b["sub_col"], out_dup=b["dup"], stream=main)
+            if incr:  # rows [|U_{h-1}|, |U_h|) of X are final now
+                self.gside.wait_stream(main)
+                d.gather_rows(b["unique"], self.U_cap[h], prev_nu, b["num_unique"], self.X, stream=self.gside)
+                prev_nu = b["num_unique"]
             tgt, tcap, tn = b["unique"], self.U_cap[h], b["num_unique"]
-        if gather and self.X is not None:
+        if gather and self.X is not None and not incr:
             self.enqueue_gather(main)
         if self.fused:
             main.wait_stream(self.side)
+        if incr:
+            main.wait_stream(self.gside)
 
     def enqueue_gather(self, stream=None):
         last = self.hops[-1]

@@ -32,14 +32,15 @@ def _check_batch(pipe, ref, fanouts):
     assert np.array_equal(pipe.features(), ref["X"])
 
 
-@pytest.mark.parametrize("fused", [True, False])
-def test_tiny_pipeline_many_batches(tiny, fused):
+@pytest.mark.parametrize("fused,incr", [(True, True), (False, True), (True, False)])
+def test_tiny_pipeline_many_batches(tiny, fused, incr):
     """Config 1 (10k nodes, [10,5], 512 seeds): 20 batches, every array bit-exact, through
     the fused hop (wg_sample_hop) and through the separate ops (wg_sample_neighbors +
     wg_append_unique)."""
     p, rp, col = tiny
     dsm, _ = loader.build_dsm(p, on_device=False)
-    pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True, fused=fused)
+    pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True, fused=fused,
+                                 incremental_gather=incr)
     rows = loader.host_row_provider(p.graph(), rp, col)
     feats = loader.host_feat_provider(p)
     for b in range(20):
