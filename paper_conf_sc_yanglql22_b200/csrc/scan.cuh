@@ -29,9 +29,29 @@ __device__ __forceinline__ unsigned long long block_lookback(unsigned long long*
     return 0ull;
   }
   if (tid == 0) st_volatile_u64(&status[tile], LB_AGG | aggregate);
-  unsigned long long excl = 0;
-  long pred = tile - 1;
-  for (;;) {
+  // fast path: warp 0 inspects the 32 closest predecessors (usually enough: tiles finish roughly
+  // in order); only if none of them holds an inclusive prefix does the whole block walk back
+  if (warp == 0) {
+    const long idx = tile - 1 - lane;
+    unsigned long long s = idx >= 0 ? ld_volatile_u64(&status[idx]) : LB_PRE;
+    while ((s >> 62) == 0) {
+      __nanosleep(32);
+      s = ld_volatile_u64(&status[idx]);
+    }
+    const unsigned pm = __ballot_sync(FULL_MASK, (s >> 62) == 2);
+    const int stop = pm ? __ffs(pm) - 1 : 31;
+    const unsigned long long v = warp_sum(lane <= stop ? (s & LB_VAL) : 0ull);
+    if (lane == 0) {
+      sm.part[0] = v;
+      sm.found = pm != 0;
+    }
+  }
+  __syncthreads();
+  unsigned long long excl = sm.part[0];
+  const bool fast = sm.found != 0;
+  __syncthreads();  // sm is reused below
+  long pred = tile - 33;
+  for (; !fast;) {
     const long idx = pred - tid;
     unsigned long long s = idx >= 0 ? ld_volatile_u64(&status[idx]) : LB_PRE;
     while ((s >> 62) == 0) {
