@@ -72,7 +72,7 @@ class ClockSampler:
     def start(self):
         try:
             self.proc = subprocess.Popen(["nvidia-smi", f"--id={self.gpu}", f"--query-gpu={self.Q}",
-                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                          "--format=csv,noheader,nounits", "-lms", "50"],
                                          stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
@@ -452,7 +452,9 @@ def bench_wg(args):
                     "d2h_bytes_per_step": int(d2h.numel() * 8),
                     "note": "public API (MiniBatchPipeline.run), one batch per step: pinned-host seeds H2D, "
                             "per-hop counts D2H, host-timed incl. sync"},
-            "gpu_launches": args.steps * (4 * len(p.fanouts) + 1) * (1 + P),
+            # our kernels per batch: 4 per hop (sample, insert, flag-scan, relabel) + the gather (pass A)
+            # or + one gather_rows per hop (the shipped incremental graph: passes A' and B)
+            "gpu_launches": args.steps * (4 * len(p.fanouts) + 1) + args.steps * (1 + P) * 5 * len(p.fanouts),
             "clocks": clk,
             "wall_s_timed_region": wall,
             "workload_stats": {"edges_per_hop_mean": hc[:, :, 0].mean(0).tolist(),
