@@ -20,8 +20,22 @@ namespace wg {
 
 constexpr int GATHER_THREADS = 256;
 
+// 32 B vectors (sm_100 LDG/STG.256) for rows that are multiples of 32 B
+struct __align__(32) u32x8 {
+  unsigned v[8];
+};
+
 template <typename V>
 __device__ __forceinline__ V ld_feat(const void* p);
+template <>
+__device__ __forceinline__ u32x8 ld_feat<u32x8>(const void* p) {
+  u32x8 r;
+  asm("ld.global.nc.L1::no_allocate.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+      : "=r"(r.v[0]), "=r"(r.v[1]), "=r"(r.v[2]), "=r"(r.v[3]), "=r"(r.v[4]), "=r"(r.v[5]), "=r"(r.v[6]),
+        "=r"(r.v[7])
+      : "l"(p));
+  return r;
+}
 template <>
 __device__ __forceinline__ uint4 ld_feat<uint4>(const void* p) { return ld_nc_na_v4(p); }
 
@@ -41,6 +55,17 @@ struct GatherArgs {
   unsigned* ctrl;
   FastDiv cpr;  // chunks per row
 };
+
+template <typename V>
+__device__ __forceinline__ void st_out(V* p, const V& v) {
+  *p = v;
+}
+template <>
+__device__ __forceinline__ void st_out<u32x8>(u32x8* p, const u32x8& r) {
+  asm volatile("st.global.v8.u32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "r"(r.v[0]), "r"(r.v[1]), "r"(r.v[2]),
+               "r"(r.v[3]), "r"(r.v[4]), "r"(r.v[5]), "r"(r.v[6]), "r"(r.v[7])
+               : "memory");
+}
 
 template <typename V, int GATHER_UNROLL>
 __global__ void __launch_bounds__(GATHER_THREADS) gather_kernel(const GatherArgs a) {
@@ -85,7 +110,7 @@ __global__ void __launch_bounds__(GATHER_THREADS) gather_kernel(const GatherArgs
     }
 #pragma unroll
     for (int j = 0; j < GATHER_UNROLL; ++j)
-      if (dst[j] < total) out[dst[j]] = val[j];
+      if (dst[j] < total) st_out<V>(&out[dst[j]], val[j]);
   }
 }
 
@@ -199,21 +224,23 @@ __global__ void __launch_bounds__(32) gather_tma_kernel(const GatherArgs a, int 
 cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int64_t* d_n, const int64_t* d_begin,
                           void* out, cudaStream_t st) {
   const int64_t rb = h->row_bytes;
-  int vb = (rb % 16 == 0 && ((uintptr_t)out % 16) == 0) ? 16 : (rb % 4 == 0 && ((uintptr_t)out % 4) == 0) ? 4 : 2;
-  GatherArgs a{h->view, ids, cap, d_n, d_begin, static_cast<uint8_t*>(out), h->ws.ctrl, FastDiv((unsigned)(rb / vb))};
-  const int64_t total = cap * (rb / vb);
-  // knobs (read once): WG_GATHER_UNROLL = independent 16 B loads in flight per thread (4 or 8),
-  // WG_GATHER_BPS = resident blocks per SM to use (0 = as many as fit: one full wave)
-  static int unroll = 0, bps = -1, use_tma = 0;
-  if (unroll == 0) {
-    const char* u = getenv("WG_GATHER_UNROLL");
-    unroll = (u && atoi(u) == 8) ? 8 : 4;
+  static int knobs = 0, bps = 0, use_tma = 0, allow32 = 1;
+  if (!knobs) {  // A/B knobs, read once: WG_GATHER_BPS (blocks per SM), WG_GATHER_TMA=1, WG_GATHER_V32=0
     const char* b = getenv("WG_GATHER_BPS");
     bps = b ? atoi(b) : 0;
     const char* t = getenv("WG_GATHER_TMA");
     use_tma = (t && t[0] == '1') ? 1 : 0;
+    const char* v = getenv("WG_GATHER_V32");
+    allow32 = (v && v[0] == '0') ? 0 : 1;
+    knobs = 1;
   }
-  if (use_tma && vb == 16 && rb <= TMA_STAGE_BYTES) {
+  const uintptr_t oa = (uintptr_t)out;
+  const int vb = (allow32 && rb % 32 == 0 && oa % 32 == 0) ? 32
+                 : (rb % 16 == 0 && oa % 16 == 0)           ? 16
+                 : (rb % 4 == 0 && oa % 4 == 0)             ? 4
+                                                            : 2;
+  GatherArgs a{h->view, ids, cap, d_n, d_begin, static_cast<uint8_t*>(out), h->ws.ctrl, FastDiv((unsigned)(rb / vb))};
+  if (use_tma && rb % 16 == 0 && oa % 16 == 0 && rb <= TMA_STAGE_BYTES) {
     const int R = (int)std::min<int64_t>(32, TMA_STAGE_BYTES / rb);
     const int smem = TMA_STAGES * R * (int)rb;
     static int tma_bps = 0;
@@ -229,36 +256,27 @@ cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int6
     gather_tma_kernel<<<(unsigned)gbk, 32, smem, st>>>(a, R, (int)rb);
     return cudaGetLastError();
   }
-  int64_t blocks = (total + GATHER_THREADS * unroll - 1) / (GATHER_THREADS * unroll);
-  static int occ[2][3] = {{0, 0, 0}, {0, 0, 0}};
-  const int which = vb == 16 ? 0 : (vb == 4 ? 1 : 2);
-  const int ui = unroll == 8 ? 1 : 0;
-  if (!occ[ui][which]) {
+  // one full wave: resident blocks per SM (occupancy calculator, cached per vector width) x SMs
+  static int occ[4] = {0, 0, 0, 0};
+  const int which = vb == 32 ? 0 : vb == 16 ? 1 : vb == 4 ? 2 : 3;
+  if (!occ[which]) {
     int nb = 0;
-    if (unroll == 8) {
-      if (vb == 16) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<uint4, 8>, GATHER_THREADS, 0);
-      else if (vb == 4) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<unsigned, 8>, GATHER_THREADS, 0);
-      else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<unsigned short, 8>, GATHER_THREADS, 0);
-    } else {
-      if (vb == 16) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<uint4, 4>, GATHER_THREADS, 0);
-      else if (vb == 4) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<unsigned, 4>, GATHER_THREADS, 0);
-      else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<unsigned short, 4>, GATHER_THREADS, 0);
-    }
-    occ[ui][which] = nb > 0 ? nb : 4;
+    if (vb == 32) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<u32x8, 4>, GATHER_THREADS, 0);
+    else if (vb == 16) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<uint4, 4>, GATHER_THREADS, 0);
+    else if (vb == 4) cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<unsigned, 4>, GATHER_THREADS, 0);
+    else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<unsigned short, 4>, GATHER_THREADS, 0);
+    occ[which] = nb > 0 ? nb : 4;
   }
-  const int per_sm = (bps > 0 && bps < occ[ui][which]) ? bps : occ[ui][which];
+  const int per_sm = (bps > 0 && bps < occ[which]) ? bps : occ[which];
+  const int64_t total = cap * (rb / vb);
+  int64_t blocks = (total + GATHER_THREADS * 4 - 1) / (GATHER_THREADS * 4);
   const int64_t max_blocks = (int64_t)h->sm_count * per_sm;
   blocks = blocks < 1 ? 1 : (blocks > max_blocks ? max_blocks : blocks);
   const unsigned gb = (unsigned)blocks;
-  if (unroll == 8) {
-    if (vb == 16) return launch_pdl(gather_kernel<uint4, 8>, gb, GATHER_THREADS, 0, st, a);
-    if (vb == 4) return launch_pdl(gather_kernel<unsigned, 8>, gb, GATHER_THREADS, 0, st, a);
-    return launch_pdl(gather_kernel<unsigned short, 8>, gb, GATHER_THREADS, 0, st, a);
-  }
+  if (vb == 32) return launch_pdl(gather_kernel<u32x8, 4>, gb, GATHER_THREADS, 0, st, a);
   if (vb == 16) return launch_pdl(gather_kernel<uint4, 4>, gb, GATHER_THREADS, 0, st, a);
   if (vb == 4) return launch_pdl(gather_kernel<unsigned, 4>, gb, GATHER_THREADS, 0, st, a);
   return launch_pdl(gather_kernel<unsigned short, 4>, gb, GATHER_THREADS, 0, st, a);
-  return cudaGetLastError();
 }
 
 }  // namespace wg
