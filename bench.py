@@ -602,7 +602,8 @@ def bench_layer(args):
     E = int(last["num_edges"].item())
     U = int(last["num_unique"].item())
     D = p.feat_dim
-    X = pipe.X[:U].view(torch.float32).reshape(U, D) if p.feat_dtype == "fp32" else torch.rand(U, D, device="cuda")
+    X = pipe.X_rows[:U].contiguous().view(torch.float32).reshape(U, D) if p.feat_dtype == "fp32" \
+        else torch.rand(U, D, device="cuda")
     row_ptr, sub_col, dup = last["row_ptr"][:T + 1], last["sub_col"][:E], last["dup"][:U]
     dY = torch.rand(T, D, device="cuda")
     peak, peak_src = peaks()

@@ -241,12 +241,14 @@ wg_status wg_dsm_chase(wg_dsm_t h, int32_t rank, int64_t span_bytes, int64_t acc
                        wg_stream_t stream);
 
 /* wg_gather restricted to rows [*d_begin, *d_end) of d_ids / d_out (device int64 scalars;
- * d_begin NULL = 0, d_end NULL = n_ids; both clamped to [0, n_ids]).  Row i is still
- * written at d_out + i * row_bytes.  Because every hop's unique list is a prefix of the
+ * d_begin NULL = 0, d_end NULL = n_ids; both clamped to [0, n_ids]).  Row i is written at
+ * d_out + i * pitch, pitch = out_pitch (0 = dense, row_bytes).  A pitched output (a multiple
+ * of 16 in (row_bytes, row pitch of the shard]) lets rows that are not a multiple of 32 B
+ * move as whole 32 B vectors: bytes [row_bytes, pitch) of each output row are unspecified.  Because every hop's unique list is a prefix of the
  * next one (targets first, L160, L168-174), the rows a batch will gather become known hop by
  * hop: a caller may gather rows [|U_{h-1}|, |U_h|) while hop h+1 is still sampling. */
 wg_status wg_gather_rows(wg_dsm_t h, const int64_t* d_ids, int64_t n_ids, const int64_t* d_begin,
-                         const int64_t* d_end, void* d_out, wg_stream_t stream);
+                         const int64_t* d_end, void* d_out, int64_t out_pitch, wg_stream_t stream);
 
 /* Read (and optionally clear) the latched device error word.  Synchronises the
  * handle's device. */

@@ -51,7 +51,7 @@ def lib():
     L.wg_append_unique.argtypes = [P, P, I64, P, P, I64, P, P, P, P, P, P]
     L.wg_sample_hop.argtypes = [P, P, I64, P, I32, U64, P, I32, P, P, P, P, P, P, P, P, P, P]
     L.wg_gather.argtypes = [P, P, I64, P, P, P]
-    L.wg_gather_rows.argtypes = [P, P, I64, P, P, P, P]
+    L.wg_gather_rows.argtypes = [P, P, I64, P, P, P, I64, P]
     L.wg_dsm_chase.argtypes = [P, I32, I64, I64, P, P]
     L.wg_bucket_by_owner.argtypes = [P, P, I64, P, P, P, P, P]
     L.wg_rows_permute.argtypes = [P, P, P, I64, I64, P]

@@ -417,24 +417,26 @@ wg_status wg_sample_hop(wg_dsm_t h, const int64_t* d_targets, int64_t n_targets,
 }
 
 wg_status wg_gather_rows(wg_dsm_t h, const int64_t* d_ids, int64_t n_ids, const int64_t* d_begin,
-                         const int64_t* d_end, void* d_out, wg_stream_t stream) {
+                         const int64_t* d_end, void* d_out, int64_t out_pitch, wg_stream_t stream) {
   if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
   if (n_ids < 0 || (n_ids > 0 && (!d_ids || !d_out))) return fail(WG_ERR_INVALID_ARG, "null pointer or negative size");
   if (h->row_bytes == 0) return fail(WG_ERR_INVALID_ARG, "DSM has no feature table");
   if (h->row_bytes % 2 != 0) return fail(WG_ERR_UNSUPPORTED, "odd row size");
-  const int64_t vb = (h->row_bytes % 16 == 0) ? 16 : (h->row_bytes % 4 == 0) ? 4 : 2;
-  if (n_ids * (h->row_bytes / 2) >= (int64_t(1) << 31) || n_ids * (h->row_bytes / vb) >= (int64_t(1) << 31))
-    return fail(WG_ERR_UNSUPPORTED, "gather too large for one launch (split the id list)");
+  if (out_pitch != 0 && out_pitch != h->row_bytes &&
+      (out_pitch < h->row_bytes || out_pitch % 16 != 0 || out_pitch > h->feat_stride))
+    return fail(WG_ERR_INVALID_ARG, "out_pitch must be 0, row_bytes, or a multiple of 16 in [row_bytes, row pitch]");
+  const int64_t cw = out_pitch > h->row_bytes ? out_pitch : h->row_bytes;
+  if (n_ids * (cw / 2) >= (int64_t(1) << 31)) return fail(WG_ERR_UNSUPPORTED, "gather too large for one launch");
   cudaSetDevice(h->device);
   if (n_ids == 0 && !d_end) return WG_OK;
-  cudaError_t e = launch_gather(h, d_ids, n_ids, d_end, d_begin, d_out, (cudaStream_t)stream);
+  cudaError_t e = launch_gather(h, d_ids, n_ids, d_end, d_begin, d_out, out_pitch, (cudaStream_t)stream);
   if (e != cudaSuccess) return fail(WG_ERR_CUDA, std::string("gather launch: ") + cudaGetErrorString(e));
   return WG_OK;
 }
 
 wg_status wg_gather(wg_dsm_t h, const int64_t* d_ids, int64_t n_ids, const int64_t* d_n_ids, void* d_out,
                     wg_stream_t stream) {
-  return wg_gather_rows(h, d_ids, n_ids, nullptr, d_n_ids, d_out, stream);
+  return wg_gather_rows(h, d_ids, n_ids, nullptr, d_n_ids, d_out, 0, stream);
 }
 
 wg_status wg_device_error(wg_dsm_t h, uint32_t* code, int32_t clear) {

@@ -1,8 +1,8 @@
 // gather.cu -- global gather over the DSM: "a single gather
 // kernel in each GPU"; NVLink/NVSwitch carry the remote reads.
 //
-// The output X[R][row_bytes] is treated as a flat stream of 16-byte chunks; thread
-// t copies chunk c -> (row c / cpr, column c % cpr), cpr = row_bytes / 16.  Adjacent
+// The output X[R][pitch] is treated as a flat stream of 32- or 16-byte chunks; thread
+// t copies chunk c -> (row c / cpr, column c % cpr), cpr = pitch / chunk.  Adjacent
 // threads therefore read adjacent 16 B pieces of the same source row (full 32 B
 // sectors, one row = one contiguous burst from local HBM or a peer) and write fully
 // coalesced 128 B lines.  Each thread keeps UNROLL independent 16 B loads in flight
@@ -222,7 +222,7 @@ __global__ void __launch_bounds__(32) gather_tma_kernel(const GatherArgs a, int 
 }
 
 cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int64_t* d_n, const int64_t* d_begin,
-                          void* out, cudaStream_t st) {
+                          void* out, int64_t out_pitch, cudaStream_t st) {
   const int64_t rb = h->row_bytes;
   static int knobs = 0, bps = 0, use_tma = 0, allow32 = 1;
   if (!knobs) {  // A/B knobs, read once: WG_GATHER_BPS (blocks per SM), WG_GATHER_TMA=1, WG_GATHER_V32=0
@@ -235,12 +235,15 @@ cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int6
     knobs = 1;
   }
   const uintptr_t oa = (uintptr_t)out;
-  const int vb = (allow32 && rb % 32 == 0 && oa % 32 == 0) ? 32
-                 : (rb % 16 == 0 && oa % 16 == 0)           ? 16
-                 : (rb % 4 == 0 && oa % 4 == 0)             ? 4
+  // copy width per row: the row, or -- for a pitched output (out_pitch > row_bytes, <= the shard's
+  // row pitch) -- the whole output pitch including padding, so 400 B rows can move as 13 x 32 B
+  const int64_t cw = out_pitch > rb ? out_pitch : rb;
+  const int vb = (allow32 && cw % 32 == 0 && oa % 32 == 0) ? 32
+                 : (cw % 16 == 0 && oa % 16 == 0)           ? 16
+                 : (cw % 4 == 0 && oa % 4 == 0)             ? 4
                                                             : 2;
-  GatherArgs a{h->view, ids, cap, d_n, d_begin, static_cast<uint8_t*>(out), h->ws.ctrl, FastDiv((unsigned)(rb / vb))};
-  if (use_tma && rb % 16 == 0 && oa % 16 == 0 && rb <= TMA_STAGE_BYTES) {
+  GatherArgs a{h->view, ids, cap, d_n, d_begin, static_cast<uint8_t*>(out), h->ws.ctrl, FastDiv((unsigned)(cw / vb))};
+  if (use_tma && cw == rb && rb % 16 == 0 && oa % 16 == 0 && rb <= TMA_STAGE_BYTES) {
     const int R = (int)std::min<int64_t>(32, TMA_STAGE_BYTES / rb);
     const int smem = TMA_STAGES * R * (int)rb;
     static int tma_bps = 0;
@@ -268,7 +271,7 @@ cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int6
     occ[which] = nb > 0 ? nb : 4;
   }
   const int per_sm = (bps > 0 && bps < occ[which]) ? bps : occ[which];
-  const int64_t total = cap * (rb / vb);
+  const int64_t total = cap * (cw / vb);
   int64_t blocks = (total + GATHER_THREADS * 4 - 1) / (GATHER_THREADS * 4);
   const int64_t max_blocks = (int64_t)h->sm_count * per_sm;
   blocks = blocks < 1 ? 1 : (blocks > max_blocks ? max_blocks : blocks);

@@ -245,10 +245,16 @@ class DSM:
         return o
 
     def gather_rows(self, ids, cap, begin_dev, end_dev, out, stream=None):
-        """Rows [*begin_dev, *end_dev) of ids -> the same rows of out (wg_gather_rows)."""
-        check(lib().wg_gather_rows(self.h, _ptr(ids), cap, _ptr(begin_dev), _ptr(end_dev), _ptr(out),
+        """Rows [*begin_dev, *end_dev) of ids -> the same rows of out (wg_gather_rows); out is
+        uint8 [*, pitch] with pitch >= row_bytes (a pitched buffer moves 32 B vectors)."""
+        pitch = out.stride(0) if out.dim() == 2 else 0
+        check(lib().wg_gather_rows(self.h, _ptr(ids), cap, _ptr(begin_dev), _ptr(end_dev), _ptr(out), pitch,
                                    _stream(stream)))
         return out
+
+    def out_pitch(self):
+        """Output row pitch that lets the gather move whole 32 B vectors (row bytes rounded up to 32)."""
+        return (self.row_bytes + 31) // 32 * 32
 
     def gather(self, ids, n_ids=None, n_ids_dev=None, out=None, stream=None):
         """Global gather: out[i] = feature row of ids[i] (uint8 rows)."""

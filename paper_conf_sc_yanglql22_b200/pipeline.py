@@ -59,8 +59,11 @@ class MiniBatchPipeline:
                 num_edges=torch.zeros(1, **i64), unique=torch.zeros(max(T + E, 1), **i64),
                 num_unique=torch.zeros(1, **i64), sub_col=torch.zeros(max(E, 1), **i32),
                 dup=torch.zeros(max(T + E, 1), **i32) if with_dup else None))
-        self.X = torch.zeros((max(self.U_cap[-1], 1), dsm.row_bytes), dtype=torch.uint8, device=dev) \
+        # X is pitched to a 32 B multiple so every row moves as whole 32 B vectors; X_rows is the
+        # [U, row_bytes] view of the feature bytes (self.X[:, :row_bytes])
+        self.X = torch.zeros((max(self.U_cap[-1], 1), dsm.out_pitch()), dtype=torch.uint8, device=dev) \
             if dsm.row_bytes else None
+        self.X_rows = self.X[:, :dsm.row_bytes] if self.X is not None else None
         self.graph = None
 
     # -- enqueue one batch (reads seeds / n_seeds / rng_seed from device buffers)
@@ -101,7 +104,7 @@ class MiniBatchPipeline:
 
     def enqueue_gather(self, stream=None):
         last = self.hops[-1]
-        self.dsm.gather(last["unique"], n_ids=self.U_cap[-1], n_ids_dev=last["num_unique"], out=self.X, stream=stream)
+        self.dsm.gather_rows(last["unique"], self.U_cap[-1], None, last["num_unique"], self.X, stream=stream)
 
     def set_inputs(self, seeds: torch.Tensor, rng_seed: int, stream=None):
         """Copy this batch's seed nodes (device or pinned host int64) and rng_seed
@@ -155,7 +158,7 @@ class MiniBatchPipeline:
 
     def features(self):
         u = int(self.hops[-1]["num_unique"].item())
-        return self.X[:u].cpu().numpy()
+        return self.X_rows[:u].contiguous().cpu().numpy()
 
 
 def to_i64(x: int) -> int:
