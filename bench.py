@@ -397,15 +397,14 @@ def bench_wg(args):
     e2e_times = []
     d2h = torch.empty((len(p.fanouts), 2), dtype=torch.int64, pin_memory=True)
     host_seeds = [seeds_dev[k % n_single].cpu().pin_memory() for k in range(args.e2e_steps)]
-    pl0, (gp0, gg0) = pipes[0], graphs[0]
+    pl0, gf0 = pipes[0], full_graphs[0]
     for i in range(args.e2e_steps + 2):
         hs = host_seeds[i % len(host_seeds)]
         torch.cuda.synchronize()
         t = time.perf_counter()
-        pl0.set_inputs(hs, rngs[i % n_single])
-        if gp0 is not None:
-            gp0.replay()
-            gg0.replay()
+        pl0.set_inputs(hs, rngs[i % n_single])   # H2D of the seeds from pinned host memory
+        if gf0 is not None:
+            gf0.replay()                          # the shipped batch graph (hops + incremental gather)
         else:
             pl0.enqueue()
         for h, b in enumerate(pl0.hops):
