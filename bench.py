@@ -176,6 +176,29 @@ def workload_config(p, W, flushed=True):
             "note": p.note}
 
 
+
+def workload_descriptors(dsm, pipe, seeds_dev, rngs, nb=20):
+    """SURVEY 8(d) workload descriptors (generator properties that drive the numbers): this rank's
+    out-degree distribution, and the share of gathered rows that falls on the top 1 % most-gathered
+    rows over nb batches (outside every timed region)."""
+    import torch
+    rp, _, _ = dsm.local_view()
+    deg = (rp[1:] - rp[:-1]).double()
+    lg = torch.floor(torch.log2(deg.clamp(min=1))).long()
+    hist = torch.bincount(lg, minlength=18).tolist()
+    cnt = torch.zeros(dsm.num_nodes, dtype=torch.int32, device=rp.device)
+    tot = 0
+    for k in range(min(nb, len(seeds_dev))):
+        pipe.run(seeds_dev[k], rngs[k])
+        u = pipe.hops[-1]["unique"][: int(pipe.hops[-1]["num_unique"].item())]
+        cnt.index_add_(0, u, torch.ones_like(u, dtype=torch.int32))
+        tot += u.numel()
+    top = torch.topk(cnt, max(1, dsm.num_nodes // 100)).values.sum().item()
+    q = torch.quantile(deg[: 1 << 24], torch.tensor([0.5, 0.99], dtype=torch.float64, device=deg.device)).tolist()
+    return {"degree_mean": float(deg.mean()), "degree_max": int(deg.max()), "degree_p50": q[0], "degree_p99": q[1],
+            "degree_log2_hist": hist, "top1pct_rows_share_of_gathered": top / max(tot, 1),
+            "batches_for_share": min(nb, len(seeds_dev))}
+
 def emit(line, args):
     s = json.dumps(line)
     print(s, flush=True)
@@ -393,28 +416,30 @@ def bench_wg(args):
         bound, alg_bytes, peak_used, peak_src_used = "hbm", hbm_bytes, peak, peak_src
     achieved = alg_bytes / gather_s / 1e9
 
-    # ---- e2e through the public API with pinned host buffers (H2D seeds, D2H counts)
-    e2e_times = []
-    d2h = torch.empty((len(p.fanouts), 2), dtype=torch.int64, pin_memory=True)
-    host_seeds = [seeds_dev[k % n_single].cpu().pin_memory() for k in range(args.e2e_steps)]
-    pl0, gf0 = pipes[0], full_graphs[0]
-    for i in range(args.e2e_steps + 2):
-        hs = host_seeds[i % len(host_seeds)]
-        torch.cuda.synchronize()
-        t = time.perf_counter()
-        pl0.set_inputs(hs, rngs[i % n_single])   # H2D of the seeds from pinned host memory
-        if gf0 is not None:
-            gf0.replay()                          # the shipped batch graph (hops + incremental gather)
-        else:
-            pl0.enqueue()
-        for h, b in enumerate(pl0.hops):
-            d2h[h, 0:1].copy_(b["num_edges"], non_blocking=True)
-            d2h[h, 1:2].copy_(b["num_unique"], non_blocking=True)
-        torch.cuda.current_stream().synchronize()
-        if i >= 2:
-            e2e_times.append(time.perf_counter() - t)
-    e2e_val = world * S / max_over_ranks(statistics.mean(e2e_times))
+    # ---- e2e through the public API (MiniBatchLoader): every batch = H2D of its seeds from pinned host
+    # memory + the batch graph + D2H of its per-hop counts, P batches in flight (as pass B), host-timed
+    # from the first submit to the last batch handed out
+    loader_ = pkg.MiniBatchLoader(dsm, p.fanouts, S, depth=P)
+    host_seeds = [seeds_dev[k % n_single].cpu().pin_memory() for k in range(args.e2e_steps * P)]
+    warm = [(host_seeds[k % len(host_seeds)], rngs[k % n_single]) for k in range(2 * P)]
+    for _ in loader_(warm):
+        pass
+    torch.cuda.synchronize()
+    todo = [(host_seeds[k], rngs[(n_single + k) % len(rngs)]) for k in range(args.e2e_steps * P)]
+    if world > 1:
+        dist.barrier()
+    torch.cuda.synchronize()
+    t = time.perf_counter()
+    e2e_rows = 0
+    for pb in loader_(todo):
+        e2e_rows += pb.counts[-1][1]
+    e2e_s = time.perf_counter() - t
+    assert loader_.device_error() == 0
+    e2e_val = world * S * len(todo) / max_over_ranks(e2e_s)
+    e2e_d2h = len(p.fanouts) * 2 * 8
+    loader_.close()
 
+    wdesc = workload_descriptors(dsm, pipes[0], seeds_dev, rngs) if rank == 0 else {}
     line = None
     if rank == 0:
         cpu = None
@@ -448,15 +473,16 @@ def bench_wg(args):
                          "timed_in": "pass A (one batch at a time, events on the launching stream)"},
             "cpu_baseline": cpu,
             "e2e": {"value": e2e_val, "unit": UNIT, "h2d_bytes_per_step": S * 8,
-                    "d2h_bytes_per_step": int(d2h.numel() * 8),
-                    "note": "public API (MiniBatchPipeline.run), one batch per step: pinned-host seeds H2D, "
-                            "per-hop counts D2H, host-timed incl. sync"},
+                    "d2h_bytes_per_step": e2e_d2h, "batches": len(todo),
+                    "note": f"public API (MiniBatchLoader, {P} batches in flight): per batch pinned-host seeds "
+                            "H2D + batch graph + per-hop counts D2H, host-timed from first submit to last "
+                            "batch handed out"},
             # our kernels per batch: 4 per hop (sample, insert, flag-scan, relabel) + the gather (pass A)
             # or + one gather_rows per hop (the shipped incremental graph: passes A' and B)
             "gpu_launches": args.steps * (4 * len(p.fanouts) + 1) + args.steps * (1 + P) * 5 * len(p.fanouts),
             "clocks": clk,
             "wall_s_timed_region": wall,
-            "workload_stats": {"edges_per_hop_mean": hc[:, :, 0].mean(0).tolist(),
+            "workload_stats": {**wdesc, "edges_per_hop_mean": hc[:, :, 0].mean(0).tolist(),
                                "unique_per_hop_mean": hc[:, :, 1].mean(0).tolist(),
                                "unique_bound_per_hop": pipes[0].U_cap, "rows_gathered_mean": float(rows.mean()),
                                "row_bytes": rb},

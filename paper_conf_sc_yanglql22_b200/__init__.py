@@ -8,4 +8,4 @@ the thin Python binding (argument marshalling) plus the batch pipeline.
 
 from ._lib import LIB_PATH, WgError, lib  # noqa: F401
 from .dsm import DSM, ThreadAllgather, TorchDistAllgather, local_num_edges, shard_csr  # noqa: F401
-from .pipeline import MiniBatchPipeline, capacities, required_keys  # noqa: F401
+from .pipeline import MiniBatchLoader, MiniBatchPipeline, PreparedBatch, capacities, required_keys  # noqa: F401

@@ -164,3 +164,129 @@ class MiniBatchPipeline:
 def to_i64(x: int) -> int:
     x &= (1 << 64) - 1
     return x - (1 << 64) if x >= (1 << 63) else x
+
+
+class PreparedBatch:
+    """One prepared mini-batch handed out by MiniBatchLoader: host-side per-hop counts and
+    DEVICE views of the pipeline slot's buffers (valid until the next batch is requested)."""
+
+    def __init__(self, index, pipe, counts, n_seeds):
+        self.index, self.pipe, self.n_seeds = index, pipe, n_seeds
+        self.counts = counts          # [(num_edges, num_unique)] per hop, host ints
+
+    def hop(self, h):
+        """Hop h's sub-graph: row_ptr [T_h+1], nbrs / sub_col [E_h], unique [U_h] (device views)."""
+        b = self.pipe.hops[h]
+        nT = self.n_seeds if h == 0 else self.counts[h - 1][1]
+        e, u = self.counts[h]
+        return dict(row_ptr=b["row_ptr"][: nT + 1], nbrs=b["nbrs"][:e], sub_col=b["sub_col"][:e],
+                    unique=b["unique"][:u], pos=None if b["pos"] is None else b["pos"][:e],
+                    dup=None if b["dup"] is None else b["dup"][:u])
+
+    @property
+    def X(self):
+        """Gathered feature bytes [U_{H-1}, row_bytes] (uint8 view, rows in unique order)."""
+        return self.pipe.X_rows[: self.counts[-1][1]]
+
+
+class MiniBatchLoader:
+    """Pipelined mini-batch preparation: `depth` independent MiniBatchPipelines (one DSM
+    workspace fork and one stream each) prepare consecutive batches concurrently, so the
+    latency-bound hops of one batch overlap the bandwidth-bound gather of another.
+
+    Every batch is: H2D of its seed ids (pinned host or device int64) and rng_seed, the
+    captured batch graph (all hops + incremental gather), and a D2H of its per-hop counts
+    into pinned memory.  `__call__(batches)` yields PreparedBatch objects in submission
+    order, keeping up to `depth` batches in flight; a slot is reused only after the
+    consumer's stream has passed the point where the batch was handed out."""
+
+    def __init__(self, dsm: DSM, fanouts, max_seeds, depth=8, with_pos=False, with_dup=False, graphs=True):
+        self.depth = max(1, depth)
+        self.handles = [dsm] + [dsm.fork() for _ in range(self.depth - 1)]
+        self.pipes = [MiniBatchPipeline(h, fanouts, max_seeds, with_pos=with_pos, with_dup=with_dup)
+                      for h in self.handles]
+        dev = dsm.device
+        self.streams = [torch.cuda.Stream(device=dev) for _ in range(self.depth)]
+        self.done = [torch.cuda.Event() for _ in range(self.depth)]
+        self.released = [None] * self.depth        # event recorded on the consumer stream at hand-out
+        self.counts = [torch.zeros((len(fanouts), 2), dtype=torch.int64, pin_memory=True)
+                       for _ in range(self.depth)]
+        self.n_seeds = [0] * self.depth
+        self.use_graphs = graphs
+        self.graphs = [None] * self.depth
+        self.warm = [0] * self.depth
+        self.next_slot = 0
+
+    def submit(self, seeds, rng_seed):
+        """Enqueue one batch on the next slot; returns the slot index (stream-ordered, no sync)."""
+        j = self.next_slot
+        self.next_slot = (j + 1) % self.depth
+        pl, st = self.pipes[j], self.streams[j]
+        if self.released[j] is not None:
+            st.wait_event(self.released[j])        # the consumer is done with the slot's last batch
+            self.released[j] = None
+        self.n_seeds[j] = seeds.numel()
+        with torch.cuda.stream(st):
+            pl.set_inputs(seeds, rng_seed, st)
+            if self.graphs[j] is not None:
+                self.graphs[j].replay()
+            else:
+                pl.enqueue(st)
+                self.warm[j] += 1
+            c = self.counts[j]
+            for h, b in enumerate(pl.hops):
+                c[h, 0:1].copy_(b["num_edges"], non_blocking=True)
+                c[h, 1:2].copy_(b["num_unique"], non_blocking=True)
+            self.done[j].record(st)
+        if self.use_graphs and self.graphs[j] is None and self.warm[j] >= 1:
+            self._capture(j)
+        return j
+
+    def _capture(self, j):
+        st = self.streams[j]
+        st.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g, stream=st):
+            self.pipes[j].enqueue(st)
+        self.graphs[j] = g
+
+    def collect(self, j, index=0):
+        """Wait (host) for slot j's batch and hand it out (call release(j) when the consumer's
+        work on it has been enqueued)."""
+        self.done[j].synchronize()
+        counts = [(int(e), int(u)) for e, u in self.counts[j].tolist()]
+        return PreparedBatch(index, self.pipes[j], counts, self.n_seeds[j])
+
+    def release(self, j):
+        """The slot may be refilled once the consumer stream reaches this point."""
+        ev = torch.cuda.Event()
+        ev.record(torch.cuda.current_stream(self.pipes[j].dsm.device))
+        self.released[j] = ev
+
+    def __call__(self, batches):
+        """batches: iterable of (seed ids int64 tensor, rng_seed).  Yields PreparedBatch in order;
+        a batch's buffers stay valid until the next batch is requested (its slot is released then,
+        stream-ordered after whatever the consumer enqueued on the current stream)."""
+        pending = []
+        for i, (s, r) in enumerate(batches):
+            if len(pending) == self.depth:
+                k, j = pending.pop(0)
+                yield self.collect(j, k)
+                self.release(j)
+            pending.append((i, self.submit(s, r)))
+        for k, j in pending:
+            yield self.collect(j, k)
+            self.release(j)
+
+    def device_error(self):
+        err = 0
+        for h in self.handles:
+            err |= h.device_error()
+        return err
+
+    def close(self):
+        torch.cuda.synchronize()
+        self.graphs = [None] * self.depth
+        for h in self.handles[1:]:
+            h.destroy()
+        self.handles = self.handles[:1]
