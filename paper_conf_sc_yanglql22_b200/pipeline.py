@@ -32,14 +32,14 @@ def required_keys(n, fanouts, max_seeds):
 
 class MiniBatchPipeline:
     def __init__(self, dsm: DSM, fanouts, max_seeds, with_pos=False, with_dup=False, fused=True,
-                 incremental_gather=True):
+                 incremental_gather=True, gather_priority=0, side_priority=0):
         self.dsm, self.fanouts, self.max_seeds = dsm, list(fanouts), max_seeds
         self.fused = fused
-        self.side = torch.cuda.Stream(device=dsm.device) if fused else None
+        self.side = torch.cuda.Stream(device=dsm.device, priority=side_priority) if fused else None
         # incremental gather: U_{h-1} is a prefix of U_h, so the feature rows of hop h's new nodes
         # are gathered on gside while hop h+1 samples; only the last hop's new rows remain at the end
         self.incremental = incremental_gather
-        self.gside = torch.cuda.Stream(device=dsm.device) if incremental_gather else None
+        self.gside = torch.cuda.Stream(device=dsm.device, priority=gather_priority) if incremental_gather else None
         self.with_pos, self.with_dup = with_pos, with_dup
         dev = dsm.device
         self.T_cap, self.E_cap, self.U_cap = capacities(dsm.num_nodes, fanouts, max_seeds)

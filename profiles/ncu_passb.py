@@ -24,7 +24,9 @@ P = int(sys.argv[2]) if len(sys.argv) > 2 else 8
 p = presets.get(os.environ.get("CONFIG", "products"))
 dsm, _ = loader.build_dsm(p)
 handles = [dsm] + [dsm.fork() for _ in range(P - 1)]
-pipes = [pkg.MiniBatchPipeline(h, p.fanouts, p.seeds_per_batch) for h in handles]
+GP, SP, MP = (int(os.environ.get(k, 0)) for k in ("PRIO_GATHER", "PRIO_SIDE", "PRIO_MAIN"))
+pipes = [pkg.MiniBatchPipeline(h, p.fanouts, p.seeds_per_batch, gather_priority=GP, side_priority=SP)
+         for h in handles]
 S = p.seeds_per_batch
 for j, pl in enumerate(pipes):   # eager warm-up; fills X / hop buffers for the gather-only mode
     pl.run(torch.from_numpy(seeds.seed_nodes(p.n, S, presets.SEED_BASE, j)).cuda(), seeds.rng_seed(presets.RNG_BASE, j))
@@ -32,7 +34,7 @@ torch.cuda.synchronize()
 
 g = torch.cuda.CUDAGraph()
 cap = torch.cuda.Stream()
-streams = [torch.cuda.Stream() for _ in range(P)]
+streams = [torch.cuda.Stream(priority=MP) for _ in range(P)]
 cap.wait_stream(torch.cuda.current_stream())
 with torch.cuda.graph(g, stream=cap):
     for j, pl in enumerate(pipes):   # fork all P batches first, then join (they run concurrently)
@@ -61,5 +63,5 @@ for i in range(int(os.environ.get("REPS", 20))):
 assert all(h.device_error() == 0 for h in handles)
 rows = sum(int(pl.hops[-1]["num_unique"].item()) for pl in pipes)
 t = statistics.median(ts)
-print(f"mode={mode} P={P} graph_ms_median={t:.4f} per_batch_us={1e3 * t / P:.1f} "
+print(f"mode={mode} P={P} prio(g,s,m)={GP},{SP},{MP} graph_ms_median={t:.4f} per_batch_us={1e3 * t / P:.1f} "
       f"seeds_per_s={P * S / (t / 1e3):.0f} rows_gathered_last={rows}", flush=True)
