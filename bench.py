@@ -541,8 +541,7 @@ def bench_sweep(args):
                               "does not fit one GPU (needs W >= 2)"})
                 continue
             dsm = pkg.DSM(n, 0, dim, dtype, 1, device=0)
-            _, _, fv = dsm.local_view()
-            sgpu.fill_features_gpu(fv, presets.FEAT_SEED, 0, 1, dim, sfeat.WG_DTYPE_CODE[dtype])
+            sgpu.fill_dsm_features_gpu(dsm, presets.FEAT_SEED, 0, 1, dim, sfeat.WG_DTYPE_CODE[dtype])
             out = torch.empty((R, rb), dtype=torch.uint8, device=dev)
             for _ in range(3):
                 dsm.gather(ids, out=out)
@@ -561,7 +560,7 @@ def bench_sweep(args):
             algo = R * rb / t / 1e9
             cells.append({"dtype": dtype, "dim": dim, "row_bytes": rb, "ms": t * 1e3, "algo_gbs": algo,
                           "hbm_gbs_read_plus_write": 2 * algo, "frac_of_hbm_roofline": 2 * algo / peak})
-            del out, fv
+            del out
             dsm.destroy()
             torch.cuda.empty_cache()
     best = max((c for c in cells if "ms" in c), key=lambda c: c["frac_of_hbm_roofline"])
@@ -589,10 +588,8 @@ def bench_latency(args):
     dsm = pkg.DSM(rows, 0, 128, "fp32", 1, device=0)   # 512 B rows, filled with generator bits
     from synth import gpu as sgpu
     from synth import presets
-    _, _, fv = dsm.local_view()
-    sgpu.fill_features_gpu(fv, presets.FEAT_SEED, 0, 1, 128, 0)
+    sgpu.fill_dsm_features_gpu(dsm, presets.FEAT_SEED, 0, 1, 128, 0)
     torch.cuda.synchronize()
-    del fv
     res = []
     for sp in spans:
         dsm.chase(0, sp, 2000)                            # warm-up (TLB, clocks)

@@ -93,8 +93,8 @@ typedef struct {
 
 /* Create the DSM (section III-B).  COLLECTIVE over the W ranks.
  * Each rank allocates its shard slab on its device -- row_ptr int64[n_local+1],
- * col_idx int64[local_num_edges], features [n_local][row stride] with the row
- * stride rounded up to 64 bytes (the DRAM access granule) -- exports a CUDA IPC handle, allgathers the
+ * col_idx int64[local_num_edges], features [n_local][row stride] (+ a tail region for the
+ * split row layout, see wg_dsm_feat_layout) -- exports a CUDA IPC handle, allgathers the
  * handles (L100), opens every peer's handle (L100-106; same-process peers are used
  * directly) and keeps the W base pointers as the "memory pointer table" (L106),
  * passed by value to every kernel.  n_local = number of v in [0,n) with v mod W == rank.
@@ -106,9 +106,23 @@ wg_status wg_dsm_create(const wg_dsm_desc* desc, wg_dsm_t* out);
 
 /* Device pointers of THIS rank's shard, for filling it (any stream; the caller
  * synchronises and barriers before other ranks read).  Any output may be NULL.
- * feat_row_stride_bytes is the padded row pitch of the feature shard. */
+ * feat_row_stride_bytes is the row pitch of the feature shard, which holds the first
+ * body_bytes bytes of every row (wg_dsm_feat_layout; the whole row unless the layout is split). */
 wg_status wg_dsm_local_view(wg_dsm_t h, int64_t** d_row_ptr, int64_t** d_col_idx, void** d_feat,
                             int64_t* n_local_rows, int64_t* feat_row_stride_bytes);
+
+/* Feature-row layout of the shards (identical on every rank).  The B200 L2 fills whole
+ * 128 B lines on a miss, so a row of R bytes with R > 128, R % 128 != 0 and R % 16 == 0 is
+ * SPLIT: its first body_bytes = R - R % 128 bytes are stored in the feature shard
+ * (wg_dsm_local_view's d_feat) at body_pitch = body_bytes, i.e. whole lines, and its last
+ * R % 128 bytes at d_tail + l * tail_pitch (tail_pitch = R % 128) in a dense tail region of
+ * THIS rank's slab.  Otherwise body_bytes = R, body_pitch = R rounded up to 64, d_tail = NULL
+ * and tail_pitch = 0.  Fillers write bytes [0, body_bytes) of local row l at
+ * d_feat + l * body_pitch and bytes [body_bytes, R) at d_tail + l * tail_pitch.  The layout is
+ * invisible to every op (wg_gather returns whole rows).  WG_FEAT_SPLIT=0 in the environment at
+ * create disables the split (A/B).  Any output may be NULL. */
+wg_status wg_dsm_feat_layout(wg_dsm_t h, int64_t* body_bytes, int64_t* body_pitch, void** d_tail,
+                             int64_t* tail_pitch);
 
 /* Geometry of rank r's shard (any r): local rows and local CSR entries. */
 wg_status wg_dsm_shard_info(wg_dsm_t h, int32_t r, int64_t* n_local_rows, int64_t* local_num_edges);

@@ -1,8 +1,9 @@
 // dsm.cu -- the multi-GPU distributed shared memory (section III-B)
 // and the C-ABI entry points of include/wg.h.
 //
-// Each rank allocates ONE slab on its GPU holding its three shards
-//   [ row_ptr int64[n_local+1] | col_idx int64[e_local] | feat[n_local][stride] ]
+// Each rank allocates ONE slab on its GPU holding its shards
+//   [ row_ptr int64[n_local+1] | col_idx int64[e_local] | feat[n_local][stride] | tail[n_local][tail_pitch] ]
+// The tail region exists only for the split feature layout (feat_geometry below).
 // (256-byte aligned sub-offsets; cudaMalloc of >= 2 MB uses 2 MB pages, so TLB reach
 // covers the shards with few entries), exports a CUDA IPC handle, allgathers a fixed
 // record {pid, device pointer, IPC handle, geometry} through the caller's callback
@@ -45,6 +46,33 @@ static int64_t local_rows(int64_t n, int rank, int world) {
   return n > rank ? (n - rank + world - 1) / world : 0;
 }
 
+// Feature-row layout.  The B200 L2 fills whole 128 B lines on a miss (measured:
+// profiles/r01/fetch_granularity.md -- a random 32 B row costs 128 B of DRAM, a 400 B row at
+// a 64 B-aligned pitch costs 4 lines = 512 B, cudaLimitMaxL2FetchGranularity has no effect).
+// A row whose size is not a multiple of 128 B (but a multiple of 16 B, > 128 B) is therefore
+// SPLIT: its first floor(row/128)*128 bytes (the body) live in the feature shard at a pitch of
+// exactly that many bytes, so a body is whole lines and costs no over-fetch; the remaining
+// row % 128 bytes (the tail) live densely in a separate tail region (pitch = tail bytes), small
+// enough to stay in L2 (products-shaped: 2.45M x 16 B = 39 MB) and read with an evict_last hint.
+// Otherwise rows stay whole at a pitch rounded up to 64 B.  WG_FEAT_SPLIT=0 disables the split.
+static void feat_geometry(int64_t row_bytes, int64_t* body, int64_t* stride, int64_t* tail_pitch) {
+  static int split = -1;
+  if (split < 0) {
+    const char* e = getenv("WG_FEAT_SPLIT");
+    split = (e && e[0] == '0') ? 0 : 1;
+  }
+  const int64_t t = row_bytes % 128;
+  if (split && row_bytes > 128 && t != 0 && t % 16 == 0) {
+    *body = row_bytes - t;
+    *stride = *body;
+    *tail_pitch = t;
+  } else {
+    *body = row_bytes;
+    *stride = round_up(row_bytes, 64);
+    *tail_pitch = 0;
+  }
+}
+
 struct PeerRecord {
   int64_t pid;
   uint64_t dev_ptr;
@@ -53,8 +81,10 @@ struct PeerRecord {
   int64_t e_local;
   int64_t off_col;
   int64_t off_feat;
+  int64_t off_tail;
   int64_t num_nodes;
   int64_t feat_stride;
+  int64_t tail_pitch;
   int32_t world;
   int32_t rank;
   cudaIpcMemHandle_t handle;
@@ -175,7 +205,7 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
   h->feat_dim = d->feat_dim;
   h->elt = d->feat_dtype == WG_F32 ? 4 : 2;
   h->row_bytes = h->feat_dim * h->elt;
-  h->feat_stride = round_up(h->row_bytes, 64);  // 64 B = the DRAM access granule: no row straddles an extra one
+  feat_geometry(h->row_bytes, &h->body_bytes, &h->feat_stride, &h->tail_pitch);
   h->allgather = d->allgather;
   h->ctx = d->ctx;
   h->sm_count = sms;
@@ -185,7 +215,8 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
   // ---- this rank's slab
   const int64_t off_col = round_up((h->n_local + 1) * 8, 256);
   const int64_t off_feat = round_up(off_col + h->e_local * 8, 256);
-  h->slab_bytes = (size_t)round_up(off_feat + h->n_local * h->feat_stride, 256);
+  const int64_t off_tail = round_up(off_feat + h->n_local * h->feat_stride, 256);
+  h->slab_bytes = (size_t)round_up(off_tail + h->n_local * h->tail_pitch, 256);
   if (cudaMalloc(&h->slab, h->slab_bytes) != cudaSuccess) {
     cudaGetLastError();
     h->slab = nullptr;
@@ -215,8 +246,10 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
   mine.e_local = h->e_local;
   mine.off_col = off_col;
   mine.off_feat = off_feat;
+  mine.off_tail = off_tail;
   mine.num_nodes = h->n;
   mine.feat_stride = h->feat_stride;
+  mine.tail_pitch = h->tail_pitch;
   mine.world = h->world;
   mine.rank = h->rank;
   PeerRecord all[WG_MAX_WORLD];
@@ -236,7 +269,7 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
   }
   for (int r = 0; r < h->world; ++r) {
     if (all[r].rank != r || all[r].world != h->world || all[r].num_nodes != h->n ||
-        all[r].feat_stride != h->feat_stride) {
+        all[r].feat_stride != h->feat_stride || all[r].tail_pitch != h->tail_pitch) {
       release(h);
       return fail(WG_ERR_INVALID_ARG, "ranks disagree on world_size / num_nodes / feat_dim");
     }
@@ -265,9 +298,12 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
     h->view.row_ptr[r] = reinterpret_cast<const int64_t*>(b);
     h->view.col[r] = reinterpret_cast<const int64_t*>(b + all[r].off_col);
     h->view.feat[r] = b + all[r].off_feat;
+    h->view.tail[r] = h->tail_pitch ? b + all[r].off_tail : nullptr;
   }
   h->view.n = h->n;
   h->view.feat_stride = h->feat_stride;
+  h->view.tail_pitch = h->tail_pitch;
+  h->view.body_bytes = h->body_bytes;
   h->view.world = h->world;
   h->view.log2w = -1;
   for (int k = 0; k <= 3; ++k)
@@ -294,6 +330,16 @@ wg_status wg_dsm_local_view(wg_dsm_t h, int64_t** row_ptr, int64_t** col, void**
   if (feat) *feat = const_cast<uint8_t*>(h->view.feat[h->rank]);
   if (n_local_rows) *n_local_rows = h->n_local;
   if (stride) *stride = h->feat_stride;
+  return WG_OK;
+}
+
+wg_status wg_dsm_feat_layout(wg_dsm_t h, int64_t* body_bytes, int64_t* body_pitch, void** d_tail,
+                             int64_t* tail_pitch) {
+  if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
+  if (body_bytes) *body_bytes = h->body_bytes;
+  if (body_pitch) *body_pitch = h->feat_stride;
+  if (d_tail) *d_tail = const_cast<uint8_t*>(h->view.tail[h->rank]);
+  if (tail_pitch) *tail_pitch = h->tail_pitch;
   return WG_OK;
 }
 
@@ -422,8 +468,11 @@ wg_status wg_gather_rows(wg_dsm_t h, const int64_t* d_ids, int64_t n_ids, const 
   if (n_ids < 0 || (n_ids > 0 && (!d_ids || !d_out))) return fail(WG_ERR_INVALID_ARG, "null pointer or negative size");
   if (h->row_bytes == 0) return fail(WG_ERR_INVALID_ARG, "DSM has no feature table");
   if (h->row_bytes % 2 != 0) return fail(WG_ERR_UNSUPPORTED, "odd row size");
+  // a pitched output may cover the row's padding in the shard (whole layout) or up to the next 32 B
+  // (split layout: the tail chunk is zero-filled past the row)
+  const int64_t max_pitch = h->tail_pitch ? round_up(h->row_bytes, 32) : h->feat_stride;
   if (out_pitch != 0 && out_pitch != h->row_bytes &&
-      (out_pitch < h->row_bytes || out_pitch % 16 != 0 || out_pitch > h->feat_stride))
+      (out_pitch < h->row_bytes || out_pitch % 16 != 0 || out_pitch > max_pitch))
     return fail(WG_ERR_INVALID_ARG, "out_pitch must be 0, row_bytes, or a multiple of 16 in [row_bytes, row pitch]");
   const int64_t cw = out_pitch > h->row_bytes ? out_pitch : h->row_bytes;
   if (n_ids * (cw / 2) >= (int64_t(1) << 31)) return fail(WG_ERR_UNSUPPORTED, "gather too large for one launch");

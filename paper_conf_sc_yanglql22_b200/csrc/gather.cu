@@ -9,7 +9,8 @@
 // (ld.global.nc.L1::no_allocate: every byte is read exactly once), so a grid of
 // ~8 x 256 threads per SM keeps ~0.5 MB in flight chip-wide -- enough to cover
 // local-HBM and NVLink latency.  Rows whose size is not a multiple of 16 use the
-// same scheme with 4- or 2-byte chunks.
+// same scheme with 4- or 2-byte chunks.  For the split row layout (dsm.cu feat_geometry) a
+// chunk at byte offset >= body_bytes comes from the owner's tail region (L2 evict_last).
 #include <algorithm>
 #include <cstdlib>
 
@@ -47,6 +48,59 @@ template <>
 __device__ __forceinline__ unsigned ld_feat<unsigned>(const void* p) { return ld_nc_na_u32(p); }
 template <>
 __device__ __forceinline__ unsigned short ld_feat<unsigned short>(const void* p) { return ld_nc_na_u16(p); }
+
+// L2 policy for tail loads: the split layout's tail region is small and re-read by every batch,
+// so it is kept in L2 with evict_last (createpolicy, the sm_80+ L2 cache-hint mechanism).
+__device__ __forceinline__ unsigned long long l2_evict_last_policy() {
+  unsigned long long p;
+  asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint4 ld_tail_v4(const void* p, unsigned long long pol) {
+  uint4 r;
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+      : "=r"(r.x), "=r"(r.y), "=r"(r.z), "=r"(r.w)
+      : "l"(p), "l"(pol));
+  return r;
+}
+__device__ __forceinline__ u32x8 ld_tail_v8(const void* p, unsigned long long pol) {
+  u32x8 r;
+  asm("ld.global.nc.L1::no_allocate.L2::cache_hint.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+      : "=r"(r.v[0]), "=r"(r.v[1]), "=r"(r.v[2]), "=r"(r.v[3]), "=r"(r.v[4]), "=r"(r.v[5]), "=r"(r.v[6]),
+        "=r"(r.v[7])
+      : "l"(p), "l"(pol));
+  return r;
+}
+
+// Chunk of `avail` (>= 16, a multiple of 16) tail bytes starting at t, as one vector V; bytes past
+// the row (a pitched output's padding) read as zero.
+template <typename V>
+__device__ __forceinline__ V ld_tail(const uint8_t* t, unsigned avail, unsigned long long pol) {
+  return ld_feat<V>(t);
+}
+template <>
+__device__ __forceinline__ uint4 ld_tail<uint4>(const uint8_t* t, unsigned avail, unsigned long long pol) {
+  return ld_tail_v4(t, pol);
+}
+template <>
+__device__ __forceinline__ u32x8 ld_tail<u32x8>(const uint8_t* t, unsigned avail, unsigned long long pol) {
+  if (avail >= 32 && ((uintptr_t)t & 31u) == 0) return ld_tail_v8(t, pol);
+  const uint4 a = ld_tail_v4(t, pol);
+  const uint4 b = avail >= 32 ? ld_tail_v4(t + 16, pol) : make_uint4(0, 0, 0, 0);
+  u32x8 r;
+  r.v[0] = a.x, r.v[1] = a.y, r.v[2] = a.z, r.v[3] = a.w, r.v[4] = b.x, r.v[5] = b.y, r.v[6] = b.z, r.v[7] = b.w;
+  return r;
+}
+
+// Chunk at byte offset boff of row l on rank o: from the body (feature shard) or, for the split
+// layout, from the tail region (boundaries are multiples of 128 B, so no chunk straddles them).
+template <typename V>
+__device__ __forceinline__ V ld_row_chunk(const ShardView& s, int o, int64_t l, unsigned boff,
+                                          unsigned long long pol) {
+  if (s.tail_pitch == 0 || boff < (unsigned)s.body_bytes) return ld_feat<V>(s.feat[o] + l * s.feat_stride + boff);
+  const unsigned toff = boff - (unsigned)s.body_bytes;
+  return ld_tail<V>(s.tail[o] + l * s.tail_pitch + toff, (unsigned)s.tail_pitch - toff, pol);
+}
 
 struct GatherArgs {
   ShardView s;
@@ -89,6 +143,7 @@ __global__ void __launch_bounds__(GATHER_THREADS) gather_kernel(const GatherArgs
   const unsigned total = (unsigned)(n * cpr);  // < 2^31 (checked on the host)
   const unsigned stride = gridDim.x * GATHER_THREADS;
   V* __restrict__ out = reinterpret_cast<V*>(a.out + begin * (int64_t)cpr * (int64_t)sizeof(V));
+  const unsigned long long pol = l2_evict_last_policy();
   for (unsigned c0 = blockIdx.x * GATHER_THREADS + threadIdx.x; c0 < total; c0 += stride * GATHER_UNROLL) {
     V val[GATHER_UNROLL];
     unsigned dst[GATHER_UNROLL];
@@ -104,7 +159,7 @@ __global__ void __launch_bounds__(GATHER_THREADS) gather_kernel(const GatherArgs
           int o;
           int64_t l;
           owner_local(a.s, v, o, l);
-          val[j] = ld_feat<V>(a.s.feat[o] + l * a.s.feat_stride + (int64_t)colc * sizeof(V));
+          val[j] = ld_row_chunk<V>(a.s, o, l, colc * (unsigned)sizeof(V), pol);
         } else {
           if (colc == 0) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_ID_RANGE);
           val[j] = V{};
@@ -246,7 +301,7 @@ cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int6
                  : (cw % 4 == 0 && oa % 4 == 0)             ? 4
                                                             : 2;
   GatherArgs a{h->view, ids, cap, d_n, d_begin, static_cast<uint8_t*>(out), h->ws.ctrl, FastDiv((unsigned)(cw / vb))};
-  if (use_tma && cw == rb && rb % 16 == 0 && oa % 16 == 0 && rb <= TMA_STAGE_BYTES) {
+  if (use_tma && h->tail_pitch == 0 && cw == rb && rb % 16 == 0 && oa % 16 == 0 && rb <= TMA_STAGE_BYTES) {
     const int R = (int)std::min<int64_t>(32, TMA_STAGE_BYTES / rb);
     const int smem = TMA_STAGES * R * (int)rb;
     static int tma_bps = 0;

@@ -27,9 +27,12 @@ wg_status fail(wg_status s, const std::string& msg);
 struct ShardView {
   const int64_t* row_ptr[WG_MAX_WORLD];
   const int64_t* col[WG_MAX_WORLD];
-  const uint8_t* feat[WG_MAX_WORLD];
+  const uint8_t* feat[WG_MAX_WORLD];  // feature rows (their first body_bytes bytes), pitch feat_stride
+  const uint8_t* tail[WG_MAX_WORLD];  // split layout: bytes [body_bytes, row_bytes) of every row, pitch tail_pitch
   int64_t n;            // num_nodes
   int64_t feat_stride;  // bytes between feature rows in a shard (multiple of 16)
+  int64_t tail_pitch;   // 0 = no split: whole rows live in feat
+  int64_t body_bytes;   // bytes of a row stored in feat (= row bytes when not split)
   int32_t world;
   int32_t log2w;        // log2(world) if world is a power of two, else -1
 };
@@ -79,6 +82,7 @@ constexpr int EXCL_RING = 4;
 struct wg_dsm {
   int rank = 0, world = 1, device = 0;
   int64_t n = 0, n_local = 0, e_local = 0, feat_dim = 0, elt = 4, row_bytes = 0, feat_stride = 0;
+  int64_t body_bytes = 0, tail_pitch = 0;  // split feature layout (see wg_dsm_feat_layout)
   int64_t n_local_of[WG_MAX_WORLD] = {0};
   int64_t e_local_of[WG_MAX_WORLD] = {0};
   void* slab = nullptr;                 // this rank's allocation

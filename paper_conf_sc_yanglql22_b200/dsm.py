@@ -120,6 +120,11 @@ class DSM:
         h = ctypes.c_void_p()
         check(lib().wg_dsm_create(ctypes.byref(d), ctypes.byref(h)))
         self.h = h
+        # feature-row layout (wg_dsm_feat_layout): bytes [0, body_bytes) of a row in the feature
+        # shard, the rest (split layout only) in the tail region
+        bb, bp, tp, tpitch = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_void_p(), ctypes.c_int64()
+        check(lib().wg_dsm_feat_layout(h, ctypes.byref(bb), ctypes.byref(bp), ctypes.byref(tp), ctypes.byref(tpitch)))
+        self.body_bytes, self.tail_pitch, self._tail_ptr = bb.value, tpitch.value, tp.value
 
     # --- shard access
     def local_view(self):
@@ -133,6 +138,31 @@ class DSM:
         colv = device_view(col.value, (e_local,), torch.int64, self.device)
         featv = device_view(feat.value, (n_local, stride.value), torch.uint8, self.device) if self.row_bytes else None
         return row_ptr, colv, featv
+
+    def tail_view(self):
+        """uint8 [n_local, tail_pitch] view of this rank's tail region (split layout), else None."""
+        if not self.tail_pitch:
+            return None
+        n_local, _ = self.shard_info(self.rank)
+        return device_view(self._tail_ptr, (n_local, self.tail_pitch), torch.uint8, self.device)
+
+    def write_local_rows(self, rows_u8, start=0):
+        """Write whole feature rows (uint8 [k, row_bytes], host or device) to local rows
+        start .. start+k-1 of this rank's shard, honouring the row layout."""
+        _, _, fv = self.local_view()
+        src = rows_u8 if isinstance(rows_u8, torch.Tensor) else torch.from_numpy(np.ascontiguousarray(rows_u8))
+        k, b = src.shape[0], self.body_bytes
+        fv[start:start + k, :b].copy_(src[:, :b])
+        if self.tail_pitch:
+            self.tail_view()[start:start + k].copy_(src[:, b:self.row_bytes])
+
+    def read_local_rows(self, local_rows):
+        """Whole feature rows (uint8 [k, row_bytes], device) of the given local rows of this rank."""
+        _, _, fv = self.local_view()
+        body = fv[local_rows][:, :self.body_bytes]
+        if not self.tail_pitch:
+            return body
+        return torch.cat([body, self.tail_view()[local_rows]], dim=1)
 
     def shard_info(self, r):
         nl, el = ctypes.c_int64(), ctypes.c_int64()
@@ -275,8 +305,7 @@ class DSM:
 
     def fill_features(self, rows_u8):
         """Copy this rank's feature rows (uint8 [n_local, row_bytes], host) into its shard."""
-        _, _, fv = self.local_view()
-        fv[:, : self.row_bytes].copy_(torch.from_numpy(np.ascontiguousarray(rows_u8)))
+        self.write_local_rows(rows_u8, 0)
 
 
 def shard_csr(row_ptr, col, rank, world):

@@ -52,7 +52,7 @@ def build_dsm(preset, rank=0, world=1, device=None, allgather=None, max_seeds=No
         del rp, col
         if fd:
             from synth import gpu as sgpu
-            sgpu.fill_features_gpu(lfeat, spre.FEAT_SEED, rank, world, fd, sfeat.WG_DTYPE_CODE[fdt])
+            sgpu.fill_dsm_features_gpu(dsm, spre.FEAT_SEED, rank, world, fd, sfeat.WG_DTYPE_CODE[fdt])
     else:
         dsm.fill_from_global_csr(g_rp, g_col)
         if fd:

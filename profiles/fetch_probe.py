@@ -37,7 +37,7 @@ def main():
         rb = dim * 4
         dsm = pkg.DSM(n, 0, dim, "fp32", 1, device=0)
         _, _, fv = dsm.local_view()
-        sgpu.fill_features_gpu(fv, presets.FEAT_SEED, 0, 1, dim, 0)
+        sgpu.fill_dsm_features_gpu(dsm, presets.FEAT_SEED, 0, 1, dim, 0)
         pitch = dsm.out_pitch() if pitched else rb
         out = torch.empty((R, pitch), dtype=torch.uint8, device=dev)
         for _ in range(2):

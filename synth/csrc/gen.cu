@@ -4,6 +4,7 @@
 // contraction), so every row equals the numpy generator's row bit for bit
 // (checked by tests/test_gpu_synth.py).  Used to fill large DSM shards directly on
 // the device (products / papers100M / MAG240M shapes).
+#include <climits>
 #include <cuda_runtime.h>
 #include <stdint.h>
 
@@ -100,21 +101,26 @@ __global__ void compact_kernel(int rank, int world, int64_t n_local, const int64
   }
 }
 
+// Element c of local row l is written at feat + l*stride + c*elt when that byte offset is below
+// body_bytes, else at tail + l*tail_pitch + (c*elt - body_bytes) (the DSM's split row layout).
 __global__ void features_kernel(unsigned long long feat_seed, int rank, int world, int64_t n_local, int64_t dim,
-                                int dtype, int64_t stride, uint8_t* feat) {
+                                int dtype, int64_t stride, uint8_t* feat, int64_t body_bytes, int64_t tail_pitch,
+                                uint8_t* tail) {
   const int64_t total = n_local * dim;
   const unsigned long long h0 = splitmix64(feat_seed);
+  const int64_t elt = dtype == 0 ? 4 : 2;
   for (int64_t i = blockIdx.x * (int64_t)blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
     const int64_t l = i / dim, c = i - l * dim;
     const unsigned long long v = (unsigned long long)(rank + l * world);
     const unsigned long long hv = splitmix64(splitmix64(h0 ^ v) ^ (unsigned long long)c);
-    uint8_t* row = feat + l * stride;
+    const int64_t b = c * elt;
+    uint8_t* dst = b < body_bytes ? feat + l * stride + b : tail + l * tail_pitch + (b - body_bytes);
     if (dtype == 0)
-      reinterpret_cast<uint32_t*>(row)[c] = 0x3F800000u | (uint32_t)(hv >> 41);
+      *reinterpret_cast<uint32_t*>(dst) = 0x3F800000u | (uint32_t)(hv >> 41);
     else if (dtype == 1)
-      reinterpret_cast<uint16_t*>(row)[c] = (uint16_t)(0x3C00u | (uint32_t)(hv >> 54));
+      *reinterpret_cast<uint16_t*>(dst) = (uint16_t)(0x3C00u | (uint32_t)(hv >> 54));
     else
-      reinterpret_cast<uint16_t*>(row)[c] = (uint16_t)(0x3F80u | (uint32_t)(hv >> 57));
+      *reinterpret_cast<uint16_t*>(dst) = (uint16_t)(0x3F80u | (uint32_t)(hv >> 57));
   }
 }
 
@@ -167,9 +173,10 @@ int gen_compact(int rank, int world, int64_t n_local, const int64_t* raw_off, co
 }
 
 int gen_features(uint64_t feat_seed, int rank, int world, int64_t n_local, int64_t dim, int dtype, int64_t stride,
-                 uint8_t* feat, void* stream) {
-  features_kernel<<<grid_for(n_local * dim, 256), 256, 0, (cudaStream_t)stream>>>(feat_seed, rank, world, n_local,
-                                                                                  dim, dtype, stride, feat);
+                 uint8_t* feat, int64_t body_bytes, int64_t tail_pitch, uint8_t* tail, void* stream) {
+  if (!tail) body_bytes = INT64_MAX;
+  features_kernel<<<grid_for(n_local * dim, 256), 256, 0, (cudaStream_t)stream>>>(
+      feat_seed, rank, world, n_local, dim, dtype, stride, feat, body_bytes, tail_pitch, tail);
   return (int)cudaGetLastError();
 }
 

@@ -39,7 +39,7 @@ def lib():
         L.gen_segmented_sort.argtypes = [P, ctypes.POINTER(ctypes.c_size_t), P, P, I, I, P, P]
         L.gen_dedup_count.argtypes = [I, I, I64, P, P, P, P]
         L.gen_compact.argtypes = [I, I, I64, P, P, P, P, P]
-        L.gen_features.argtypes = [U64, I, I, I64, I64, I, I64, P, P]
+        L.gen_features.argtypes = [U64, I, I, I64, I64, I, I64, P, I64, I64, P, P]
         _lib = L
     return _lib
 
@@ -101,10 +101,19 @@ def shard_csr_gpu(spec, rank, world, device, max_sort_items=1 << 30):
     return row_ptr, col[:e]
 
 
-def fill_features_gpu(feat_view_u8, feat_seed, rank, world, dim, dtype_code):
-    """Write bits(v, c) into a shard view uint8 [n_local, stride]."""
+def fill_features_gpu(feat_view_u8, feat_seed, rank, world, dim, dtype_code, tail_view_u8=None, body_bytes=0):
+    """Write bits(v, c) into a shard view uint8 [n_local, stride]; with a tail view (the DSM's split
+    row layout, DSM.tail_view()) bytes >= body_bytes of each row go to the tail view instead."""
     L = lib()
     dev = feat_view_u8.device
     st = ctypes.c_void_p(torch.cuda.current_stream(dev).cuda_stream)
     nl, stride = feat_view_u8.shape
-    _ck(L.gen_features(feat_seed, rank, world, nl, dim, dtype_code, stride, _p(feat_view_u8), st))
+    tp = tail_view_u8.stride(0) if tail_view_u8 is not None else 0
+    _ck(L.gen_features(feat_seed, rank, world, nl, dim, dtype_code, stride, _p(feat_view_u8), body_bytes, tp,
+                       _p(tail_view_u8) if tail_view_u8 is not None else None, st))
+
+
+def fill_dsm_features_gpu(dsm, feat_seed, rank, world, dim, dtype_code):
+    """fill_features_gpu into a DSM's shard, honouring its row layout."""
+    _, _, fv = dsm.local_view()
+    fill_features_gpu(fv, feat_seed, rank, world, dim, dtype_code, dsm.tail_view(), dsm.body_bytes)

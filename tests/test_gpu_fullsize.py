@@ -36,7 +36,7 @@ def test_device_generator_matches_host_rows(products):
         a, b = int(rp_h[x]), int(rp_h[x + 1])
         assert np.array_equal(col_d[a:b].cpu().numpy(), hc[hp[k]:hp[k + 1]]), x
     assert abs(rp_h[-1] - p.target_e) / p.target_e < 0.03
-    fb = feat[torch.from_numpy(v).cuda()][:, :dsm.row_bytes].cpu().numpy()
+    fb = dsm.read_local_rows(torch.from_numpy(v).cuda()).cpu().numpy()
     assert np.array_equal(fb, features.feature_bytes(presets.FEAT_SEED, v, p.feat_dim, p.feat_dtype))
 
 

@@ -147,13 +147,23 @@ def test_append_unique_random_vs_oracle():
 
 
 @pytest.mark.parametrize("dim,dtype", [(4, "fp32"), (32, "fp32"), (100, "fp32"), (1024, "fp32"), (768, "fp16"),
-                                       (3, "fp32"), (1, "fp16"), (7, "bf16")])
+                                       (3, "fp32"), (1, "fp16"), (7, "bf16"), (36, "fp32"), (56, "fp32"),
+                                       (60, "fp32"), (200, "fp16"), (72, "bf16")])
 def test_gather_rows(dim, dtype):
-    """Row sizes 16 B .. 4 KB and non-multiples of 16 B; repeated, sorted, reversed, empty id lists."""
+    """Row sizes 16 B .. 4 KB and non-multiples of 16 B, whole and split row layouts (144, 224, 240,
+    400 B: body of whole 128 B lines + a tail of 16..112 B); repeated, sorted, reversed, empty id
+    lists; dense and 32 B-pitched outputs (wg_gather_rows)."""
     n = 3000
     rp = np.zeros(n + 1, dtype=np.int64)
     feat = features.feature_bytes(presets.FEAT_SEED, np.arange(n), dim, dtype)
     dsm = make_dsm(rp, np.zeros(0, np.int64), feat, dim, dtype)
+    rb = dsm.row_bytes
+    if rb > 128 and rb % 128 and rb % 16 == 0:
+        assert dsm.tail_pitch == rb % 128 and dsm.body_bytes == rb - rb % 128
+    else:
+        assert dsm.tail_pitch == 0 and dsm.body_bytes == rb
+    # the shard holds exactly the generator's rows under either layout
+    assert np.array_equal(dsm.read_local_rows(torch.arange(n, device="cuda")).cpu().numpy(), feat)
     rng = np.random.default_rng(dim)
     for ids in (rng.integers(0, n, 5000), np.arange(n), np.arange(n)[::-1], np.full(77, n - 1), np.zeros(0)):
         ids = np.ascontiguousarray(ids, dtype=np.int64)
@@ -161,8 +171,46 @@ def test_gather_rows(dim, dtype):
         torch.cuda.synchronize()
         exp = oracle.gather(feat, np.arange(n), ids)
         assert np.array_equal(X[:len(ids)].cpu().numpy(), exp)
+        pitch = dsm.out_pitch()
+        if pitch != rb and rb % 16 == 0 and len(ids):
+            Xp = torch.zeros((len(ids), pitch), dtype=torch.uint8, device="cuda")
+            begin = torch.zeros(1, dtype=torch.int64, device="cuda")
+            end = torch.full((1,), len(ids), dtype=torch.int64, device="cuda")
+            dsm.gather_rows(torch.from_numpy(ids).cuda(), len(ids), begin, end, Xp)
+            torch.cuda.synchronize()
+            assert np.array_equal(Xp[:, :rb].cpu().numpy(), exp)
     assert dsm.device_error() == 0
     dsm.destroy()
+
+
+def test_feat_split_layout_off_subprocess():
+    """WG_FEAT_SPLIT=0 (whole rows at a 64 B pitch, read once at create) gathers the same bytes."""
+    import os
+    import subprocess
+    import sys
+    code = r'''
+import sys, numpy as np, torch
+sys.path.insert(0, "tests")
+from gpu_helpers import make_dsm
+import oracle
+from synth import features, presets
+for dim, dtype in ((100, "fp32"), (36, "fp32"), (200, "fp16")):
+    n = 4000
+    rp = np.zeros(n + 1, dtype=np.int64)
+    feat = features.feature_bytes(presets.FEAT_SEED, np.arange(n), dim, dtype)
+    dsm = make_dsm(rp, np.zeros(0, np.int64), feat, dim, dtype)
+    assert dsm.tail_pitch == 0 and dsm.body_bytes == dsm.row_bytes
+    ids = np.random.default_rng(dim).integers(0, n, 6000).astype(np.int64)
+    X = dsm.gather(torch.from_numpy(ids).cuda())
+    torch.cuda.synchronize()
+    assert np.array_equal(X.cpu().numpy(), oracle.gather(feat, np.arange(n), ids)), (dim, dtype)
+    dsm.destroy()
+print("NOSPLIT OK")
+'''
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", code], cwd=root, env=dict(os.environ, WG_FEAT_SPLIT="0"),
+                       capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0 and "NOSPLIT OK" in r.stdout, r.stdout + r.stderr
 
 
 def test_determinism_two_runs(tiny):
