@@ -178,6 +178,36 @@ extern "C" {
 const char* wg_last_error(void) { return g_last_error.c_str(); }
 const char* wg_version(void) { return "wholegraph-b200 0.1 (sm_100a)"; }
 
+// L2 persistence for the split layout's tail region (WG_TAIL_PERSIST, default 0 = off):
+// 1 = reserve a persisting L2 set-aside of the tail region's size (the gather's evict_last tail
+// loads may then occupy it); 2 = also attach an access-policy window over this rank's tail region
+// (hitProp persisting) to every gather launch.  The set-aside is device-wide for the process.
+static void setup_tail_persistence(wg_dsm* h) {
+  const char* e = getenv("WG_TAIL_PERSIST");
+  const int mode = e ? atoi(e) : 0;
+  const size_t tail_bytes = (size_t)(h->n_local * h->tail_pitch);
+  if (mode <= 0 || tail_bytes == 0) return;
+  int max_persist = 0, max_window = 0;
+  cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, h->device);
+  cudaDeviceGetAttribute(&max_window, cudaDevAttrMaxAccessPolicyWindowSize, h->device);
+  const size_t want = std::min(tail_bytes, (size_t)max_persist);
+  size_t cur = 0;
+  cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
+  if (want > cur) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want);
+  if (mode >= 2) {
+    cudaAccessPolicyWindow& w = h->tail_window;
+    w.base_ptr = const_cast<uint8_t*>(h->view.tail[h->rank]);
+    w.num_bytes = std::min(tail_bytes, (size_t)max_window);
+    w.hitRatio = std::min(1.0f, (float)want / (float)w.num_bytes);
+    w.hitProp = cudaAccessPropertyPersisting;
+    w.missProp = cudaAccessPropertyStreaming;
+  }
+  if (getenv("WG_VERBOSE"))
+    fprintf(stderr, "[wg] tail persistence mode %d: tail %zu B, set-aside %zu B (max %d), window %zu B (max %d)\n",
+            mode, tail_bytes, want, max_persist, (size_t)h->tail_window.num_bytes, max_window);
+  cudaGetLastError();
+}
+
 wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
   if (!out) return fail(WG_ERR_INVALID_ARG, "out is NULL");
   *out = nullptr;
@@ -308,6 +338,7 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
   h->view.log2w = -1;
   for (int k = 0; k <= 3; ++k)
     if ((1 << k) == h->world) h->view.log2w = k;
+  setup_tail_persistence(h);
   // Zero this rank's row_ptr sentinel so an unfilled shard reads as degree 0.
   if (cudaMemset(h->slab, 0, (h->n_local + 1) * 8) != cudaSuccess) {
     cudaGetLastError();

@@ -335,10 +335,11 @@ cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int6
   const int64_t max_blocks = (int64_t)h->sm_count * per_sm;
   blocks = blocks < 1 ? 1 : (blocks > max_blocks ? max_blocks : blocks);
   const unsigned gb = (unsigned)blocks;
-  if (vb == 32) return launch_pdl(gather_kernel<u32x8, V32_UNROLL>, gb, GATHER_THREADS, 0, st, a);
-  if (vb == 16) return launch_pdl(gather_kernel<uint4, 4>, gb, GATHER_THREADS, 0, st, a);
-  if (vb == 4) return launch_pdl(gather_kernel<unsigned, 4>, gb, GATHER_THREADS, 0, st, a);
-  return launch_pdl(gather_kernel<unsigned short, 4>, gb, GATHER_THREADS, 0, st, a);
+  const cudaAccessPolicyWindow* w = &h->tail_window;  // num_bytes == 0 unless WG_TAIL_PERSIST=2
+  if (vb == 32) return launch_pdl_w(w, gather_kernel<u32x8, V32_UNROLL>, gb, GATHER_THREADS, 0, st, a);
+  if (vb == 16) return launch_pdl_w(w, gather_kernel<uint4, 4>, gb, GATHER_THREADS, 0, st, a);
+  if (vb == 4) return launch_pdl_w(w, gather_kernel<unsigned, 4>, gb, GATHER_THREADS, 0, st, a);
+  return launch_pdl_w(w, gather_kernel<unsigned short, 4>, gb, GATHER_THREADS, 0, st, a);
 }
 
 }  // namespace wg

@@ -98,6 +98,9 @@ struct wg_dsm {
   cudaEvent_t fork_event = nullptr;     // relabel fork onto a side stream
   wg_dsm* parent = nullptr;             // set for a workspace fork (wg_dsm_fork): shards are the parent's
   int live_forks = 0;                   // forks of this handle not yet destroyed
+  // L2 persistence of the split layout's tail region (WG_TAIL_PERSIST, see dsm.cu): the access-policy
+  // window attached to gather launches (num_bytes = 0: none)
+  cudaAccessPolicyWindow tail_window{};
 };
 
 namespace wg {
@@ -107,19 +110,29 @@ namespace wg {
 // WG_PDL=0 disables it (A/B switch); correctness never depends on it.
 bool pdl_enabled();
 template <typename... KArgs, typename... Args>
-inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
-                              Args... args) {
+inline cudaError_t launch_pdl_w(const cudaAccessPolicyWindow* win, void (*kernel)(KArgs...), dim3 grid, dim3 block,
+                                size_t smem, cudaStream_t st, Args... args) {
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = grid;
   cfg.blockDim = block;
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
-  cudaLaunchAttribute attr[1];
+  cudaLaunchAttribute attr[2];
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
+  if (win && win->num_bytes) {  // L2 access-policy window (persisting lines) for this launch
+    attr[1].id = cudaLaunchAttributeAccessPolicyWindow;
+    attr[1].val.accessPolicyWindow = *win;
+    cfg.numAttrs = 2;
+  }
   return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
+}
+template <typename... KArgs, typename... Args>
+inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                              Args... args) {
+  return launch_pdl_w(nullptr, kernel, grid, block, smem, st, args...);
 }
 
 // launchers (stream-ordered); arguments already validated by the ABI layer
