@@ -48,6 +48,13 @@ def parse():
     ap.add_argument("--pass-b", default="both", choices=["both", "prep", "gather"],
                     help="diagnostics: run only the prep or only the gather in the throughput pass")
     ap.add_argument("--compare-gather", action="store_true", help="NEXT #1: P2P vs distributed-memory gather")
+    ap.add_argument("--gather-occupancy", type=int, default=None,
+                    help="gather blocks per SM in the throughput pass (default: pipeline.THROUGHPUT_GATHER_OCCUPANCY "
+                         "when more than 3 batches are in flight; 0 = occupancy maximum)")
+    ap.add_argument("--placement", default="dsm", choices=["dsm", "replicas"],
+                    help="dsm (default, the paper's method): graph + features row-sharded over the W GPUs, remote "
+                         "rows read over NVLink; replicas (SURVEY 8(e) lever, labelled): every GPU holds the whole "
+                         "graph + table (a W=1 DSM each) when it fits in its HBM, no NVLink traffic")
     ap.add_argument("--chase-accesses", type=int, default=100_000)
     return ap.parse_args()
 
@@ -168,10 +175,12 @@ def bench_reference(args):
     emit(line, args)
 
 
-def workload_config(p, W, flushed=True):
+def workload_config(p, W, flushed=True, placement="dsm"):
+    par = (f"dsm-w{W} (row-sharded CSR+features, P2P loads, no hot-path collective)" if placement == "dsm" else
+           f"replicas-x{W} (SURVEY 8(e) lever: whole graph + table on every GPU, no NVLink, no hot-path collective)")
     return {"workload": p.name, "nodes": p.n, "csr_entries_target": p.target_e, "fanouts": p.fanouts,
             "seeds_per_gpu": p.seeds_per_batch, "features": f"{p.feat_dim}x{p.feat_dtype}",
-            "parallelism": f"dsm-w{W} (row-sharded CSR+features, P2P loads, no hot-path collective)",
+            "parallelism": par,
             "l2": "flushed between steps (512 MB write outside the events)" if flushed else "not flushed",
             "note": p.note}
 
@@ -238,7 +247,10 @@ def bench_wg(args):
     S = p.seeds_per_batch
     P = max(1, args.concurrency)
     t0 = time.perf_counter()
-    dsm, info = loader.build_dsm(p, rank=rank, world=world, device=local, allgather=ag)
+    if args.placement == "replicas":  # every rank its own whole copy (a W=1 DSM); batches still b = r mod W
+        dsm, info = loader.build_dsm(p, rank=0, world=1, device=local, allgather=None)
+    else:
+        dsm, info = loader.build_dsm(p, rank=rank, world=world, device=local, allgather=ag)
     setup_s = time.perf_counter() - t0
     # P independent batch pipelines on P streams; pipeline j > 0 runs on a workspace fork of the DSM
     handles = [dsm] + [dsm.fork() for _ in range(P - 1)]
@@ -256,11 +268,16 @@ def bench_wg(args):
         for pl in pipes:
             pl.run(seeds_dev[k], rngs[k])
     torch.cuda.synchronize()
-    graphs, full_graphs = [], []
+    from paper_conf_sc_yanglql22_b200 import pipeline as pipemod
+    occ_b = args.gather_occupancy
+    if occ_b is None:
+        occ_b = pipemod.THROUGHPUT_GATHER_OCCUPANCY if P >= 4 else 0
+    graphs, full_graphs, tput_graphs = [], [], []
     for pl, st in zip(pipes, streams):
         if args.no_graph:
             graphs.append((None, None))
             full_graphs.append(None)
+            tput_graphs.append(None)
             continue
         st.wait_stream(torch.cuda.current_stream())
         gp, gg, gf = torch.cuda.CUDAGraph(), torch.cuda.CUDAGraph(), torch.cuda.CUDAGraph()
@@ -268,10 +285,14 @@ def bench_wg(args):
             pl.enqueue(gather=False)
         with torch.cuda.graph(gg, stream=st):      # ... then the whole gather (the roofline kernel)
             pl.enqueue_gather()
-        with torch.cuda.graph(gf, stream=st):      # pass B: the batch as shipped (incremental gather)
-            pl.enqueue(gather=True)
+        with torch.cuda.graph(gf, stream=st):      # pass A': the batch as shipped (incremental gather)
+            pl.enqueue(gather=True, gather_occupancy=0)
+        gb = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(gb, stream=st):      # pass B: the same with the throughput gather occupancy
+            pl.enqueue(gather=True, gather_occupancy=occ_b)
         graphs.append((gp, gg))
         full_graphs.append(gf)
+        tput_graphs.append(gb)
     torch.cuda.synchronize()
 
     def launch(j, k, st):
@@ -293,21 +314,24 @@ def bench_wg(args):
             else:
                 pl.enqueue_gather()
 
-    def whole(j, k, st):
-        """batch k through pipeline j as one graph: hops + incremental gather."""
+    def whole(j, k, st, tput=False):
+        """batch k through pipeline j as one graph: hops + incremental gather (tput: the gathers at
+        the throughput occupancy, for batches prepared concurrently)."""
         pl = pipes[j]
+        g = (tput_graphs if tput else full_graphs)[j]
         with torch.cuda.stream(st):
             pl.set_inputs(seeds_dev[k], rngs[k])
-            if full_graphs[j] is not None:
-                full_graphs[j].replay()
+            if g is not None:
+                g.replay()
             else:
-                pl.enqueue()
+                pl.enqueue(gather_occupancy=occ_b if tput else 0)
 
     for k in range(args.warmup):     # warm the graphs
         for j in range(P):
             launch(j, k, streams[j])
             gather(j, streams[j])
             whole(j, k, streams[j])
+            whole(j, k, streams[j], tput=True)
     torch.cuda.synchronize()
     for h in handles:
         err = h.device_error()
@@ -368,7 +392,7 @@ def bench_wg(args):
     for i in range(args.steps):
         for j in range(P):
             if args.pass_b == "both":
-                whole(j, n_single + args.warmup + i * P + j, streams[j])
+                whole(j, n_single + args.warmup + i * P + j, streams[j], tput=True)
                 continue
             if args.pass_b != "gather":
                 launch(j, n_single + args.warmup + i * P + j, streams[j])
@@ -406,7 +430,8 @@ def bench_wg(args):
     # peer bandwidth per direction, B200_PROFILING.md; 900 nominal) and bounds the kernel.
     peak, peak_src = peaks()
     hbm_bytes = float(2 * rows.sum() * rb)
-    nvl_bytes = float((world - 1) / world * rows.sum() * rb)
+    wd = world if args.placement == "dsm" else 1  # replicas: every row is local
+    nvl_bytes = float((wd - 1) / wd * rows.sum() * rb)
     t_hbm = hbm_bytes / (peak * 1e9)
     t_nvl = nvl_bytes / 770e9
     if t_nvl > t_hbm:
@@ -419,7 +444,7 @@ def bench_wg(args):
     # ---- e2e through the public API (MiniBatchLoader): every batch = H2D of its seeds from pinned host
     # memory + the batch graph + D2H of its per-hop counts, P batches in flight (as pass B), host-timed
     # from the first submit to the last batch handed out
-    loader_ = pkg.MiniBatchLoader(dsm, p.fanouts, S, depth=P)
+    loader_ = pkg.MiniBatchLoader(dsm, p.fanouts, S, depth=P, gather_occupancy=occ_b)
     host_seeds = [seeds_dev[k % n_single].cpu().pin_memory() for k in range(args.e2e_steps * P)]
     warm = [(host_seeds[k % len(host_seeds)], rngs[k % n_single]) for k in range(2 * P)]
     for _ in loader_(warm):
@@ -448,8 +473,9 @@ def bench_wg(args):
             cpu = {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
                    "sample": f"{done} whole batches of {S} seeds (fanout {p.fanouts} + gather) of the same workload, "
                              f"{s_spent:.1f} s of single-threaded oracle work (row regeneration untimed)"}
-        cfg = workload_config(p, world, flush is not None)
+        cfg = workload_config(p, world, flush is not None, args.placement)
         cfg["concurrent_batches_per_gpu"] = P
+        cfg["gather_blocks_per_sm_throughput_pass"] = occ_b or "occupancy max"
         cfg["l2"] = ("pass A (single batch, roofline): L2 flushed between batches; pass B (value): continuous, "
                      "inputs (2 GB graph + features) >> 126 MB L2, every batch new")
         line = {
@@ -465,7 +491,7 @@ def bench_wg(args):
                              "hops_then_full_gather_ms": 1e3 * dev_s_single / args.steps},
             "roofline": {"kernel": "wg::gather_kernel", "bound": bound, "achieved": achieved, "peak": peak_used,
                          "unit": "GB/s", "frac": achieved / peak_used,
-                         "traffic": gather_traffic() if world == 1 else None,
+                         "traffic": gather_traffic() if wd == 1 else None,
                          "peak_source": peak_src_used,
                          "algorithmic_bytes_per_launch": alg_bytes / args.steps,
                          "gather_ms_per_launch": 1e3 * gather_s / args.steps,

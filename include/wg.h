@@ -264,6 +264,16 @@ wg_status wg_dsm_chase(wg_dsm_t h, int32_t rank, int64_t span_bytes, int64_t acc
 wg_status wg_gather_rows(wg_dsm_t h, const int64_t* d_ids, int64_t n_ids, const int64_t* d_begin,
                          const int64_t* d_end, void* d_out, int64_t out_pitch, wg_stream_t stream);
 
+/* Occupancy of this handle's gather launches (wg_gather, wg_gather_rows): at most blocks_per_sm
+ * resident 256-thread blocks per SM; 0 (the default) = the occupancy maximum, which keeps the most
+ * bytes in flight and is fastest for a gather running alone.  When several batches are prepared
+ * concurrently on one GPU (wg_dsm_fork), a smaller value leaves register file and warp slots to the
+ * latency-bound sampling / append-unique kernels of the other streams so they overlap the gather
+ * (measured in DESIGN.md).  Read when a gather is enqueued (so a captured CUDA graph keeps the value
+ * it was captured with); results never depend on it.  Errors: WG_ERR_INVALID_ARG if h is NULL or
+ * blocks_per_sm < 0. */
+wg_status wg_dsm_set_gather_occupancy(wg_dsm_t h, int32_t blocks_per_sm);
+
 /* Read (and optionally clear) the latched device error word.  Synchronises the
  * handle's device. */
 wg_status wg_device_error(wg_dsm_t h, uint32_t* code, int32_t clear);

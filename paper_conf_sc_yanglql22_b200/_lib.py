@@ -60,10 +60,11 @@ def lib():
     L.wg_spmm_mean_backward.argtypes = [P, I64, P, P, P, P, I64, P, I64, P]
     L.wg_device_error.argtypes = [P, P, I32]
     L.wg_dsm_reset_workspace.argtypes = [P, P]
+    L.wg_dsm_set_gather_occupancy.argtypes = [P, I32]
     for f in ("wg_dsm_create", "wg_dsm_fork", "wg_dsm_local_view", "wg_dsm_shard_info", "wg_dsm_feat_layout",
               "wg_dsm_destroy", "wg_sample_neighbors", "wg_append_unique", "wg_sample_hop", "wg_gather", "wg_gather_rows",
               "wg_dsm_chase", "wg_spmm_mean_forward", "wg_spmm_mean_backward", "wg_bucket_by_owner", "wg_rows_permute",
-              "wg_device_error", "wg_dsm_reset_workspace"):
+              "wg_device_error", "wg_dsm_reset_workspace", "wg_dsm_set_gather_occupancy"):
         getattr(L, f).restype = ctypes.c_int
     L.wg_last_error.restype = ctypes.c_char_p
     L.wg_last_error.argtypes = []
@@ -80,5 +81,5 @@ def check(status):
 
 EXPORTS = ["wg_dsm_create", "wg_dsm_fork", "wg_dsm_local_view", "wg_dsm_shard_info", "wg_dsm_feat_layout", "wg_dsm_destroy", "wg_sample_neighbors",
            "wg_append_unique", "wg_sample_hop", "wg_gather", "wg_gather_rows", "wg_dsm_chase", "wg_spmm_mean_forward",
-           "wg_spmm_mean_backward", "wg_bucket_by_owner", "wg_rows_permute", "wg_device_error", "wg_dsm_reset_workspace", "wg_last_error",
+           "wg_spmm_mean_backward", "wg_bucket_by_owner", "wg_rows_permute", "wg_device_error", "wg_dsm_reset_workspace", "wg_dsm_set_gather_occupancy", "wg_last_error",
            "wg_version"]

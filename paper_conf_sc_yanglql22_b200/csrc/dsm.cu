@@ -381,6 +381,13 @@ wg_status wg_dsm_shard_info(wg_dsm_t h, int32_t r, int64_t* n_local_rows, int64_
   return WG_OK;
 }
 
+wg_status wg_dsm_set_gather_occupancy(wg_dsm_t h, int32_t blocks_per_sm) {
+  if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
+  if (blocks_per_sm < 0) return fail(WG_ERR_INVALID_ARG, "blocks_per_sm < 0");
+  h->gather_bps = blocks_per_sm;
+  return WG_OK;
+}
+
 wg_status wg_dsm_fork(wg_dsm_t parent, int64_t max_batch_keys, wg_dsm_t* out) {
   if (!out) return fail(WG_ERR_INVALID_ARG, "out is NULL");
   *out = nullptr;

@@ -173,12 +173,14 @@ __global__ void __launch_bounds__(GATHER_THREADS) gather_kernel(const GatherArgs
 }
 
 // ---------------------------------------------------------------------------- TMA variant
-// One warp per block; the warp owns TMA_STAGES smem stages of R rows.  For each tile of
-// R consecutive output rows, lane r issues one bulk copy (cp.async.bulk, the TMA engine,
-// no registers involved) of row r from the owner shard into the stage, all signalling
-// one mbarrier with complete_tx; when the stage is full, lane 0 writes the whole tile
-// (R * row_bytes contiguous bytes of X) with ONE bulk smem->global store.  TMA_STAGES
-// tiles are in flight per warp.  Requires row_bytes % 16 == 0.
+// One warp per block; the warp owns TMA_STAGES shared-memory stages of R rows at the output pitch.
+// For each tile of R consecutive output rows, lane r issues the bulk copies (cp.async.bulk, the TMA
+// engine: no registers hold the bytes in flight) of row r from the owner shard into the stage -- one
+// copy for a whole row, or body + tail for the split layout -- all signalling one mbarrier with
+// complete_tx; when the stage is full, lane 0 writes the whole tile (R * pitch contiguous bytes of X)
+// with ONE bulk smem->global store.  TMA_STAGES tiles are in flight per warp.  The bytes in flight
+// live in shared memory, so the kernel leaves the register file and the warp slots to kernels of other
+// streams (concurrent batches).  Requires row_bytes, body/tail sizes and the pitch to be multiples of 16.
 constexpr int TMA_STAGES = 4;
 constexpr int TMA_STAGE_BYTES = 16 * 1024;
 
@@ -186,7 +188,15 @@ __device__ __forceinline__ unsigned smem_u32(const void* p) {
   return (unsigned)__cvta_generic_to_shared(p);
 }
 
-__global__ void __launch_bounds__(32) gather_tma_kernel(const GatherArgs a, int rows_per_tile, int row_bytes) {
+__device__ __forceinline__ void bulk_g2s(uint8_t* dst, const uint8_t* src, unsigned bytes, unsigned long long* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(smem_u32(dst)),
+      "l"(src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+__global__ void __launch_bounds__(32) gather_tma_kernel(const GatherArgs a, int rows_per_tile, int row_bytes,
+                                                        int pitch) {
   pdl_enter();
   extern __shared__ __align__(128) uint8_t smem[];
   __shared__ __align__(8) unsigned long long mbar[TMA_STAGES];
@@ -202,51 +212,56 @@ __global__ void __launch_bounds__(32) gather_tma_kernel(const GatherArgs a, int 
   int64_t begin = a.d_begin ? *a.d_begin : 0;
   begin = begin < 0 ? 0 : (begin > n ? n : begin);
   const int64_t* ids = a.ids + begin;
-  uint8_t* outp = a.out + begin * (int64_t)row_bytes;
+  uint8_t* outp = a.out + begin * (int64_t)pitch;
   n -= begin;
   const int R = rows_per_tile;
   const int64_t ntiles = (n + R - 1) / R;
+  const bool split = a.s.tail_pitch != 0;
+  const unsigned body = split ? (unsigned)a.s.body_bytes : (unsigned)row_bytes;
+  const unsigned tail = (unsigned)row_bytes - body;
   if (lane == 0) {
     for (int s = 0; s < TMA_STAGES; ++s)
       asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(smem_u32(&mbar[s])));
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
+  if (pitch > row_bytes)  // the bulk copies never write a row's padding: zero it once per stage
+    for (int s = 0; s < TMA_STAGES; ++s)
+      for (int r = lane; r < R; r += 32)
+        for (int c = row_bytes; c < pitch; c += 16)
+          *reinterpret_cast<uint4*>(smem + ((size_t)s * R + r) * pitch + c) = make_uint4(0, 0, 0, 0);
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
   __syncwarp();
 
   auto issue = [&](int64_t tile, int s) {
     const int64_t r0 = tile * R;
     const int rows = (int)min((int64_t)R, n - r0);
-    uint8_t* stage = smem + (size_t)s * R * row_bytes;
+    uint8_t* stage = smem + (size_t)s * R * pitch;
     bool ok = false;
-    const uint8_t* src = nullptr;
+    int o = 0;
+    int64_t l = 0;
     if (lane < rows) {
       const int64_t v = ids[r0 + lane];
       if (v >= 0 && v < a.s.n) {
-        int o;
-        int64_t l;
         owner_local(a.s, v, o, l);
-        src = a.s.feat[o] + l * a.s.feat_stride;
         ok = true;
       } else {
         latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_ID_RANGE);
-        uint4* z = reinterpret_cast<uint4*>(stage + (size_t)lane * row_bytes);
+        uint4* z = reinterpret_cast<uint4*>(stage + (size_t)lane * pitch);
         for (int c = 0; c < row_bytes / 16; ++c) z[c] = make_uint4(0, 0, 0, 0);
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // zero row visible to the bulk store
       }
     }
     const unsigned nvalid = __popc(__ballot_sync(FULL_MASK, ok));
-    if (lane == 0) {
-      asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // zero rows visible to the bulk store
+    if (lane == 0)
       asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(&mbar[s])),
                    "r"(nvalid * (unsigned)row_bytes)
                    : "memory");
-    }
     __syncwarp();
-    if (ok)
-      asm volatile(
-          "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-              smem_u32(stage + (size_t)lane * row_bytes)),
-          "l"(src), "r"(row_bytes), "r"(smem_u32(&mbar[s]))
-          : "memory");
+    if (ok) {
+      uint8_t* dst = stage + (size_t)lane * pitch;
+      bulk_g2s(dst, a.s.feat[o] + l * a.s.feat_stride, body, &mbar[s]);
+      if (split) bulk_g2s(dst + body, a.s.tail[o] + l * a.s.tail_pitch, tail, &mbar[s]);
+    }
   };
 
   int64_t k = 0;
@@ -264,10 +279,10 @@ __global__ void __launch_bounds__(32) gather_tma_kernel(const GatherArgs a, int 
         : "memory");
     const int64_t r0 = t * R;
     const int rows = (int)min((int64_t)R, n - r0);
-    uint8_t* stage = smem + (size_t)s * R * row_bytes;
+    uint8_t* stage = smem + (size_t)s * R * pitch;
     if (lane == 0) {
-      asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(outp + r0 * row_bytes),
-                   "r"(smem_u32(stage)), "r"((unsigned)(rows * row_bytes))
+      asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;" ::"l"(outp + r0 * pitch),
+                   "r"(smem_u32(stage)), "r"((unsigned)(rows * pitch))
                    : "memory");
       asm volatile("cp.async.bulk.commit_group;" ::: "memory");
       asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");  // stage may be refilled
@@ -301,9 +316,10 @@ cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int6
                  : (cw % 4 == 0 && oa % 4 == 0)             ? 4
                                                             : 2;
   GatherArgs a{h->view, ids, cap, d_n, d_begin, static_cast<uint8_t*>(out), h->ws.ctrl, FastDiv((unsigned)(cw / vb))};
-  if (use_tma && h->tail_pitch == 0 && cw == rb && rb % 16 == 0 && oa % 16 == 0 && rb <= TMA_STAGE_BYTES) {
-    const int R = (int)std::min<int64_t>(32, TMA_STAGE_BYTES / rb);
-    const int smem = TMA_STAGES * R * (int)rb;
+  const int64_t body = h->tail_pitch ? h->body_bytes : rb;
+  if (use_tma && rb % 16 == 0 && cw % 16 == 0 && body % 16 == 0 && oa % 16 == 0 && cw <= TMA_STAGE_BYTES) {
+    const int R = (int)std::min<int64_t>(32, TMA_STAGE_BYTES / cw);
+    const int smem = TMA_STAGES * R * (int)cw;
     static int tma_bps = 0;
     if (!tma_bps) {
       cudaFuncSetAttribute(gather_tma_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, TMA_STAGES * TMA_STAGE_BYTES);
@@ -311,11 +327,12 @@ cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int6
       cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_tma_kernel, 32, TMA_STAGES * TMA_STAGE_BYTES);
       tma_bps = nb > 0 ? nb : 2;
     }
+    const int want = bps > 0 ? bps : h->gather_bps;
+    const int per_sm = (want > 0 && want < tma_bps) ? want : tma_bps;
     const int64_t tiles = (cap + R - 1) / R;
-    int64_t gbk = (int64_t)h->sm_count * tma_bps;
+    int64_t gbk = (int64_t)h->sm_count * per_sm;
     gbk = std::max<int64_t>(1, std::min(gbk, tiles));
-    gather_tma_kernel<<<(unsigned)gbk, 32, smem, st>>>(a, R, (int)rb);
-    return cudaGetLastError();
+    return launch_pdl(gather_tma_kernel, (unsigned)gbk, 32, (size_t)smem, st, a, R, (int)rb, (int)cw);
   }
   // one full wave: resident blocks per SM (occupancy calculator, cached per vector width) x SMs
   static int occ[4] = {0, 0, 0, 0};
@@ -328,7 +345,8 @@ cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int6
     else cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<unsigned short, 4>, GATHER_THREADS, 0);
     occ[which] = nb > 0 ? nb : 4;
   }
-  const int per_sm = (bps > 0 && bps < occ[which]) ? bps : occ[which];
+  const int want = bps > 0 ? bps : h->gather_bps;  // env knob (A/B) overrides the handle's setting
+  const int per_sm = (want > 0 && want < occ[which]) ? want : occ[which];
   const int64_t total = cap * (cw / vb);
   const int unr = vb == 32 ? V32_UNROLL : 4;
   int64_t blocks = (total + GATHER_THREADS * unr - 1) / (GATHER_THREADS * unr);

@@ -98,6 +98,7 @@ struct wg_dsm {
   cudaEvent_t fork_event = nullptr;     // relabel fork onto a side stream
   wg_dsm* parent = nullptr;             // set for a workspace fork (wg_dsm_fork): shards are the parent's
   int live_forks = 0;                   // forks of this handle not yet destroyed
+  int gather_bps = 0;                   // wg_dsm_set_gather_occupancy (0 = occupancy maximum)
   // L2 persistence of the split layout's tail region (WG_TAIL_PERSIST, see dsm.cu): the access-policy
   // window attached to gather launches (num_bytes = 0: none)
   cudaAccessPolicyWindow tail_window{};

@@ -120,6 +120,7 @@ class DSM:
         h = ctypes.c_void_p()
         check(lib().wg_dsm_create(ctypes.byref(d), ctypes.byref(h)))
         self.h = h
+        self.gather_occupancy = 0
         # feature-row layout (wg_dsm_feat_layout): bytes [0, body_bytes) of a row in the feature
         # shard, the rest (split layout only) in the tail region
         bb, bp, tp, tpitch = ctypes.c_int64(), ctypes.c_int64(), ctypes.c_void_p(), ctypes.c_int64()
@@ -203,7 +204,7 @@ class DSM:
         h = ctypes.c_void_p()
         check(lib().wg_dsm_fork(self.h, max_batch_keys, ctypes.byref(h)))
         f.h = h
-        return f
+        return f  # the fork starts with the parent's gather occupancy (copied by wg_dsm_fork)
 
     # --- the three ops --------------------------------------------------------
     def sample_neighbors(self, targets, fanout, seed, hop, n_targets_dev=None, seed_dev=None, out_row_ptr=None,
@@ -281,6 +282,12 @@ class DSM:
         check(lib().wg_gather_rows(self.h, _ptr(ids), cap, _ptr(begin_dev), _ptr(end_dev), _ptr(out), pitch,
                                    _stream(stream)))
         return out
+
+    def set_gather_occupancy(self, blocks_per_sm):
+        """Resident gather blocks per SM for this handle's gathers (0 = occupancy maximum);
+        read at enqueue / capture time (wg_dsm_set_gather_occupancy)."""
+        check(lib().wg_dsm_set_gather_occupancy(self.h, int(blocks_per_sm)))
+        self.gather_occupancy = int(blocks_per_sm)
 
     def out_pitch(self):
         """Output row pitch that lets the gather move whole 32 B vectors (row bytes rounded up to 32)."""

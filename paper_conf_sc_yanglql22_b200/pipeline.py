@@ -30,10 +30,18 @@ def required_keys(n, fanouts, max_seeds):
     return max(t + e for t, e in zip(T, E))
 
 
+# Gather occupancy (resident gather blocks per SM, wg_dsm_set_gather_occupancy) for batches prepared
+# several at a time on one GPU: a gather at full occupancy holds the whole register file and keeps
+# the other streams' latency-bound hop kernels from overlapping it ("Concurrency").
+THROUGHPUT_GATHER_OCCUPANCY = 1
+
+
 class MiniBatchPipeline:
     def __init__(self, dsm: DSM, fanouts, max_seeds, with_pos=False, with_dup=False, fused=True,
-                 incremental_gather=True, gather_priority=0, side_priority=0):
+                 incremental_gather=True, gather_priority=0, side_priority=0, gather_occupancy=None):
         self.dsm, self.fanouts, self.max_seeds = dsm, list(fanouts), max_seeds
+        # None: use the handle's setting; an int: applied to this pipeline's gathers at enqueue
+        self.gather_occupancy = gather_occupancy
         self.fused = fused
         self.side = torch.cuda.Stream(device=dsm.device, priority=side_priority) if fused else None
         # incremental gather: U_{h-1} is a prefix of U_h, so the feature rows of hop h's new nodes
@@ -67,10 +75,22 @@ class MiniBatchPipeline:
         self.graph = None
 
     # -- enqueue one batch (reads seeds / n_seeds / rng_seed from device buffers)
-    def enqueue(self, stream=None, gather=True):
+    def enqueue(self, stream=None, gather=True, gather_occupancy=None):
         """Enqueue every hop (fused wg_sample_hop: sample + append-unique; the
         relabel of each hop runs on a side stream, joined at the end) and, unless
-        gather=False, the feature gather."""
+        gather=False, the feature gather.  gather_occupancy (else the pipeline's) sets
+        the gathers' blocks per SM for this enqueue only."""
+        occ = self.gather_occupancy if gather_occupancy is None else gather_occupancy
+        if occ is None or occ == self.dsm.gather_occupancy:
+            return self._enqueue(stream, gather)
+        prev = self.dsm.gather_occupancy
+        self.dsm.set_gather_occupancy(occ)
+        try:
+            return self._enqueue(stream, gather)
+        finally:
+            self.dsm.set_gather_occupancy(prev)
+
+    def _enqueue(self, stream=None, gather=True):
         d = self.dsm
         main = stream or torch.cuda.current_stream(d.device)
         if self.fused:
@@ -200,11 +220,14 @@ class MiniBatchLoader:
     order, keeping up to `depth` batches in flight; a slot is reused only after the
     consumer's stream has passed the point where the batch was handed out."""
 
-    def __init__(self, dsm: DSM, fanouts, max_seeds, depth=8, with_pos=False, with_dup=False, graphs=True):
+    def __init__(self, dsm: DSM, fanouts, max_seeds, depth=8, with_pos=False, with_dup=False, graphs=True,
+                 gather_occupancy="auto"):
         self.depth = max(1, depth)
         self.handles = [dsm] + [dsm.fork() for _ in range(self.depth - 1)]
-        self.pipes = [MiniBatchPipeline(h, fanouts, max_seeds, with_pos=with_pos, with_dup=with_dup)
-                      for h in self.handles]
+        if gather_occupancy == "auto":  # throughput mode when several batches share the GPU
+            gather_occupancy = THROUGHPUT_GATHER_OCCUPANCY if self.depth >= 4 else None
+        self.pipes = [MiniBatchPipeline(h, fanouts, max_seeds, with_pos=with_pos, with_dup=with_dup,
+                                        gather_occupancy=gather_occupancy) for h in self.handles]
         dev = dsm.device
         self.streams = [torch.cuda.Stream(device=dev) for _ in range(self.depth)]
         self.done = [torch.cuda.Event() for _ in range(self.depth)]

@@ -286,6 +286,17 @@ for dim, dtype in ((100, "fp32"), (4, "fp32"), (768, "fp16"), (1024, "fp32"), (3
         X = dsm.gather(torch.from_numpy(ids).cuda())
         torch.cuda.synchronize()
         assert np.array_equal(X[:len(ids)].cpu().numpy(), oracle.gather(feat, np.arange(n), ids)), (dim, dtype)
+        # pitched output through wg_gather_rows (rows [begin, end) only)
+        if len(ids) > 10:
+            pitch = dsm.out_pitch()
+            out = torch.full((len(ids), pitch), 0xAB, dtype=torch.uint8, device="cuda")
+            be = torch.tensor([5, len(ids) - 3], dtype=torch.int64, device="cuda")
+            dsm.gather_rows(torch.from_numpy(ids).cuda(), len(ids), be[0:1], be[1:2], out)
+            torch.cuda.synchronize()
+            o = out.cpu().numpy()
+            rb = dsm.row_bytes
+            assert np.array_equal(o[5:len(ids) - 3, :rb], oracle.gather(feat, np.arange(n), ids[5:len(ids) - 3]))
+            assert (o[:5] == 0xAB).all() and (o[len(ids) - 3:] == 0xAB).all()
     assert dsm.device_error() == 0
     dsm.destroy()
 print("TMA OK")
@@ -456,3 +467,27 @@ print("EPOCH OK")
                        env=dict(os.environ, WG_EPOCH_START=str((1 << 23) - 3)), capture_output=True, text=True,
                        timeout=600)
     assert r.returncode == 0 and "EPOCH OK" in r.stdout, r.stdout + r.stderr
+
+
+def test_gather_occupancy_setting(tiny):
+    """wg_dsm_set_gather_occupancy changes only the launch shape: every occupancy gathers the same
+    bytes, directly and through a captured pipeline graph (values restored after enqueue)."""
+    p, rp, col = tiny
+    dsm, _ = loader.build_dsm(p, on_device=False)
+    S = seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 5)
+    rs = seeds.rng_seed(presets.RNG_BASE, 5)
+    ref = oracle.minibatch(loader.host_row_provider(p.graph(), rp, col), loader.host_feat_provider(p), S,
+                           p.fanouts, rs)
+    for occ in (1, 2, 3, 0):
+        pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, gather_occupancy=occ)
+        pipe.run(torch.from_numpy(S).cuda(), rs)
+        pipe.capture()
+        pipe.X.zero_()
+        pipe.run(torch.from_numpy(S).cuda(), rs)
+        torch.cuda.synchronize()
+        assert dsm.gather_occupancy == 0
+        assert np.array_equal(pipe.features(), ref["X"]), occ
+    with pytest.raises(pkg.WgError):
+        dsm.set_gather_occupancy(-1)
+    assert dsm.device_error() == 0
+    dsm.destroy()
