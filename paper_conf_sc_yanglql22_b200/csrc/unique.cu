@@ -285,7 +285,12 @@ static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, c
   a.ctrl = h->ws.ctrl;
   a.n = h->n;
   const int64_t total = a.capT + a.capE;
-  const int64_t max_blocks = (int64_t)h->sm_count * 8;
+  static int prep_bps = -1;  // A/B knob WG_PREP_BPS: insert / relabel blocks per SM (default 8 = full occupancy)
+  if (prep_bps < 0) {
+    const char* e = getenv("WG_PREP_BPS");
+    prep_bps = (e && atoi(e) > 0) ? atoi(e) : 8;
+  }
+  const int64_t max_blocks = (int64_t)h->sm_count * prep_bps;
   int64_t ib = (total + UQ_THREADS - 1) / UQ_THREADS;
   ib = ib < 1 ? 1 : (ib > max_blocks ? max_blocks : ib);
   // items per thread: the largest of 8/4/2/1 that still gives >= 2 tiles per SM
