@@ -83,3 +83,23 @@ def test_two_processes_cuda_ipc(mode):
     for p, o in zip(procs, outs):
         assert p.returncode == 0, o
         assert "PARITY OK" in o, o
+
+
+@pytest.mark.parametrize("placement", ["dsm", "replicas"])
+def test_bench_torchrun_two_ranks(placement):
+    """The driver's N>1 launch of bench.py (torchrun, one process per rank) on the one test GPU:
+    every rank must reach the same collectives (max over ranks, barriers, collective destroy) and
+    rank 0 prints one JSON line with the whole-job value."""
+    import json
+    port = 29600 + os.getpid() % 500 + (3 if placement == "dsm" else 0)
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.join(ROOT, "bench.py"),
+           "--gpus", "2", "--steps", "3", "--warmup", "3", "--cpu-sample-s", "0", "--e2e-steps", "1",
+           "--concurrency", "2", "--config", "tiny", "--placement", placement]
+    r = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    d = json.loads(lines[0])
+    assert d["n_gpus"] == 2 and d["value"] > 0 and d["e2e"]["value"] > 0 and d["single_batch"]["value"] > 0
+    assert d["config"]["parallelism"].startswith("dsm-w2" if placement == "dsm" else "replicas-x2")
