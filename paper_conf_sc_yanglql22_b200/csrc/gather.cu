@@ -172,6 +172,113 @@ __global__ void __launch_bounds__(GATHER_THREADS) gather_kernel(const GatherArgs
   }
 }
 
+// ---------------------------------------------------------------------------- cp.async variant
+// The same flat 16 B chunk stream as gather_kernel<uint4>, but every thread's loads are
+// cp.async (LDGSTS) copies into shared memory: ASYNC_STAGES stages of ASYNC_K chunks per thread
+// are in flight, and a thread stores a stage (ld.shared -> st.global, coalesced) once its own
+// copies have landed (cp.async.wait_group; each thread reads back only what it copied, so no
+// block barrier is needed).  The bytes in flight live in shared memory instead of registers
+// (64 KB per 256-thread block), so the kernel needs few registers and leaves the register file
+// to the hop kernels of concurrent batches.  Chunks past a row (pitched output) or of an
+// invalid id are zero-filled by the copy itself (src-size 0).
+constexpr int ASYNC_THREADS = 256;
+constexpr int ASYNC_STAGES = 4;
+constexpr int ASYNC_K = 4;
+constexpr int ASYNC_SMEM = ASYNC_STAGES * ASYNC_K * ASYNC_THREADS * 16;
+
+__device__ __forceinline__ void cp_async16(void* sdst, const void* gsrc, unsigned src_bytes) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"((unsigned)__cvta_generic_to_shared(sdst)),
+               "l"(gsrc), "r"(src_bytes)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_wait(int pending) {
+  switch (pending) {  // wait_group takes an immediate
+    case 0: asm volatile("cp.async.wait_group 0;" ::: "memory"); break;
+    case 1: asm volatile("cp.async.wait_group 1;" ::: "memory"); break;
+    case 2: asm volatile("cp.async.wait_group 2;" ::: "memory"); break;
+    default: asm volatile("cp.async.wait_group 3;" ::: "memory"); break;
+  }
+}
+
+__global__ void __launch_bounds__(ASYNC_THREADS) gather_async_kernel(const GatherArgs a) {
+  pdl_enter();
+  extern __shared__ __align__(16) uint4 sbuf[];  // [ASYNC_STAGES][ASYNC_K][ASYNC_THREADS]
+  int64_t n = a.cap;
+  if (a.d_n) {
+    n = *a.d_n;
+    if (n > a.cap || n < 0) {
+      if (threadIdx.x == 0 && blockIdx.x == 0) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_CAPACITY);
+      n = n < 0 ? 0 : a.cap;
+    }
+  }
+  int64_t begin = a.d_begin ? *a.d_begin : 0;
+  begin = begin < 0 ? 0 : (begin > n ? n : begin);
+  const int64_t* __restrict__ ids = a.ids + begin;
+  n -= begin;
+  const unsigned cpr = a.cpr.d;
+  const unsigned total = (unsigned)(n * cpr);
+  uint4* __restrict__ out = reinterpret_cast<uint4*>(a.out + begin * (int64_t)cpr * 16);
+  const unsigned per_stage = ASYNC_THREADS * ASYNC_K;
+  const unsigned gstride = gridDim.x * per_stage;
+  const unsigned first = blockIdx.x * per_stage;
+  const unsigned tid = threadIdx.x;
+  const unsigned row_bytes = (unsigned)(a.s.tail_pitch ? a.s.body_bytes + a.s.tail_pitch : a.s.body_bytes);
+
+  auto issue = [&](unsigned base, int slot) {
+#pragma unroll
+    for (int k = 0; k < ASYNC_K; ++k) {
+      const unsigned c = base + (unsigned)k * ASYNC_THREADS + tid;
+      if (c < total) {
+        const unsigned row = a.cpr.div(c);
+        const unsigned boff = (c - row * cpr) * 16u;
+        const int64_t v = ids[row];
+        const void* src = a.s.feat[0];
+        unsigned bytes = 0;
+        if (v >= 0 && v < a.s.n) {
+          int o;
+          int64_t l;
+          owner_local(a.s, v, o, l);
+          if (a.s.tail_pitch == 0 || boff < (unsigned)a.s.body_bytes) {
+            src = a.s.feat[o] + l * a.s.feat_stride + boff;
+            bytes = 16;  // whole layout: a pitched chunk may cover the shard row's padding
+          } else if (boff < row_bytes) {
+            src = a.s.tail[o] + l * a.s.tail_pitch + (boff - (unsigned)a.s.body_bytes);
+            bytes = 16;
+          }  // else: output padding past a split row -> zeros
+        } else if (boff == 0) {
+          latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_ID_RANGE);
+        }
+        cp_async16(&sbuf[((size_t)slot * ASYNC_K + k) * ASYNC_THREADS + tid], src, bytes);
+      }
+    }
+    asm volatile("cp.async.commit_group;" ::: "memory");
+  };
+
+  unsigned next = first;
+  int issued = 0, done = 0;
+  while (issued < ASYNC_STAGES && next < total) {
+    issue(next, issued % ASYNC_STAGES);
+    next += gstride;
+    ++issued;
+  }
+  while (done < issued) {
+    cp_async_wait(issued - done - 1);  // this thread's copies of stage `done` have landed
+    const int slot = done % ASYNC_STAGES;
+    const unsigned base = first + (unsigned)done * gstride;
+#pragma unroll
+    for (int k = 0; k < ASYNC_K; ++k) {
+      const unsigned c = base + (unsigned)k * ASYNC_THREADS + tid;
+      if (c < total) out[c] = sbuf[((size_t)slot * ASYNC_K + k) * ASYNC_THREADS + tid];
+    }
+    ++done;
+    if (next < total) {  // refill the slot just drained
+      issue(next, slot);
+      next += gstride;
+      ++issued;
+    }
+  }
+}
+
 // ---------------------------------------------------------------------------- TMA variant
 // One warp per block; the warp owns TMA_STAGES shared-memory stages of R rows at the output pitch.
 // For each tile of R consecutive output rows, lane r issues the bulk copies (cp.async.bulk, the TMA
@@ -297,8 +404,11 @@ __global__ void __launch_bounds__(32) gather_tma_kernel(const GatherArgs a, int 
 cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int64_t* d_n, const int64_t* d_begin,
                           void* out, int64_t out_pitch, cudaStream_t st) {
   const int64_t rb = h->row_bytes;
-  static int knobs = 0, bps = 0, use_tma = 0, allow32 = 1;
-  if (!knobs) {  // A/B knobs, read once: WG_GATHER_BPS (blocks per SM), WG_GATHER_TMA=1, WG_GATHER_V32=0
+  static int knobs = 0, bps = 0, use_tma = 0, allow32 = 1, use_async = 0;
+  if (!knobs) {  // A/B knobs, read once: WG_GATHER_BPS (blocks per SM), WG_GATHER_TMA=1, WG_GATHER_V32=0,
+                 // WG_GATHER_ASYNC=1 (cp.async variant)
+    const char* ca = getenv("WG_GATHER_ASYNC");
+    use_async = (ca && ca[0] == '1') ? 1 : 0;
     const char* b = getenv("WG_GATHER_BPS");
     bps = b ? atoi(b) : 0;
     const char* t = getenv("WG_GATHER_TMA");
@@ -316,6 +426,25 @@ cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int6
                  : (cw % 4 == 0 && oa % 4 == 0)             ? 4
                                                             : 2;
   GatherArgs a{h->view, ids, cap, d_n, d_begin, static_cast<uint8_t*>(out), h->ws.ctrl, FastDiv((unsigned)(cw / vb))};
+  if (use_async && cw % 16 == 0 && oa % 16 == 0) {
+    static int async_bps = 0;
+    if (!async_bps) {
+      cudaFuncSetAttribute(gather_async_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, ASYNC_SMEM);
+      int nb = 0;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_async_kernel, ASYNC_THREADS, ASYNC_SMEM);
+      async_bps = nb > 0 ? nb : 1;
+    }
+    GatherArgs a16 = a;
+    a16.cpr = FastDiv((unsigned)(cw / 16));
+    const int want = bps > 0 ? bps : h->gather_bps;
+    const int per_sm = (want > 0 && want < async_bps) ? want : async_bps;
+    const int64_t total = cap * (cw / 16);
+    int64_t blocks = (total + ASYNC_THREADS * ASYNC_K - 1) / (ASYNC_THREADS * ASYNC_K);
+    const int64_t max_blocks = (int64_t)h->sm_count * per_sm;
+    blocks = blocks < 1 ? 1 : (blocks > max_blocks ? max_blocks : blocks);
+    return launch_pdl_w(&h->tail_window, gather_async_kernel, (unsigned)blocks, ASYNC_THREADS, (size_t)ASYNC_SMEM,
+                        st, a16);
+  }
   const int64_t body = h->tail_pitch ? h->body_bytes : rb;
   if (use_tma && rb % 16 == 0 && cw % 16 == 0 && body % 16 == 0 && oa % 16 == 0 && cw <= TMA_STAGE_BYTES) {
     const int R = (int)std::min<int64_t>(32, TMA_STAGE_BYTES / cw);

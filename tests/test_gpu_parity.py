@@ -264,8 +264,10 @@ def test_fork_concurrent_streams(tiny):
     dsm.destroy()
 
 
-def test_gather_tma_variant_subprocess():
-    """The TMA bulk-copy gather (WG_GATHER_TMA=1, chosen once per process) is bit-exact too."""
+@pytest.mark.parametrize("knob", ["WG_GATHER_TMA", "WG_GATHER_ASYNC"])
+def test_gather_tma_variant_subprocess(knob):
+    """The TMA bulk-copy gather (WG_GATHER_TMA=1) and the cp.async gather (WG_GATHER_ASYNC=1), chosen
+    once per process, are bit-exact too (whole / split rows, pitched outputs, partial ranges)."""
     import os
     import subprocess
     import sys
@@ -302,7 +304,7 @@ for dim, dtype in ((100, "fp32"), (4, "fp32"), (768, "fp16"), (1024, "fp32"), (3
 print("TMA OK")
 '''
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    r = subprocess.run([sys.executable, "-c", code], cwd=root, env=dict(os.environ, WG_GATHER_TMA="1"),
+    r = subprocess.run([sys.executable, "-c", code], cwd=root, env=dict(os.environ, **{knob: "1"}),
                        capture_output=True, text=True, timeout=600)
     assert r.returncode == 0 and "TMA OK" in r.stdout, r.stdout + r.stderr
 
