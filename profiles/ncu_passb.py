@@ -25,6 +25,10 @@ p = presets.get(os.environ.get("CONFIG", "products"))
 dsm, _ = loader.build_dsm(p)
 handles = [dsm] + [dsm.fork() for _ in range(P - 1)]
 GP, SP, MP = (int(os.environ.get(k, 0)) for k in ("PRIO_GATHER", "PRIO_SIDE", "PRIO_MAIN"))
+# gathers at the throughput occupancy bench pass B / MiniBatchLoader use (GATHER_OCC, 0 = occupancy max)
+OCC = int(os.environ.get("GATHER_OCC", pkg.pipeline.THROUGHPUT_GATHER_OCCUPANCY))
+for h in handles:
+    h.set_gather_occupancy(OCC)
 pipes = [pkg.MiniBatchPipeline(h, p.fanouts, p.seeds_per_batch, gather_priority=GP, side_priority=SP)
          for h in handles]
 S = p.seeds_per_batch
