@@ -90,3 +90,72 @@ def test_papers100m_shaped_batch_bit_exact():
         assert dsm.device_error() == 0
     finally:
         dsm.destroy()
+
+
+@pytest.mark.slow
+def test_mag240m_shaped_graph_w4_virtual_ranks_bit_exact():
+    """configs[4]'s graph at full size (244M nodes, ~3.4B CSR entries, fanout [25,15]) sharded
+    over W=4 in-process virtual ranks on the one GPU (the config needs W >= 4).  The 768 x fp16
+    table (375 GB) cannot fit one GPU, so the rows are narrowed to 16 x fp16 (32 B): the graph,
+    the 4-way sharding, the G=32 lane groups of fanout 25 and the gather addressing are the
+    config's; one batch per probed rank, every array compared with the oracle."""
+    import threading
+
+    from paper_conf_sc_yanglql22_b200.pipeline import required_keys
+    from synth import gpu as sgpu
+
+    p = presets.get("mag240m")
+    W, FD, FDT = 4, 16, "fp16"
+    free, _ = torch.cuda.mem_get_info()
+    if free < 150e9:
+        pytest.skip("needs a whole B200")
+    spec = p.graph()
+    shards = []
+    for r in range(W):  # one shard at a time (generator temporaries are large)
+        rp_r, col_r = sgpu.shard_csr_gpu(spec, r, W, torch.device("cuda", 0))
+        shards.append((rp_r, col_r))
+        torch.cuda.empty_cache()
+    assert abs(sum(int(c.numel()) for _, c in shards) - p.target_e) / p.target_e < 0.03
+    keys = required_keys(p.n, p.fanouts, p.seeds_per_batch)
+    ag = pkg.ThreadAllgather(W)
+    dsms, errs = [None] * W, []
+
+    def create(r):
+        try:
+            dsms[r] = pkg.DSM(p.n, int(shards[r][1].numel()), FD, FDT, keys, rank=r, world_size=W, device=0,
+                              allgather=ag.for_rank(r))
+        except Exception as e:  # pragma: no cover
+            errs.append(e)
+    ths = [threading.Thread(target=create, args=(r,)) for r in range(W)]
+    [t.start() for t in ths]
+    [t.join() for t in ths]
+    assert not errs, errs
+    try:
+        for r, d in enumerate(dsms):
+            lrp, lcol, _ = d.local_view()
+            lrp.copy_(shards[r][0])
+            lcol.copy_(shards[r][1])
+            sgpu.fill_dsm_features_gpu(d, presets.FEAT_SEED, r, W, FD, features.WG_DTYPE_CODE[FDT])
+        del shards
+        torch.cuda.synchronize()
+        rows = loader.host_row_provider(spec)
+        feats = loader.host_feat_provider(p, FD, FDT)
+        for r in (0, 3):
+            pipe = pkg.MiniBatchPipeline(dsms[r], p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
+            b = next(iter(seeds.rank_batches(W, r, W)))
+            S = seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, b)
+            rs = seeds.rng_seed(presets.RNG_BASE, b)
+            pipe.run(torch.from_numpy(S).cuda(), rs)
+            torch.cuda.synchronize()
+            ref = oracle.minibatch(rows, feats, S, p.fanouts, rs)
+            for h in range(len(p.fanouts)):
+                got, exp = pipe.result(h), ref["hops"][h]
+                for k in ("row_ptr", "nbrs", "pos", "unique", "sub_col", "dup"):
+                    assert np.array_equal(got[k], exp[k]), (r, h, k)
+            assert np.array_equal(pipe.features(), ref["X"]), r
+            assert dsms[r].device_error() == 0
+            del pipe
+    finally:
+        ths = [threading.Thread(target=d.destroy) for d in dsms if d is not None]
+        [t.start() for t in ths]
+        [t.join() for t in ths]
