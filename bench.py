@@ -175,6 +175,20 @@ def bench_reference(args):
     emit(line, args)
 
 
+# The paper's own numbers (DGX-A100 = 8 x A100 on NVSwitch, NVLink3 300 GB/s per direction):
+# context next to ours, never the target.
+PAPER_CONTEXT = {
+    "hardware": "DGX-A100 (8x A100 80GB, NVSwitch, NVLink3 300 GB/s/dir), CUDA 11.4",
+    "dsm_random_gather_busbw_gbs_ge128B": 230, "dsm_random_gather_busbw_frac_of_nvlink": 0.77,
+    "p2p_dependent_load_latency_us_8_128GB": [1.35, 1.56],
+    "epoch_speedup_vs_dgl_max": 57.32, "epoch_speedup_vs_pyg_max": 242.98,
+    "ogbn_products_graphsage_epoch_s": {"wholegraph": 0.99, "dgl": 30.8, "pyg": 228.96},
+    "seed_nodes_per_s": None,
+    "note": "PAPER.md L5, L66-80, L266, L272-275; end-to-end training epochs, not this metric (the paper "
+            "reports no seeds/s); context only",
+}
+
+
 def workload_config(p, W, flushed=True, placement="dsm"):
     par = (f"dsm-w{W} (row-sharded CSR+features, P2P loads, no hot-path collective)" if placement == "dsm" else
            f"replicas-x{W} (SURVEY 8(e) lever: whole graph + table on every GPU, no NVLink, no hot-path collective)")
@@ -500,6 +514,7 @@ def bench_wg(args):
                          "gather_share_of_single_batch": gather_s / (sum(step_ms) / 1e3),
                          "timed_in": "pass A (one batch at a time, events on the launching stream)"},
             "cpu_baseline": cpu,
+            "paper_context": PAPER_CONTEXT,
             "e2e": {"value": e2e_val, "unit": UNIT, "h2d_bytes_per_step": S * 8,
                     "d2h_bytes_per_step": e2e_d2h, "batches": len(todo),
                     "note": f"public API (MiniBatchLoader, {P} batches in flight): per batch pinned-host seeds "
