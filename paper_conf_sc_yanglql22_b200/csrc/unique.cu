@@ -280,7 +280,27 @@ static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, c
   a.excl = h->ws.excl[h->excl_next];
   h->excl_next = (h->excl_next + 1) % EXCL_RING;
   a.slot_of = h->ws.slot_of;
-  a.ht = HashTable{h->ws.hslots, (unsigned long long)h->ws.hcap - 1};
+  // Each call uses only a power-of-two prefix of the table sized for ITS key bound (capT + capE):
+  // a small hop then touches a few MB of lines instead of random lines all over the table sized
+  // for the largest hop.  Slots outside the prefix, or left by earlier calls, carry older epochs
+  // and read as empty.  WG_HASH_PER_CALL=0 uses the whole table for every call (A/B).
+  // The prefix has at least WG_HASH_MIN_SLOTS slots: a small hop's keys then stay sparse (short
+  // probe chains, single-batch latency) while touching no more lines than it has keys.
+  static int per_call = -1;
+  static int64_t min_slots = 0;
+  if (per_call < 0) {
+    const char* e = getenv("WG_HASH_PER_CALL");
+    per_call = (e && e[0] == '0') ? 0 : 1;
+    const char* m = getenv("WG_HASH_MIN_SLOTS");
+    min_slots = m ? atoll(m) : (int64_t(1) << 20);
+  }
+  int64_t hc = h->ws.hcap;
+  if (per_call) {
+    hc = 1024;
+    while (hc < h->ws.hcap && hc < min_slots) hc <<= 1;
+    while (hc < h->ws.hcap && (double)hc < h->ws.hfactor * (double)(a.capT + a.capE)) hc <<= 1;
+  }
+  a.ht = HashTable{h->ws.hslots, (unsigned long long)hc - 1};
   a.status = h->ws.status_unique;
   a.ctrl = h->ws.ctrl;
   a.n = h->n;
