@@ -113,18 +113,18 @@ static void free_workspace(wg_dsm* h) {
 static wg_status alloc_workspace(wg_dsm* h, int64_t max_keys) {
   Workspace& w = h->ws;
   if (max_keys < 1) max_keys = 1;
-  // Table size = WG_HASH_FACTOR (default 1.5) x the capacity bound.  Trade-off measured on B200:
+  // Table size = WG_HASH_FACTOR (default 2) x the capacity bound (a multiple of 8 slots).  Trade-off measured on B200:
   // a larger table shortens the warp-max linear-probe chains (single-batch latency), a smaller
   // one packs the touched slots into fewer DRAM lines, which matters when several batches (one
   // table each) are in flight and compete for the 126 MB L2.
   static double factor = 0.0;
   if (factor == 0.0) {
     const char* f = getenv("WG_HASH_FACTOR");
-    factor = f ? atof(f) : 1.5;
+    factor = f ? atof(f) : 2.0;
     if (factor < 1.25) factor = 1.25;
   }
-  int64_t cap = 1024;
-  while ((double)cap < factor * (double)max_keys) cap <<= 1;
+  int64_t cap = (int64_t)(factor * (double)max_keys) + 8;
+  cap = std::max<int64_t>(1024, (cap + 7) / 8 * 8);
   w.hcap = cap;
   w.hfactor = factor;
   w.max_keys = max_keys;

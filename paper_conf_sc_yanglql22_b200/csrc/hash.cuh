@@ -5,7 +5,8 @@
 // sector): key = (epoch << 40) | node id, val = ((EPOCH_MAX - epoch) << 40) | first
 // position.  A key from an older epoch reads as an empty slot and an older
 // value always loses an atomicMin against the current epoch, so the table is never
-// cleared between calls.  Linear probing, fmix64 hash, load factor <= 1/4.
+// cleared between calls.  Linear probing, fmix64 hash mapped onto [0, size) by a multiply-high,
+// load factor <= 1 / WG_HASH_FACTOR at the capacity bound.
 #pragma once
 
 #include "device_util.cuh"
@@ -17,7 +18,7 @@ constexpr unsigned long long KEY_MASK = (1ull << 40) - 1;
 
 struct HashTable {
   HashSlot* slots;
-  unsigned long long mask;  // capacity - 1
+  unsigned long long size;  // slots in use (any size: slot = high half of hash * size)
 };
 
 __device__ __forceinline__ unsigned long long stored_key(unsigned epoch, int64_t key) {
@@ -33,8 +34,8 @@ __device__ __forceinline__ unsigned long long pack_pos(unsigned epoch, int64_t q
 // key was already present, or ~0 when this call claimed the slot.
 __device__ __forceinline__ long long hash_insert(const HashTable& t, unsigned long long stored, unsigned epoch,
                                                  unsigned long long* seen) {
-  unsigned long long slot = fmix64(stored & KEY_MASK) & t.mask;
-  for (unsigned long long probe = 0; probe <= t.mask; ++probe) {
+  unsigned long long slot = __umul64hi(fmix64(stored & KEY_MASK), t.size);  // uniform in [0, size)
+  for (unsigned long long probe = 0; probe < t.size; ++probe) {
     unsigned long long cur, val;
     asm volatile("ld.volatile.global.v2.u64 {%0, %1}, [%2];" : "=l"(cur), "=l"(val) : "l"(&t.slots[slot]));
     for (;;) {
@@ -54,7 +55,7 @@ __device__ __forceinline__ long long hash_insert(const HashTable& t, unsigned lo
       }
       cur = prev;
     }
-    slot = (slot + 1) & t.mask;
+    slot = slot + 1 == t.size ? 0 : slot + 1;
   }
   return -1;
 }

@@ -49,7 +49,19 @@ struct SampleArgs {
   int32_t* pos_pad;   // [nT * M]
   int32_t* cnt;       // [nT]
   unsigned* ctrl;
+  int rp_keep;        // 1: row_ptr loads carry an L2 evict_last hint (WG_RP_EVICT_LAST)
 };
+
+// row_ptr is read by every target of every batch (2.45M x 8 B = 20 MB for products): an
+// evict_last hint asks L2 to keep it over the streaming gather bytes.
+__device__ __forceinline__ int64_t ld_rp(const int64_t* p, int keep) {
+  if (!keep) return *p;
+  unsigned long long pol;
+  asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
+  long long v;
+  asm volatile("ld.global.nc.L2::cache_hint.s64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
+  return v;
+}
 
 template <int SAMPLE_UNR>
 __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs a) {
@@ -87,8 +99,8 @@ __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs
         int64_t l;
         owner_local(a.s, my_v, o, l);
         const int64_t* rp = a.s.row_ptr[o] + l;
-        my_start = rp[0];
-        const int64_t d = rp[1] - my_start;
+        my_start = ld_rp(rp, a.rp_keep);
+        const int64_t d = ld_rp(rp + 1, a.rp_keep) - my_start;
         if (d >= (int64_t(1) << 32) || d < 0)
           latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DEGREE);
         else
@@ -359,6 +371,12 @@ cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap,
   a.pos_pad = want_pos ? h->ws.pos_pad : nullptr;
   a.cnt = h->ws.cnt;
   a.ctrl = h->ws.ctrl;
+  static int rp_keep = -1;
+  if (rp_keep < 0) {
+    const char* e = getenv("WG_RP_EVICT_LAST");
+    rp_keep = (e && e[0] == '1') ? 1 : 0;
+  }
+  a.rp_keep = rp_keep;
   if (fanout > 32) {  // block per target (Algorithm 1 with a block sort)
     const unsigned blocks = (unsigned)(cap > 0 ? cap : 1);
     if (fanout <= 64) return launch_pdl(sample_block_kernel<64>, blocks, 64, 0, st, a);

@@ -280,12 +280,11 @@ static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, c
   a.excl = h->ws.excl[h->excl_next];
   h->excl_next = (h->excl_next + 1) % EXCL_RING;
   a.slot_of = h->ws.slot_of;
-  // Each call uses only a power-of-two prefix of the table sized for ITS key bound (capT + capE):
-  // a small hop then touches a few MB of lines instead of random lines all over the table sized
-  // for the largest hop.  Slots outside the prefix, or left by earlier calls, carry older epochs
-  // and read as empty.  WG_HASH_PER_CALL=0 uses the whole table for every call (A/B).
-  // The prefix has at least WG_HASH_MIN_SLOTS slots: a small hop's keys then stay sparse (short
-  // probe chains, single-batch latency) while touching no more lines than it has keys.
+  // Each call uses only a prefix of the table sized for ITS key bound (capT + capE): factor x bound
+  // slots (any size, a multiple of 8 = one 128 B line; at least WG_HASH_MIN_SLOTS), so a hop touches
+  // about as many lines as it has keys instead of random lines all over the table sized for the
+  // largest hop.  Slots outside the prefix, or left by earlier calls, carry older epochs and read as
+  // empty.  WG_HASH_PER_CALL=0 uses the whole table for every call (A/B).
   static int per_call = -1;
   static int64_t min_slots = 0;
   if (per_call < 0) {
@@ -296,11 +295,11 @@ static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, c
   }
   int64_t hc = h->ws.hcap;
   if (per_call) {
-    hc = 1024;
-    while (hc < h->ws.hcap && hc < min_slots) hc <<= 1;
-    while (hc < h->ws.hcap && (double)hc < h->ws.hfactor * (double)(a.capT + a.capE)) hc <<= 1;
+    hc = (int64_t)(h->ws.hfactor * (double)(a.capT + a.capE)) + 8;
+    hc = std::max<int64_t>(hc, min_slots);
+    hc = std::min<int64_t>((hc + 7) / 8 * 8, h->ws.hcap);
   }
-  a.ht = HashTable{h->ws.hslots, (unsigned long long)hc - 1};
+  a.ht = HashTable{h->ws.hslots, (unsigned long long)hc};
   a.status = h->ws.status_unique;
   a.ctrl = h->ws.ctrl;
   a.n = h->n;

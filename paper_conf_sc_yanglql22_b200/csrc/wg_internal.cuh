@@ -58,8 +58,8 @@ struct __align__(16) HashSlot {
 };
 struct Workspace {
   HashSlot* hslots = nullptr;            // [hcap] append-unique hash table (hash.cuh)
-  int64_t hcap = 0;                      // power of two
-  double hfactor = 1.5;                  // slots per key bound (WG_HASH_FACTOR)
+  int64_t hcap = 0;                      // slots (a multiple of 8); each call uses a prefix
+  double hfactor = 2.0;                  // slots per key bound (WG_HASH_FACTOR)
   unsigned long long* status_sample = nullptr;  // decoupled look-back tile status
   unsigned long long* status_unique = nullptr;
   int64_t status_cap = 0;
