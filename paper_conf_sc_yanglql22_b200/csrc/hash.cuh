@@ -19,6 +19,7 @@ constexpr unsigned long long KEY_MASK = (1ull << 40) - 1;
 struct HashTable {
   HashSlot* slots;
   unsigned long long size;  // slots in use (any size: slot = high half of hash * size)
+  int cas128;               // claim with one 128-bit CAS of {key, value} (WG_HASH_CAS128)
 };
 
 __device__ __forceinline__ unsigned long long stored_key(unsigned epoch, int64_t key) {
@@ -29,11 +30,24 @@ __device__ __forceinline__ unsigned long long pack_pos(unsigned epoch, int64_t q
   return ((unsigned long long)(EPOCH_MAX - epoch) << 40) | (unsigned long long)q;
 }
 
+// 128-bit compare-and-swap (sm_90+): claims a slot by writing key AND value in one atomic.
+__device__ __forceinline__ void cas128(HashSlot* p, unsigned long long& k, unsigned long long& v,
+                                       unsigned long long nk, unsigned long long nv) {
+  asm volatile(
+      "{\n .reg .b128 c, n, d;\n mov.b128 c, {%0, %1};\n mov.b128 n, {%2, %3};\n"
+      " atom.global.cas.b128 d, [%4], c, n;\n mov.b128 {%0, %1}, d;\n}"
+      : "+l"(k), "+l"(v)
+      : "l"(nk), "l"(nv), "l"(p)
+      : "memory");
+}
+
 // Returns the slot holding `stored` (claiming an empty one if needed), or -1 if full.
 // *seen receives the slot's value as read together with its key (one 16 B load) when the
-// key was already present, or ~0 when this call claimed the slot.
+// key was already present, or ~0 when the value may still be stale (the caller then records
+// its position with an atomicMin).  With t.cas128 a claim writes the key together with the
+// value `mine` in one 128-bit CAS, and *seen = 0 tells the caller nothing is left to do.
 __device__ __forceinline__ long long hash_insert(const HashTable& t, unsigned long long stored, unsigned epoch,
-                                                 unsigned long long* seen) {
+                                                 unsigned long long mine, unsigned long long* seen) {
   unsigned long long slot = __umul64hi(fmix64(stored & KEY_MASK), t.size);  // uniform in [0, size)
   for (unsigned long long probe = 0; probe < t.size; ++probe) {
     unsigned long long cur, val;
@@ -44,6 +58,15 @@ __device__ __forceinline__ long long hash_insert(const HashTable& t, unsigned lo
         return (long long)slot;
       }
       if ((unsigned)(cur >> 40) == epoch) break;  // occupied by another key this epoch
+      if (t.cas128) {
+        const unsigned long long ck = cur, cv = val;
+        cas128(&t.slots[slot], cur, val, stored, mine);  // cur, val <- the slot's previous contents
+        if (cur == ck && val == cv) {
+          *seen = 0;  // claimed with our position already in place
+          return (long long)slot;
+        }
+        continue;  // re-examine what is there now (our key, another key, or a newer stale pair)
+      }
       const unsigned long long prev = atomicCAS(&t.slots[slot].key, cur, stored);
       if (prev == cur) {
         *seen = ~0ull;
@@ -65,8 +88,8 @@ __device__ __forceinline__ long long hash_insert(const HashTable& t, unsigned lo
 // most of the same-address atomics they would otherwise serialise on.
 __device__ __forceinline__ long long hash_insert_min(const HashTable& t, int64_t key, int64_t q, unsigned epoch) {
   unsigned long long seen;
-  const long long slot = hash_insert(t, stored_key(epoch, key), epoch, &seen);
   const unsigned long long mine = pack_pos(epoch, q);
+  const long long slot = hash_insert(t, stored_key(epoch, key), epoch, mine, &seen);
   if (slot >= 0 && seen > mine) atomicMin(&t.slots[slot].val, mine);
   return slot;
 }
@@ -78,10 +101,11 @@ __device__ __forceinline__ long long hash_insert_min(const HashTable& t, int64_t
 __device__ __forceinline__ long long hash_insert_target(const HashTable& t, int64_t key, int64_t q, int64_t nT,
                                                         unsigned epoch, bool* dup) {
   unsigned long long seen;
-  const long long slot = hash_insert(t, stored_key(epoch, key), epoch, &seen);
+  const unsigned long long mine = pack_pos(epoch, q);
+  const long long slot = hash_insert(t, stored_key(epoch, key), epoch, mine, &seen);
   *dup = false;
-  if (slot >= 0) {
-    const unsigned long long old = atomicMin(&t.slots[slot].val, pack_pos(epoch, q));
+  if (slot >= 0 && seen != 0) {  // seen == 0: claimed by our 128-bit CAS, no earlier record
+    const unsigned long long old = atomicMin(&t.slots[slot].val, mine);
     *dup = (old >> 40) == (unsigned long long)(EPOCH_MAX - epoch) && (int64_t)(old & KEY_MASK) < nT;
   }
   return slot;

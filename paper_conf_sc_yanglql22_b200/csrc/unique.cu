@@ -299,7 +299,12 @@ static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, c
     hc = std::max<int64_t>(hc, min_slots);
     hc = std::min<int64_t>((hc + 7) / 8 * 8, h->ws.hcap);
   }
-  a.ht = HashTable{h->ws.hslots, (unsigned long long)hc};
+  static int cas128 = -1;
+  if (cas128 < 0) {
+    const char* e = getenv("WG_HASH_CAS128");
+    cas128 = (e && e[0] == '0') ? 0 : 1;
+  }
+  a.ht = HashTable{h->ws.hslots, (unsigned long long)hc, cas128};
   a.status = h->ws.status_unique;
   a.ctrl = h->ws.ctrl;
   a.n = h->n;
