@@ -65,6 +65,7 @@ typedef enum { WG_F32 = 0, WG_F16 = 1, WG_BF16 = 2 } wg_dtype;
 #define WG_DEVERR_CAPACITY   0x4u  /* a device count exceeded its host capacity, or the hash table filled */
 #define WG_DEVERR_DEGREE     0x8u  /* a degree >= 2^32 (A3 requires N < 2^32) */
 #define WG_DEVERR_EPOCH      0x10u /* hash-table epoch space exhausted: call wg_dsm_reset_workspace */
+#define WG_DEVERR_TMA        0x20u /* a TMA gather stage never completed (the kernel stopped instead of hanging) */
 
 /* Allgather of host bytes across the W ranks of the DSM ("an
  * AllGather pattern communication is performed so that each process can get all

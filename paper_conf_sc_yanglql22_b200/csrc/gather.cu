@@ -404,9 +404,11 @@ __global__ void __launch_bounds__(32) gather_tma_kernel(const GatherArgs a, int 
 cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int64_t* d_n, const int64_t* d_begin,
                           void* out, int64_t out_pitch, cudaStream_t st) {
   const int64_t rb = h->row_bytes;
-  static int knobs = 0, bps = 0, use_tma = 0, allow32 = 1, use_async = 0;
+  static int knobs = 0, bps = 0, use_tma = 0, allow32 = 1, use_async = 0, use_g4 = 0;
   if (!knobs) {  // A/B knobs, read once: WG_GATHER_BPS (blocks per SM), WG_GATHER_TMA=1, WG_GATHER_V32=0,
                  // WG_GATHER_ASYNC=1 (cp.async variant)
+    const char* g4 = getenv("WG_GATHER_G4");
+    use_g4 = (g4 && g4[0] == '1') ? 1 : 0;
     const char* ca = getenv("WG_GATHER_ASYNC");
     use_async = (ca && ca[0] == '1') ? 1 : 0;
     const char* b = getenv("WG_GATHER_BPS");
@@ -426,6 +428,10 @@ cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int6
                  : (cw % 4 == 0 && oa % 4 == 0)             ? 4
                                                             : 2;
   GatherArgs a{h->view, ids, cap, d_n, d_begin, static_cast<uint8_t*>(out), h->ws.ctrl, FastDiv((unsigned)(cw / vb))};
+  if (use_g4) {
+    const cudaError_t e = launch_gather_g4(h, ids, cap, d_n, d_begin, out, cw, st);
+    if (e != cudaErrorNotSupported) return e;
+  }
   if (use_async && cw % 16 == 0 && oa % 16 == 0) {
     static int async_bps = 0;
     if (!async_bps) {

@@ -264,7 +264,7 @@ def test_fork_concurrent_streams(tiny):
     dsm.destroy()
 
 
-@pytest.mark.parametrize("knob", ["WG_GATHER_TMA", "WG_GATHER_ASYNC"])
+@pytest.mark.parametrize("knob", ["WG_GATHER_TMA", "WG_GATHER_ASYNC", "WG_GATHER_G4"])
 def test_gather_tma_variant_subprocess(knob):
     """The TMA bulk-copy gather (WG_GATHER_TMA=1) and the cp.async gather (WG_GATHER_ASYNC=1), chosen
     once per process, are bit-exact too (whole / split rows, pitched outputs, partial ranges)."""
