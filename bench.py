@@ -222,6 +222,39 @@ def workload_descriptors(dsm, pipe, seeds_dev, rngs, nb=20):
             "degree_log2_hist": hist, "top1pct_rows_share_of_gathered": top / max(tot, 1),
             "batches_for_share": min(nb, len(seeds_dev))}
 
+def stage_breakdown(pipe, seeds_dev, rngs, flush, nb=20):
+    """SURVEY 8(d) per-stage device times of one batch (outside every timed region): each hop's
+    fused op (sample + append-unique + relabel, all on one stream here) and the whole gather,
+    with a CUDA event after every op, eager launches, L2 flushed before each batch; medians."""
+    import torch
+    st = torch.cuda.current_stream()
+    H = len(pipe.fanouts)
+    names = [f"hop{h}" for h in range(H)] + ["gather"]
+    acc = {n: [] for n in names}
+    for b in range(nb + 2):
+        pipe.set_inputs(seeds_dev[b % len(seeds_dev)], rngs[b % len(rngs)])
+        if flush is not None:
+            flush.fill_(b & 0xFF)
+        evs = [torch.cuda.Event(enable_timing=True) for _ in range(H + 2)]
+        evs[0].record(st)
+        tgt, tcap, tn = pipe.seeds, pipe.max_seeds, pipe.n_seeds
+        for h, m in enumerate(pipe.fanouts):
+            bb = pipe.hops[h]
+            pipe.dsm.sample_hop(tgt, m, 0, h, n_targets_dev=tn, seed_dev=pipe.rng_seed, out=bb, cap=tcap, stream=st)
+            evs[h + 1].record(st)
+            tgt, tcap, tn = bb["unique"], pipe.U_cap[h], bb["num_unique"]
+        pipe.enqueue_gather(st)
+        evs[H + 1].record(st)
+        torch.cuda.synchronize()
+        if b >= 2:
+            for i, n in enumerate(names):
+                acc[n].append(evs[i].elapsed_time(evs[i + 1]))
+    out = {n: statistics.median(v) for n, v in acc.items()}
+    out["note"] = ("median ms per stage of one batch (eager launches, event after every op, L2 flushed per "
+                   "batch; hop h = wg_sample_hop: sample + insert + flag-scan + relabel)")
+    return out
+
+
 def emit(line, args):
     s = json.dumps(line)
     print(s, flush=True)
@@ -481,6 +514,7 @@ def bench_wg(args):
     loader_.close()
 
     wdesc = workload_descriptors(dsm, pipes[0], seeds_dev, rngs) if rank == 0 else {}
+    stages = stage_breakdown(pipes[0], seeds_dev, rngs, flush) if rank == 0 else {}
     line = None
     if rank == 0:
         cpu = None
@@ -514,6 +548,7 @@ def bench_wg(args):
                          "gather_share_of_single_batch": gather_s / (sum(step_ms) / 1e3),
                          "timed_in": "pass A (one batch at a time, events on the launching stream)"},
             "cpu_baseline": cpu,
+            "stages_ms": stages,
             "paper_context": PAPER_CONTEXT,
             "e2e": {"value": e2e_val, "unit": UNIT, "h2d_bytes_per_step": S * 8,
                     "d2h_bytes_per_step": e2e_d2h, "batches": len(todo),
