@@ -159,3 +159,29 @@ def test_mag240m_shaped_graph_w4_virtual_ranks_bit_exact():
         ths = [threading.Thread(target=d.destroy) for d in dsms if d is not None]
         [t.start() for t in ths]
         [t.join() for t in ths]
+
+
+def test_products_throughput_configuration_bit_exact(products):
+    """The launch configuration of bench.py's throughput pass and e2e (8 batches in flight on DSM
+    workspace forks and 8 streams, graph replay, gathers at the throughput occupancy, pinned-host
+    seeds) at full products size: 16 batches, every array of every batch compared with the oracle."""
+    p, dsm, _ = products
+    depth, nb = 8, 16
+    ld = pkg.MiniBatchLoader(dsm, p.fanouts, p.seeds_per_batch, depth=depth, with_pos=True, with_dup=True)
+    assert all(pl.gather_occupancy == pkg.pipeline.THROUGHPUT_GATHER_OCCUPANCY for pl in ld.pipes)
+    S = [seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 500 + b) for b in range(nb)]
+    rs = [seeds.rng_seed(presets.RNG_BASE, 500 + b) for b in range(nb)]
+    batches = [(torch.from_numpy(s).pin_memory(), r) for s, r in zip(S, rs)]
+    rows = loader.host_row_provider(p.graph())
+    feats = loader.host_feat_provider(p)
+    seen = 0
+    for pb in ld(batches):
+        ref = oracle.minibatch(rows, feats, S[seen], p.fanouts, rs[seen])
+        for h in range(len(p.fanouts)):
+            got, exp = pb.hop(h), ref["hops"][h]
+            for k in ("row_ptr", "nbrs", "pos", "unique", "sub_col", "dup"):
+                assert np.array_equal(got[k].cpu().numpy(), exp[k]), (seen, h, k)
+        assert np.array_equal(pb.X.cpu().numpy(), ref["X"]), seen
+        seen += 1
+    assert seen == nb and ld.device_error() == 0
+    ld.close()
