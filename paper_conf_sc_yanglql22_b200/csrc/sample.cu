@@ -387,7 +387,13 @@ cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap,
   }
   const int G = sample_group(fanout);
   const int tpw = 32 / G;
-  int unr = 4;  // largest of 4/2/1 that still gives >= 2 blocks per SM
+  static int unr_max = -1;  // A/B knob WG_SAMPLE_UNR_MAX (4, 2 or 1)
+  if (unr_max < 0) {
+    const char* e = getenv("WG_SAMPLE_UNR_MAX");
+    unr_max = e ? std::max(1, std::min(4, atoi(e))) : 4;
+    if (unr_max == 3) unr_max = 2;
+  }
+  int unr = unr_max;  // largest of 4/2/1 that still gives >= 2 blocks per SM
   while (unr > 1 && cap < (int64_t)(SAMPLE_THREADS / 32) * tpw * unr * 2 * h->sm_count) unr >>= 1;
   const int64_t tile = (int64_t)(SAMPLE_THREADS / 32) * tpw * unr;
   const unsigned blocks = (unsigned)(cap > 0 ? (cap + tile - 1) / tile : 1);

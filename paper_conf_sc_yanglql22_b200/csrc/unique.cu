@@ -318,7 +318,13 @@ static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, c
   int64_t ib = (total + UQ_THREADS - 1) / UQ_THREADS;
   ib = ib < 1 ? 1 : (ib > max_blocks ? max_blocks : ib);
   // items per thread: the largest of 8/4/2/1 that still gives >= 2 tiles per SM
-  int items = 8;
+  static int items_max = -1;  // A/B knob WG_FLAG_ITEMS_MAX (8, 4, 2 or 1)
+  if (items_max < 0) {
+    const char* e = getenv("WG_FLAG_ITEMS_MAX");
+    const int v = e ? atoi(e) : 8;
+    items_max = v >= 8 ? 8 : v >= 4 ? 4 : v >= 2 ? 2 : 1;
+  }
+  int items = items_max;
   while (items > 1 && a.capE < (int64_t)items * UQ_THREADS * 2 * h->sm_count) items >>= 1;
   const int64_t tile = (int64_t)items * UQ_THREADS;
   const unsigned fb = (unsigned)(a.capE > 0 ? (a.capE + tile - 1) / tile : 1);
