@@ -236,8 +236,8 @@ cudaError_t launch_gather_g4(wg_dsm* h, const int64_t* ids, int64_t cap, const i
   if (cw % 32 != 0 || ((uintptr_t)out & 31) || body % 16 || tail % 16 || body > 1024 || body < 16 ||
       h->feat_stride % 16 || (tail && h->tail_pitch != tail))
     return cudaErrorNotSupported;
-  static G4Maps maps;  // per process, rebuilt when the handle's shards change
-  static const void* built_for = nullptr;
+  thread_local G4Maps maps;  // per host thread (virtual ranks), rebuilt when the shards change
+  thread_local const void* built_for = nullptr;
   if (built_for != h->view.feat[0]) {
     for (int r = 0; r < h->world; ++r) {
       if (!encode_rows(&maps.body[r], h->view.feat[r], std::max<int64_t>(1, h->n_local_of[r]), (int)body,
