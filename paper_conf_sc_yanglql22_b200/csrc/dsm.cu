@@ -141,8 +141,19 @@ static wg_status alloc_workspace(wg_dsm* h, int64_t max_keys) {
     free_workspace(h);
     return fail(WG_ERR_OOM, "workspace allocation failed");
   }
-  WG_CUDA_TRY(cudaMemset(w.hslots, 0xff, cap * sizeof(HashSlot)));                   // val = all ones
-  WG_CUDA_TRY(cudaMemset2D(w.hslots, sizeof(HashSlot), 0, sizeof(unsigned long long), cap));  // key = 0 (empty)
+  // compact 8 B slots (hash.cuh) when node ids and positions fit 28 bits (WG_HASH_COMPACT=0: 16 B slots)
+  static int compact_ok = -1;
+  if (compact_ok < 0) {
+    const char* c = getenv("WG_HASH_COMPACT");
+    compact_ok = (c && c[0] == '0') ? 0 : 1;
+  }
+  w.compact = compact_ok && h->n <= (int64_t(1) << 28) && max_keys < (int64_t(1) << 28) ? 1 : 0;
+  if (w.compact) {
+    WG_CUDA_TRY(cudaMemset(w.hslots, 0, cap * sizeof(HashSlot)));  // every word stale (epoch 0)
+  } else {
+    WG_CUDA_TRY(cudaMemset(w.hslots, 0xff, cap * sizeof(HashSlot)));                   // val = all ones
+    WG_CUDA_TRY(cudaMemset2D(w.hslots, sizeof(HashSlot), 0, sizeof(unsigned long long), cap));  // key = 0 (empty)
+  }
   WG_CUDA_TRY(cudaMemset(w.status_sample, 0, w.status_cap * 8));
   WG_CUDA_TRY(cudaMemset(w.status_unique, 0, w.status_cap * 8));
   unsigned ctrl[CTRL_WORDS] = {0};
@@ -540,8 +551,12 @@ wg_status wg_dsm_reset_workspace(wg_dsm_t h, wg_stream_t stream) {
   if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
   cudaSetDevice(h->device);
   cudaStream_t st = (cudaStream_t)stream;
-  WG_CUDA_TRY(cudaMemsetAsync(h->ws.hslots, 0xff, h->ws.hcap * sizeof(HashSlot), st));
-  WG_CUDA_TRY(cudaMemset2DAsync(h->ws.hslots, sizeof(HashSlot), 0, sizeof(unsigned long long), h->ws.hcap, st));
+  if (h->ws.compact) {
+    WG_CUDA_TRY(cudaMemsetAsync(h->ws.hslots, 0, h->ws.hcap * sizeof(HashSlot), st));
+  } else {
+    WG_CUDA_TRY(cudaMemsetAsync(h->ws.hslots, 0xff, h->ws.hcap * sizeof(HashSlot), st));
+    WG_CUDA_TRY(cudaMemset2DAsync(h->ws.hslots, sizeof(HashSlot), 0, sizeof(unsigned long long), h->ws.hcap, st));
+  }
   static const unsigned one = 1;
   WG_CUDA_TRY(cudaMemcpyAsync(h->ws.ctrl + CTRL_EPOCH, &one, 4, cudaMemcpyHostToDevice, st));
   return WG_OK;

@@ -20,7 +20,54 @@ struct HashTable {
   HashSlot* slots;
   unsigned long long size;  // slots in use (any size: slot = high half of hash * size)
   int cas128;               // claim with one 128-bit CAS of {key, value} (WG_HASH_CAS128)
+  int compact;              // 8 B slots (below) instead of 16 B HashSlots
 };
+
+// ---- compact table: one 64-bit word per slot, [63:56] epoch (1..255), [55:28] node id, [27:0]
+// first position (nodes and positions < 2^28).  Claimed with one 64-bit CAS of the whole word;
+// later occurrences of the key lower it with a 64-bit atomicMin (epoch and id bits are equal,
+// so the minimum is taken over the position).  Stale words (another epoch, or 0 after a clear)
+// read as empty; the table is cleared when the 255-epoch cycle restarts (sample_kernel /
+// hash_clear_kernel), so it never needs a per-call memset.
+constexpr unsigned long long CPOS_MASK = (1ull << 28) - 1;
+__device__ __forceinline__ unsigned long long cword(unsigned ce, int64_t key, int64_t q) {
+  return ((unsigned long long)ce << 56) | ((unsigned long long)key << 28) | (unsigned long long)q;
+}
+// Returns the slot of `key` (claimed with position q if new), or -1 if full; *old = the word seen
+// (0 if this call claimed the slot).  Applies the atomicMin (with return if want_old).
+__device__ __forceinline__ long long chash_insert(const HashTable& t, int64_t key, int64_t q, unsigned ce,
+                                                  bool want_old, unsigned long long* old) {
+  unsigned long long* w = reinterpret_cast<unsigned long long*>(t.slots);
+  const unsigned long long mine = cword(ce, key, q);
+  unsigned long long slot = __umul64hi(fmix64((unsigned long long)key), t.size);
+  for (unsigned long long probe = 0; probe < t.size; ++probe) {
+    unsigned long long cur;
+    asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(cur) : "l"(&w[slot]));
+    for (;;) {
+      if ((cur >> 28) == (mine >> 28)) {  // our key, this epoch
+        if (want_old) {
+          *old = atomicMin(&w[slot], mine);
+        } else {
+          if ((cur & CPOS_MASK) > (unsigned long long)q) atomicMin(&w[slot], mine);
+          *old = cur;
+        }
+        return (long long)slot;
+      }
+      if ((unsigned)(cur >> 56) == ce) break;  // another key this epoch
+      const unsigned long long prev = atomicCAS(&w[slot], cur, mine);
+      if (prev == cur) {
+        *old = 0;
+        return (long long)slot;
+      }
+      cur = prev;
+    }
+    slot = slot + 1 == t.size ? 0 : slot + 1;
+  }
+  return -1;
+}
+__device__ __forceinline__ int64_t chash_min_pos(const HashTable& t, long long slot) {
+  return (int64_t)(reinterpret_cast<const unsigned long long*>(t.slots)[slot] & CPOS_MASK);
+}
 
 __device__ __forceinline__ unsigned long long stored_key(unsigned epoch, int64_t key) {
   return ((unsigned long long)epoch << 40) | (unsigned long long)key;

@@ -50,7 +50,17 @@ struct SampleArgs {
   int32_t* cnt;       // [nT]
   unsigned* ctrl;
   int rp_keep;        // 1: row_ptr loads carry an L2 evict_last hint (WG_RP_EVICT_LAST)
+  unsigned long long* hclear;  // fused hop, compact hash table: zeroed here when its epoch cycle restarts
+  int64_t hwords;
 };
+
+// The insert pass that follows this sampler (same hop) needs a zeroed compact table when the epoch
+// cycle restarts (hash.cuh); every block clears a grid-strided share before sampling.
+__device__ __noinline__ void clear_table_if_cycle_restarts(unsigned long long* w, int64_t words, const unsigned* ctrl) {
+  if (compact_epoch(ctrl[CTRL_EPOCH]) != 1u) return;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < words; i += stride) w[i] = 0ull;
+}
 
 // row_ptr is read by every target of every batch (2.45M x 8 B = 20 MB for products): an
 // evict_last hint asks L2 to keep it over the streaming gather bytes.
@@ -63,9 +73,10 @@ __device__ __forceinline__ int64_t ld_rp(const int64_t* p, int keep) {
   return v;
 }
 
-template <int SAMPLE_UNR>
+template <int SAMPLE_UNR, bool CLR>
 __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs a) {
   pdl_enter();
+  if (CLR) clear_table_if_cycle_restarts(a.hclear, a.hwords, a.ctrl);
   __shared__ unsigned sm_chain[SAMPLE_THREADS / 32][32];
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   int64_t nT = a.cap;
@@ -176,9 +187,10 @@ __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs
 // (L118): Algorithm 1 exactly as listed (L122-158), with parallel_sort = a block bitonic
 // sort of the packed 64-bit keys (r << 32 | i) (L118-120) in shared memory, chain / q /
 // last in shared memory and path doubling as ceil(log2 M) synchronous rounds.
-template <int BT>
+template <int BT, bool CLR>
 __global__ void __launch_bounds__(BT) sample_block_kernel(const SampleArgs a) {
   pdl_enter();
+  if (CLR) clear_table_if_cycle_restarts(a.hclear, a.hwords, a.ctrl);
   __shared__ unsigned long long s_key[BT];
   __shared__ unsigned s_r[BT], s_chain[BT], s_q[BT], s_last[BT];
   __shared__ int64_t s_v, s_start;
@@ -356,6 +368,15 @@ __global__ void __launch_bounds__(COMPACT_THREADS) sample_compact_kernel(const C
   }
 }
 
+template <bool CLR>
+static cudaError_t launch_block_sampler(int fanout, unsigned blocks, const SampleArgs& a, cudaStream_t st) {
+  if (fanout <= 64) return launch_pdl(sample_block_kernel<64, CLR>, blocks, 64, 0, st, a);
+  if (fanout <= 128) return launch_pdl(sample_block_kernel<128, CLR>, blocks, 128, 0, st, a);
+  if (fanout <= 256) return launch_pdl(sample_block_kernel<256, CLR>, blocks, 256, 0, st, a);
+  if (fanout <= 512) return launch_pdl(sample_block_kernel<512, CLR>, blocks, 512, 0, st, a);
+  return launch_pdl(sample_block_kernel<1024, CLR>, blocks, 1024, 0, st, a);
+}
+
 cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap, const int64_t* d_n, int fanout,
                                  uint64_t seed, const uint64_t* d_seed, int hop, bool want_pos, cudaStream_t st) {
   SampleArgs a;
@@ -371,6 +392,8 @@ cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap,
   a.pos_pad = want_pos ? h->ws.pos_pad : nullptr;
   a.cnt = h->ws.cnt;
   a.ctrl = h->ws.ctrl;
+  a.hclear = h->ws.compact ? reinterpret_cast<unsigned long long*>(h->ws.hslots) : nullptr;
+  a.hwords = h->ws.hcap;
   static int rp_keep = -1;
   if (rp_keep < 0) {
     const char* e = getenv("WG_RP_EVICT_LAST");
@@ -379,11 +402,8 @@ cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap,
   a.rp_keep = rp_keep;
   if (fanout > 32) {  // block per target (Algorithm 1 with a block sort)
     const unsigned blocks = (unsigned)(cap > 0 ? cap : 1);
-    if (fanout <= 64) return launch_pdl(sample_block_kernel<64>, blocks, 64, 0, st, a);
-    if (fanout <= 128) return launch_pdl(sample_block_kernel<128>, blocks, 128, 0, st, a);
-    if (fanout <= 256) return launch_pdl(sample_block_kernel<256>, blocks, 256, 0, st, a);
-    if (fanout <= 512) return launch_pdl(sample_block_kernel<512>, blocks, 512, 0, st, a);
-    return launch_pdl(sample_block_kernel<1024>, blocks, 1024, 0, st, a);
+    if (a.hclear) return launch_block_sampler<true>(fanout, blocks, a, st);
+    return launch_block_sampler<false>(fanout, blocks, a, st);
   }
   const int G = sample_group(fanout);
   const int tpw = 32 / G;
@@ -397,9 +417,14 @@ cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap,
   while (unr > 1 && cap < (int64_t)(SAMPLE_THREADS / 32) * tpw * unr * 2 * h->sm_count) unr >>= 1;
   const int64_t tile = (int64_t)(SAMPLE_THREADS / 32) * tpw * unr;
   const unsigned blocks = (unsigned)(cap > 0 ? (cap + tile - 1) / tile : 1);
-  if (unr == 4) return launch_pdl(sample_kernel<4>, blocks, SAMPLE_THREADS, 0, st, a);
-  if (unr == 2) return launch_pdl(sample_kernel<2>, blocks, SAMPLE_THREADS, 0, st, a);
-  return launch_pdl(sample_kernel<1>, blocks, SAMPLE_THREADS, 0, st, a);
+  if (a.hclear) {
+    if (unr == 4) return launch_pdl(sample_kernel<4, true>, blocks, SAMPLE_THREADS, 0, st, a);
+    if (unr == 2) return launch_pdl(sample_kernel<2, true>, blocks, SAMPLE_THREADS, 0, st, a);
+    return launch_pdl(sample_kernel<1, true>, blocks, SAMPLE_THREADS, 0, st, a);
+  }
+  if (unr == 4) return launch_pdl(sample_kernel<4, false>, blocks, SAMPLE_THREADS, 0, st, a);
+  if (unr == 2) return launch_pdl(sample_kernel<2, false>, blocks, SAMPLE_THREADS, 0, st, a);
+  return launch_pdl(sample_kernel<1, false>, blocks, SAMPLE_THREADS, 0, st, a);
 }
 
 cudaError_t launch_sample(wg_dsm* h, const int64_t* targets, int64_t cap, const int64_t* d_n, int fanout,

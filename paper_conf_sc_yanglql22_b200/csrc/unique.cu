@@ -84,7 +84,7 @@ __device__ __forceinline__ void load_counts(const UniqueArgs& a, int64_t& nT, in
   nE = PADDED ? nT * a.M : clamp_count(a.d_nE, a.capE, a.ctrl);
 }
 
-template <bool PADDED>
+template <bool PADDED, bool COMPACT>
 __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueArgs a) {
   pdl_enter();
   int64_t nT, nE;
@@ -130,7 +130,13 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueA
       latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DUP_TARGET);
     long long slot = -1;
     if (valid && leader == lane) {
-      if (is_target) {
+      if (COMPACT) {
+        unsigned long long old;
+        slot = chash_insert(a.ht, key, q, compact_epoch(epoch), is_target, &old);
+        // a target meeting an earlier TARGET record of its key: duplicate target (A8)
+        if (is_target && slot >= 0 && old != 0 && (int64_t)(old & CPOS_MASK) < nT)
+          latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DUP_TARGET);
+      } else if (is_target) {
         bool dup = false;
         slot = hash_insert_target(a.ht, key, q, nT, epoch, &dup);
         if (dup) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DUP_TARGET);
@@ -144,12 +150,14 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueA
   }
 }
 
+template <bool COMPACT>
 __device__ __forceinline__ int64_t min_pos_at(const UniqueArgs& a, int32_t slot) {
   if (slot < 0) return -1;
+  if (COMPACT) return chash_min_pos(a.ht, slot);
   return (int64_t)(a.ht.slots[slot].val & KEY_MASK);
 }
 
-template <bool PADDED, int UQ_ITEMS>
+template <bool PADDED, int UQ_ITEMS, bool COMPACT>
 __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArgs a) {
   pdl_enter();
   // warp-striped: warp w of the tile covers 32 * UQ_ITEMS consecutive positions, lane l the
@@ -195,7 +203,7 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArg
       const int64_t j = wbase + 32 * t;
       const bool valid = j < nE && (!PADDED || slots[t] != SLOT_EMPTY);
       poss[t] = (PADDED && a.out_pos && valid) ? a.pos_pad[j] : 0;
-      mps[t] = min_pos_at(a, slots[t]);  // independent L2 reads
+      mps[t] = min_pos_at<COMPACT>(a, slots[t]);  // independent L2 reads
       vm[t] = __ballot_sync(FULL_MASK, valid);
     }
 #pragma unroll
@@ -252,8 +260,11 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArg
     for (int t = tid; t < (int)gridDim.x; t += UQ_THREADS) a.status[t] = 0ull;
     if (tid == 0) {
       a.ctrl[CTRL_DONE_UNIQUE] = 0u;
-      // the table is not read again in this call: advance its epoch
-      if (epoch + 1u >= EPOCH_MAX)
+      // the table is not read again in this call: advance its epoch (the compact table cycles
+      // through 255 epochs and is cleared when a cycle restarts; the wide one has 2^23)
+      if (COMPACT)
+        a.ctrl[CTRL_EPOCH] = epoch + 1u >= CEPOCHS * 4096u ? (epoch + 1u) % CEPOCHS + CEPOCHS : epoch + 1u;
+      else if (epoch + 1u >= EPOCH_MAX)
         latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_EPOCH);
       else
         a.ctrl[CTRL_EPOCH] = epoch + 1u;
@@ -273,6 +284,38 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_relabel_kernel(const Unique
     if (mp >= 0) id = mp < nT ? mp : (int32_t)nT + a.excl[mp - nT];
     a.sub_col[p] = id;
     if (a.dup && id >= 0) atomicAdd(&a.dup[id], 1);
+  }
+}
+
+// Compact table: zero it when the epoch cycle restarts (compact_epoch == 1).  Launched before the
+// insert pass of a standalone append-unique; the fused hop does the same inside its sampler.
+__global__ void __launch_bounds__(256) hash_clear_kernel(unsigned long long* w, int64_t words, const unsigned* ctrl) {
+  pdl_enter();
+  if (compact_epoch(ctrl[CTRL_EPOCH]) != 1u) return;
+  for (int64_t i = (int64_t)blockIdx.x * 256 + threadIdx.x; i < words; i += (int64_t)gridDim.x * 256) w[i] = 0ull;
+}
+
+template <bool C>
+static cudaError_t launch_insert_flag(bool padded, int items, int64_t ib, unsigned fb, const UniqueArgs& a,
+                                      cudaStream_t st) {
+  cudaError_t e;
+  if (padded) {
+    e = launch_pdl(unique_insert_kernel<true, C>, (unsigned)ib, UQ_THREADS, 0, st, a);
+    if (e != cudaSuccess) return e;
+    switch (items) {
+      case 8: return launch_pdl(unique_flag_kernel<true, 8, C>, fb, UQ_THREADS, 0, st, a);
+      case 4: return launch_pdl(unique_flag_kernel<true, 4, C>, fb, UQ_THREADS, 0, st, a);
+      case 2: return launch_pdl(unique_flag_kernel<true, 2, C>, fb, UQ_THREADS, 0, st, a);
+      default: return launch_pdl(unique_flag_kernel<true, 1, C>, fb, UQ_THREADS, 0, st, a);
+    }
+  }
+  e = launch_pdl(unique_insert_kernel<false, C>, (unsigned)ib, UQ_THREADS, 0, st, a);
+  if (e != cudaSuccess) return e;
+  switch (items) {
+    case 8: return launch_pdl(unique_flag_kernel<false, 8, C>, fb, UQ_THREADS, 0, st, a);
+    case 4: return launch_pdl(unique_flag_kernel<false, 4, C>, fb, UQ_THREADS, 0, st, a);
+    case 2: return launch_pdl(unique_flag_kernel<false, 2, C>, fb, UQ_THREADS, 0, st, a);
+    default: return launch_pdl(unique_flag_kernel<false, 1, C>, fb, UQ_THREADS, 0, st, a);
   }
 }
 
@@ -304,7 +347,7 @@ static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, c
     const char* e = getenv("WG_HASH_CAS128");
     cas128 = (e && e[0] == '0') ? 0 : 1;
   }
-  a.ht = HashTable{h->ws.hslots, (unsigned long long)hc, cas128};
+  a.ht = HashTable{h->ws.hslots, (unsigned long long)hc, cas128, h->ws.compact};
   a.status = h->ws.status_unique;
   a.ctrl = h->ws.ctrl;
   a.n = h->n;
@@ -329,25 +372,15 @@ static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, c
   const int64_t tile = (int64_t)items * UQ_THREADS;
   const unsigned fb = (unsigned)(a.capE > 0 ? (a.capE + tile - 1) / tile : 1);
   cudaError_t e;
-  if (padded) {
-    e = launch_pdl(unique_insert_kernel<true>, (unsigned)ib, UQ_THREADS, 0, st, a);
+  if (!padded && h->ws.compact) {
+    e = launch_pdl(hash_clear_kernel, (unsigned)h->sm_count * 4, 256, 0, st,
+                   reinterpret_cast<unsigned long long*>(h->ws.hslots), (int64_t)h->ws.hcap, (const unsigned*)h->ws.ctrl);
     if (e != cudaSuccess) return e;
-    switch (items) {
-      case 8: e = launch_pdl(unique_flag_kernel<true, 8>, fb, UQ_THREADS, 0, st, a); break;
-      case 4: e = launch_pdl(unique_flag_kernel<true, 4>, fb, UQ_THREADS, 0, st, a); break;
-      case 2: e = launch_pdl(unique_flag_kernel<true, 2>, fb, UQ_THREADS, 0, st, a); break;
-      default: e = launch_pdl(unique_flag_kernel<true, 1>, fb, UQ_THREADS, 0, st, a); break;
-    }
-  } else {
-    e = launch_pdl(unique_insert_kernel<false>, (unsigned)ib, UQ_THREADS, 0, st, a);
-    if (e != cudaSuccess) return e;
-    switch (items) {
-      case 8: e = launch_pdl(unique_flag_kernel<false, 8>, fb, UQ_THREADS, 0, st, a); break;
-      case 4: e = launch_pdl(unique_flag_kernel<false, 4>, fb, UQ_THREADS, 0, st, a); break;
-      case 2: e = launch_pdl(unique_flag_kernel<false, 2>, fb, UQ_THREADS, 0, st, a); break;
-      default: e = launch_pdl(unique_flag_kernel<false, 1>, fb, UQ_THREADS, 0, st, a); break;
-    }
   }
+  if (h->ws.compact)
+    e = launch_insert_flag<true>(padded, items, ib, fb, a, st);
+  else
+    e = launch_insert_flag<false>(padded, items, ib, fb, a, st);
   if (e != cudaSuccess) return e;
   if (a.capE > 0) {
     // relabel runs over the DENSE neighbours: count = num_edges (padded) or d_nE

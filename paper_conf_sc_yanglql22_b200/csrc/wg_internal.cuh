@@ -60,6 +60,7 @@ struct Workspace {
   HashSlot* hslots = nullptr;            // [hcap] append-unique hash table (hash.cuh)
   int64_t hcap = 0;                      // slots (a multiple of 8); each call uses a prefix
   double hfactor = 2.0;                  // slots per key bound (WG_HASH_FACTOR)
+  int compact = 0;                       // 8 B slots {epoch8, key28, pos28} (hash.cuh), else 16 B slots
   unsigned long long* status_sample = nullptr;  // decoupled look-back tile status
   unsigned long long* status_unique = nullptr;
   int64_t status_cap = 0;
@@ -75,6 +76,9 @@ struct Workspace {
 };
 enum { CTRL_ERR = 0, CTRL_EPOCH = 1, CTRL_DONE_SAMPLE = 2, CTRL_DONE_UNIQUE = 3, CTRL_WORDS = 16 };
 constexpr unsigned EPOCH_MAX = (1u << 23) - 1;
+// compact hash table (8 B slots): epochs 1..255 cycle; the table is cleared when a cycle restarts
+constexpr unsigned CEPOCHS = 255;
+__host__ __device__ inline unsigned compact_epoch(unsigned e) { return e % CEPOCHS + 1u; }
 constexpr int EXCL_RING = 4;
 
 }  // namespace wg

@@ -466,9 +466,64 @@ print("EPOCH OK")
 '''
     root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
     r = subprocess.run([sys.executable, "-c", code], cwd=root,
-                       env=dict(os.environ, WG_EPOCH_START=str((1 << 23) - 3)), capture_output=True, text=True,
-                       timeout=600)
+                       env=dict(os.environ, WG_EPOCH_START=str((1 << 23) - 3), WG_HASH_COMPACT="0"),
+                       capture_output=True, text=True, timeout=600)
     assert r.returncode == 0 and "EPOCH OK" in r.stdout, r.stdout + r.stderr
+
+
+def test_compact_table_epoch_cycles(tiny):
+    """The compact 8 B hash table cycles through 255 epochs and is cleared when a cycle restarts
+    (by the fused hop's sampler, or before a standalone insert): 140 tiny batches (280 fused hops,
+    more than a whole cycle, starting just before a restart) and standalone append-unique calls
+    across a restart, all bit-exact against the oracle."""
+    import os
+    import subprocess
+    import sys
+    code = r'''
+import sys, numpy as np, torch
+sys.path.insert(0, "tests")
+import oracle
+import paper_conf_sc_yanglql22_b200 as pkg
+from paper_conf_sc_yanglql22_b200 import loader
+from gpu_helpers import make_dsm, gpu_unique
+from synth import graph, presets, seeds
+p = presets.get("tiny")
+rp, col = graph.csr(p.graph())
+rows = loader.host_row_provider(p.graph(), rp, col)
+feats = loader.host_feat_provider(p)
+dsm, _ = loader.build_dsm(p, on_device=False)
+pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
+pipe.run(torch.from_numpy(seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 0)).cuda(), 5)
+pipe.capture()
+for b in range(140):
+    S = seeds.seed_nodes(p.n, p.seeds_per_batch - (b % 5) * 11, presets.SEED_BASE, 1000 + b)
+    rs = seeds.rng_seed(presets.RNG_BASE, 1000 + b)
+    pipe.run(torch.from_numpy(S).cuda(), rs)
+    torch.cuda.synchronize()
+    ref = oracle.minibatch(rows, feats, S, p.fanouts, rs)
+    for h in range(len(p.fanouts)):
+        got, exp = pipe.result(h), ref["hops"][h]
+        for k in ("row_ptr", "nbrs", "pos", "unique", "sub_col", "dup"):
+            assert np.array_equal(got[k], exp[k]), (b, h, k)
+    assert np.array_equal(pipe.features(), ref["X"]), b
+assert dsm.device_error() == 0
+dsm.destroy()
+rng = np.random.default_rng(3)
+d2 = make_dsm(np.zeros(2001, np.int64), np.zeros(0, np.int64), max_keys=4096)
+for i in range(300):
+    T = rng.choice(2000, 40, replace=False).astype(np.int64)
+    nb = rng.integers(0, 2000, 600).astype(np.int64)
+    U, sc, dup = gpu_unique(d2, T, nb)
+    Uo, sco, dupo = oracle.append_unique(T, nb)
+    assert np.array_equal(U, Uo) and np.array_equal(sc, sco) and np.array_equal(dup, dupo), i
+assert d2.device_error() == 0
+d2.destroy()
+print("CYCLE OK")
+'''
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", code], cwd=root, env=dict(os.environ, WG_EPOCH_START="250"),
+                       capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0 and "CYCLE OK" in r.stdout, r.stdout + r.stderr
 
 
 def test_gather_occupancy_setting(tiny):
