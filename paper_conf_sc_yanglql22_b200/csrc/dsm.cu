@@ -148,6 +148,12 @@ static wg_status alloc_workspace(wg_dsm* h, int64_t max_keys) {
     compact_ok = (c && c[0] == '0') ? 0 : 1;
   }
   w.compact = compact_ok && h->n <= (int64_t(1) << 28) && max_keys < (int64_t(1) << 28) ? 1 : 0;
+  static int pad32_ok = -1;
+  if (pad32_ok < 0) {
+    const char* c = getenv("WG_PAD32");
+    pad32_ok = (c && c[0] == '0') ? 0 : 1;
+  }
+  w.pad32 = pad32_ok && h->n < (int64_t(1) << 32) ? 1 : 0;
   if (w.compact) {
     WG_CUDA_TRY(cudaMemset(w.hslots, 0, cap * sizeof(HashSlot)));  // every word stale (epoch 0)
   } else {

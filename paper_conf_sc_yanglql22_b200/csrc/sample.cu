@@ -45,12 +45,13 @@ struct SampleArgs {
   int hop;
   unsigned long long seed;
   const unsigned long long* d_seed;
-  int64_t* nbrs_pad;  // [nT * M]
+  int64_t* nbrs_pad;  // [nT * M] (uint32 elements when pad32)
   int32_t* pos_pad;   // [nT * M]
   int32_t* cnt;       // [nT]
   unsigned* ctrl;
   int rp_keep;        // 1: row_ptr loads carry an L2 evict_last hint (WG_RP_EVICT_LAST)
   unsigned long long* hclear;  // fused hop, compact hash table: zeroed here when its epoch cycle restarts
+  int pad32;                   // padded neighbour slots hold uint32 ids (num_nodes < 2^32)
   int64_t hwords;
 };
 
@@ -175,7 +176,7 @@ __global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs
 #pragma unroll
   for (int u = 0; u < SAMPLE_UNR; ++u) {
     if (ok[u]) {
-      a.nbrs_pad[dst[u]] = nb[u];
+      st_pad(a.nbrs_pad, a.pad32, dst[u], nb[u]);
       if (a.pos_pad) a.pos_pad[dst[u]] = (int32_t)pos[u];
     }
   }
@@ -237,7 +238,7 @@ __global__ void __launch_bounds__(BT) sample_block_kernel(const SampleArgs a) {
   const int64_t* col = a.s.col[o] + s_start;
   if (N <= (unsigned)M) {  // L118: all of N neighbours, CSR order (A5)
     for (unsigned j = i; j < N; j += BT) {
-      a.nbrs_pad[k * M + j] = col[j];
+      st_pad(a.nbrs_pad, a.pad32, k * M + j, col[j]);
       if (a.pos_pad) a.pos_pad[k * M + j] = (int32_t)j;
     }
     return;
@@ -299,7 +300,7 @@ __global__ void __launch_bounds__(BT) sample_block_kernel(const SampleArgs a) {
       res = s_r[i];
     else
       res = s_last[(unsigned)(s_key[qi - 1] & 0xffffffffu)];
-    a.nbrs_pad[k * M + i] = col[res];
+    st_pad(a.nbrs_pad, a.pad32, k * M + i, col[res]);
     if (a.pos_pad) a.pos_pad[k * M + i] = (int32_t)res;
   }
 }
@@ -323,6 +324,7 @@ struct CompactArgs {
   int64_t* d_num_edges;
   unsigned long long* status;
   unsigned* ctrl;
+  int pad32;
 };
 
 __global__ void __launch_bounds__(COMPACT_THREADS) sample_compact_kernel(const CompactArgs a) {
@@ -353,7 +355,7 @@ __global__ void __launch_bounds__(COMPACT_THREADS) sample_compact_kernel(const C
     if (k < nT) {
       a.out_row_ptr[k] = off;
       for (int i = 0; i < c; ++i) {
-        a.out_nbrs[off + i] = a.nbrs_pad[k * a.M + i];
+        a.out_nbrs[off + i] = ld_pad(a.nbrs_pad, a.pad32, k * a.M + i);
         if (a.out_pos) a.out_pos[off + i] = a.pos_pad[k * a.M + i];
       }
       if (k == nT - 1) {
@@ -389,6 +391,7 @@ cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap,
   a.seed = seed;
   a.d_seed = reinterpret_cast<const unsigned long long*>(d_seed);
   a.nbrs_pad = h->ws.nbrs_pad;
+  a.pad32 = h->ws.pad32;
   a.pos_pad = want_pos ? h->ws.pos_pad : nullptr;
   a.cnt = h->ws.cnt;
   a.ctrl = h->ws.ctrl;
@@ -433,7 +436,7 @@ cudaError_t launch_sample(wg_dsm* h, const int64_t* targets, int64_t cap, const 
   cudaError_t e = launch_sample_padded(h, targets, cap, d_n, fanout, seed, d_seed, hop, out_pos != nullptr, st);
   if (e != cudaSuccess) return e;
   CompactArgs c{cap, d_n, fanout, h->ws.nbrs_pad, h->ws.pos_pad, h->ws.cnt, out_row_ptr, out_nbrs, out_pos,
-                d_num_edges, h->ws.status_sample, h->ws.ctrl};
+                d_num_edges, h->ws.status_sample, h->ws.ctrl, h->ws.pad32};
   const unsigned blocks = (unsigned)(cap > 0 ? (cap + COMPACT_TILE - 1) / COMPACT_TILE : 1);
   return launch_pdl(sample_compact_kernel, blocks, COMPACT_THREADS, 0, st, c);
 }

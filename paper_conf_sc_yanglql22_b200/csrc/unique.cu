@@ -63,6 +63,7 @@ struct UniqueArgs {
   int32_t* excl;
   int32_t* slot_of;
   HashTable ht;
+  int pad32;               // PADDED: nbrs holds uint32 ids
   unsigned long long* status;
   unsigned* ctrl;
   int64_t n;
@@ -104,7 +105,7 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueA
       } else if (PADDED) {
         const int64_t j = q - nT;
         const unsigned k = a.Mdiv.div((unsigned)j);
-        key = a.nbrs[j];  // loaded together with the count (ignored for a padding slot)
+        key = ld_pad(a.nbrs, a.pad32, j);  // loaded together with the count (ignored for a padding slot)
         valid = (int)((unsigned)j - k * (unsigned)a.M) < a.cnt[k];
         if (!valid) a.slot_of[q] = SLOT_EMPTY;  // padding slot: no sample here
       } else {
@@ -195,7 +196,7 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArg
       const bool in = j < nE;
       // every position's slot (the insert pass wrote SLOT_EMPTY for padding): no count read needed
       slots[t] = in ? a.slot_of[nT + j] : SLOT_EMPTY;
-      keys[t] = in ? a.nbrs[j] : -1;  // needed only after the scan: issued now
+      keys[t] = in ? (PADDED ? ld_pad(a.nbrs, a.pad32, j) : a.nbrs[j]) : -1;  // needed after the scan: issued now
     }
     unsigned long long wv = 0, wf = 0;
 #pragma unroll
@@ -434,6 +435,7 @@ cudaError_t launch_hop(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t*
   a.capT = capT;
   a.d_nT = d_nT;
   a.nbrs = h->ws.nbrs_pad;
+  a.pad32 = h->ws.pad32;
   a.capE = capT * fanout;
   a.d_nE = nullptr;
   a.M = fanout;

@@ -61,6 +61,7 @@ struct Workspace {
   int64_t hcap = 0;                      // slots (a multiple of 8); each call uses a prefix
   double hfactor = 2.0;                  // slots per key bound (WG_HASH_FACTOR)
   int compact = 0;                       // 8 B slots {epoch8, key28, pos28} (hash.cuh), else 16 B slots
+  int pad32 = 0;                         // padded sampler slots hold uint32 ids (num_nodes < 2^32)
   unsigned long long* status_sample = nullptr;  // decoupled look-back tile status
   unsigned long long* status_unique = nullptr;
   int64_t status_cap = 0;
@@ -139,6 +140,17 @@ template <typename... KArgs, typename... Args>
 inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
                               Args... args) {
   return launch_pdl_w(nullptr, kernel, grid, block, smem, st, args...);
+}
+
+// padded sampler slots: int64 ids, or uint32 ids when every id fits (half the bytes)
+__device__ __forceinline__ void st_pad(int64_t* p, int pad32, int64_t i, int64_t v) {
+  if (pad32)
+    reinterpret_cast<uint32_t*>(p)[i] = (uint32_t)v;
+  else
+    p[i] = v;
+}
+__device__ __forceinline__ int64_t ld_pad(const int64_t* p, int pad32, int64_t i) {
+  return pad32 ? (int64_t)reinterpret_cast<const uint32_t*>(p)[i] : p[i];
 }
 
 // launchers (stream-ordered); arguments already validated by the ABI layer
