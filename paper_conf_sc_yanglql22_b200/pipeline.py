@@ -34,6 +34,7 @@ def required_keys(n, fanouts, max_seeds):
 # several at a time on one GPU: a gather at full occupancy holds the whole register file and keeps
 # the other streams' latency-bound hop kernels from overlapping it ("Concurrency").
 THROUGHPUT_GATHER_OCCUPANCY = 1
+PARAMS_RING = 64  # pinned staging slots for the per-batch scalars (batches enqueued ahead per pipeline)
 
 
 class MiniBatchPipeline:
@@ -56,16 +57,23 @@ class MiniBatchPipeline:
         i64 = dict(dtype=torch.int64, device=dev)
         i32 = dict(dtype=torch.int32, device=dev)
         self.seeds = torch.zeros(max(self.max_seeds, 1), **i64)
-        self.n_seeds = torch.zeros(1, **i64)
-        self.rng_seed = torch.zeros(1, **i64)       # uint64 bit pattern
+        # per-batch scalars in one device buffer [n_seeds, rng_seed (uint64 bit pattern)], written by ONE
+        # H2D copy from a pinned staging buffer; per-hop counts in one [H, 2] buffer (one D2H copy)
+        self.params = torch.zeros(2, **i64)
+        self.n_seeds, self.rng_seed = self.params[0:1], self.params[1:2]
+        # a ring of pinned staging buffers, so the host can enqueue many batches ahead without waiting
+        self._params_host = torch.zeros((PARAMS_RING, 2), dtype=torch.int64, pin_memory=True)
+        self._params_ev = [None] * PARAMS_RING
+        self._params_next = 0
+        self.counts_dev = torch.zeros((len(self.fanouts), 2), **i64)
         self.hops = []
         for h, m in enumerate(self.fanouts):
             T, E, U = self.T_cap[h], self.E_cap[h], self.U_cap[h]
             self.hops.append(dict(
                 row_ptr=torch.zeros(T + 1, **i64), nbrs=torch.zeros(max(E, 1), **i64),
                 pos=torch.zeros(max(E, 1), **i32) if with_pos else None,
-                num_edges=torch.zeros(1, **i64), unique=torch.zeros(max(T + E, 1), **i64),
-                num_unique=torch.zeros(1, **i64), sub_col=torch.zeros(max(E, 1), **i32),
+                num_edges=self.counts_dev[h, 0:1], unique=torch.zeros(max(T + E, 1), **i64),
+                num_unique=self.counts_dev[h, 1:2], sub_col=torch.zeros(max(E, 1), **i32),
                 dup=torch.zeros(max(T + E, 1), **i32) if with_dup else None))
         # X is pitched to a 32 B multiple so every row moves as whole 32 B vectors; X_rows is the
         # [U, row_bytes] view of the feature bytes (self.X[:, :row_bytes])
@@ -127,16 +135,25 @@ class MiniBatchPipeline:
         self.dsm.gather_rows(last["unique"], self.U_cap[-1], None, last["num_unique"], self.X, stream=stream)
 
     def set_inputs(self, seeds: torch.Tensor, rng_seed: int, stream=None):
-        """Copy this batch's seed nodes (device or pinned host int64) and rng_seed
-        into the pipeline's device buffers (stream-ordered)."""
+        """Copy this batch's seed nodes (device or pinned host int64) and (n_seeds, rng_seed) into the
+        pipeline's device buffers: two stream-ordered copies, no kernel."""
         n = seeds.numel()
         if n > self.max_seeds:
             raise ValueError("too many seeds")
         s = stream or torch.cuda.current_stream()
+        k = self._params_next
+        self._params_next = (k + 1) % PARAMS_RING
+        if self._params_ev[k] is not None:
+            self._params_ev[k].synchronize()   # that slot's earlier copy has read it (PARAMS_RING batches ago)
+        else:
+            self._params_ev[k] = torch.cuda.Event()
+        stage = self._params_host[k]
+        stage[0] = n
+        stage[1] = to_i64(rng_seed)
         with torch.cuda.stream(s):
             self.seeds[:n].copy_(seeds, non_blocking=True)
-            self.n_seeds.fill_(n)
-            self.rng_seed.fill_(to_i64(rng_seed))
+            self.params.copy_(stage, non_blocking=True)
+            self._params_ev[k].record(s)
 
     def run(self, seeds, rng_seed, stream=None):
         self.set_inputs(seeds, rng_seed, stream)
@@ -256,10 +273,7 @@ class MiniBatchLoader:
             else:
                 pl.enqueue(st)
                 self.warm[j] += 1
-            c = self.counts[j]
-            for h, b in enumerate(pl.hops):
-                c[h, 0:1].copy_(b["num_edges"], non_blocking=True)
-                c[h, 1:2].copy_(b["num_unique"], non_blocking=True)
+            self.counts[j].copy_(pl.counts_dev, non_blocking=True)  # every hop's (edges, unique): one D2H
             self.done[j].record(st)
         if self.use_graphs and self.graphs[j] is None and self.warm[j] >= 1:
             self._capture(j)
