@@ -5,7 +5,7 @@ import sys
 from collections import OrderedDict
 
 rows = list(csv.reader(open(sys.argv[1])))
-n = int(sys.argv[2]) if len(sys.argv) > 2 else 15  # one batch of the shipped graph: (sample, insert, flag, relabel, gather_rows) x 3 hops
+n = int(sys.argv[2]) if len(sys.argv) > 2 else 13  # bench.py ends with its stage breakdown: one batch = (sample, insert, flag, relabel) x 3 hops + the whole gather
 for i, r in enumerate(rows):
     if r and r[0] == "ID":
         hdr, start = r, i
