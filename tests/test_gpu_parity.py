@@ -548,3 +548,57 @@ def test_gather_occupancy_setting(tiny):
         dsm.set_gather_occupancy(-1)
     assert dsm.device_error() == 0
     dsm.destroy()
+
+
+@pytest.mark.parametrize("env", [{"WG_HASH_COMPACT": "0"}, {"WG_HASH_COMPACT": "0", "WG_HASH_CAS128": "0"},
+                                 {"WG_PAD32": "0"}, {"WG_HASH_PER_CALL": "0"}])
+def test_table_and_slot_formats_subprocess(env):
+    """The non-default hash-table / padded-slot formats (16 B wide slots with 128-bit or 64-bit CAS
+    claims, int64 padded sampler slots, whole-table calls) stay bit-exact: 12 tiny batches through
+    the fused pipeline and hub-heavy standalone append-unique calls."""
+    import os
+    import subprocess
+    import sys
+    code = r'''
+import sys, numpy as np, torch
+sys.path.insert(0, "tests")
+import oracle
+import paper_conf_sc_yanglql22_b200 as pkg
+from paper_conf_sc_yanglql22_b200 import loader
+from gpu_helpers import make_dsm, gpu_unique
+from synth import graph, presets, seeds
+p = presets.get("tiny")
+rp, col = graph.csr(p.graph())
+rows = loader.host_row_provider(p.graph(), rp, col)
+feats = loader.host_feat_provider(p)
+dsm, _ = loader.build_dsm(p, on_device=False)
+pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
+for b in range(12):
+    S = seeds.seed_nodes(p.n, p.seeds_per_batch - b * 7, presets.SEED_BASE, 300 + b)
+    rs = seeds.rng_seed(presets.RNG_BASE, 300 + b)
+    pipe.run(torch.from_numpy(S).cuda(), rs)
+    torch.cuda.synchronize()
+    ref = oracle.minibatch(rows, feats, S, p.fanouts, rs)
+    for h in range(len(p.fanouts)):
+        got, exp = pipe.result(h), ref["hops"][h]
+        for k in ("row_ptr", "nbrs", "pos", "unique", "sub_col", "dup"):
+            assert np.array_equal(got[k], exp[k]), (b, h, k)
+    assert np.array_equal(pipe.features(), ref["X"]), b
+assert dsm.device_error() == 0
+dsm.destroy()
+rng = np.random.default_rng(11)
+d2 = make_dsm(np.zeros(5001, np.int64), np.zeros(0, np.int64), max_keys=1 << 16)
+for i in range(20):
+    T = rng.choice(5000, 300, replace=False).astype(np.int64)
+    nb = np.minimum((rng.pareto(1.2, 20000) * 3).astype(np.int64), 4999)   # hub-heavy
+    U, sc, dup = gpu_unique(d2, T, nb)
+    Uo, sco, dupo = oracle.append_unique(T, nb)
+    assert np.array_equal(U, Uo) and np.array_equal(sc, sco) and np.array_equal(dup, dupo), i
+assert d2.device_error() == 0
+d2.destroy()
+print("FORMAT OK")
+'''
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-c", code], cwd=root, env=dict(os.environ, **env),
+                       capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0 and "FORMAT OK" in r.stdout, r.stdout + r.stderr
