@@ -111,6 +111,7 @@ struct GatherArgs {
   uint8_t* out;
   unsigned* ctrl;
   FastDiv cpr;  // chunks per row
+  int st_hint;  // X stores: 0 default, 1 L2 evict_first policy, 2 .cs (streaming) (WG_GATHER_ST_HINT)
 };
 
 template <typename V>
@@ -122,6 +123,17 @@ __device__ __forceinline__ void st_out<u32x8>(u32x8* p, const u32x8& r) {
   asm volatile("st.global.v8.u32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "r"(r.v[0]), "r"(r.v[1]), "r"(r.v[2]),
                "r"(r.v[3]), "r"(r.v[4]), "r"(r.v[5]), "r"(r.v[6]), "r"(r.v[7])
                : "memory");
+}
+
+__device__ __forceinline__ void st_out_hint(u32x8* p, const u32x8& r, int hint, unsigned long long pol) {
+  if (hint == 1)
+    asm volatile("st.global.L2::cache_hint.v8.u32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8}, %9;" ::"l"(p), "r"(r.v[0]),
+                 "r"(r.v[1]), "r"(r.v[2]), "r"(r.v[3]), "r"(r.v[4]), "r"(r.v[5]), "r"(r.v[6]), "r"(r.v[7]), "l"(pol)
+                 : "memory");
+  else
+    asm volatile("st.global.cs.v8.u32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"l"(p), "r"(r.v[0]), "r"(r.v[1]),
+                 "r"(r.v[2]), "r"(r.v[3]), "r"(r.v[4]), "r"(r.v[5]), "r"(r.v[6]), "r"(r.v[7])
+                 : "memory");
 }
 
 template <typename V, int GATHER_UNROLL>
@@ -144,6 +156,8 @@ __global__ void __launch_bounds__(GATHER_THREADS) gather_kernel(const GatherArgs
   const unsigned stride = gridDim.x * GATHER_THREADS;
   V* __restrict__ out = reinterpret_cast<V*>(a.out + begin * (int64_t)cpr * (int64_t)sizeof(V));
   const unsigned long long pol = l2_evict_last_policy();
+  unsigned long long stp;
+  asm("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(stp));
   for (unsigned c0 = blockIdx.x * GATHER_THREADS + threadIdx.x; c0 < total; c0 += stride * GATHER_UNROLL) {
     V val[GATHER_UNROLL];
     unsigned dst[GATHER_UNROLL];
@@ -168,7 +182,15 @@ __global__ void __launch_bounds__(GATHER_THREADS) gather_kernel(const GatherArgs
     }
 #pragma unroll
     for (int j = 0; j < GATHER_UNROLL; ++j)
-      if (dst[j] < total) st_out<V>(&out[dst[j]], val[j]);
+      if (dst[j] < total) {
+        if constexpr (sizeof(V) == 32) {
+          if (a.st_hint) {
+            st_out_hint(reinterpret_cast<u32x8*>(&out[dst[j]]), *reinterpret_cast<const u32x8*>(&val[j]), a.st_hint, stp);
+            continue;
+          }
+        }
+        st_out<V>(&out[dst[j]], val[j]);
+      }
   }
 }
 
@@ -427,7 +449,13 @@ cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int6
                  : (cw % 16 == 0 && oa % 16 == 0)           ? 16
                  : (cw % 4 == 0 && oa % 4 == 0)             ? 4
                                                             : 2;
-  GatherArgs a{h->view, ids, cap, d_n, d_begin, static_cast<uint8_t*>(out), h->ws.ctrl, FastDiv((unsigned)(cw / vb))};
+  static int st_hint = -1;
+  if (st_hint < 0) {
+    const char* e = getenv("WG_GATHER_ST_HINT");
+    st_hint = e ? atoi(e) : 0;
+  }
+  GatherArgs a{h->view, ids, cap, d_n, d_begin, static_cast<uint8_t*>(out), h->ws.ctrl, FastDiv((unsigned)(cw / vb)),
+               st_hint};
   if (use_g4) {
     const cudaError_t e = launch_gather_g4(h, ids, cap, d_n, d_begin, out, cw, st);
     if (e != cudaErrorNotSupported) return e;
