@@ -279,8 +279,10 @@ wg_status wg_dsm_set_gather_occupancy(wg_dsm_t h, int32_t blocks_per_sm);
  * handle's device. */
 wg_status wg_device_error(wg_dsm_t h, uint32_t* code, int32_t clear);
 
-/* Clear the append-unique hash table and restart its epoch counter (needed only
- * after WG_DEVERR_EPOCH, i.e. after ~8M wg_append_unique calls).  Stream-ordered. */
+/* Clear the append-unique hash table and restart its epoch counter.  Stream-ordered.
+ * Needed only with the wide 16 B table format (node ids or positions >= 2^28, or
+ * WG_HASH_COMPACT=0) after WG_DEVERR_EPOCH, i.e. after ~8M append-unique calls; the compact
+ * 8 B format cycles through 255 epochs and clears itself when a cycle restarts. */
 wg_status wg_dsm_reset_workspace(wg_dsm_t h, wg_stream_t stream);
 
 /* Thread-local message describing the last non-OK status. */
