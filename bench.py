@@ -43,6 +43,7 @@ def parse():
     ap.add_argument("--sweep", action="store_true", help="config 4: feature-gather sweep over row sizes")
     ap.add_argument("--sweep-rows", type=int, default=100_000_000)
     ap.add_argument("--sweep-ids", type=int, default=1_000_000)
+    ap.add_argument("--sweep-cells", default=None, help="comma list of dtype:dim cells (default: the whole grid)")
     ap.add_argument("--latency", action="store_true", help="Table I analogue: dependent-load latency vs span")
     ap.add_argument("--layer", action="store_true", help="NEXT #2: g-SpMM mean aggregation on a prepared batch")
     ap.add_argument("--pass-b", default="both", choices=["both", "prep", "gather"],
@@ -645,6 +646,22 @@ def bench_sweep(args):
     cells = []
     grid = [("fp16", d) for d in (2, 4, 8, 16, 32)]  # 4-64 B segments (Fig. 8's small sizes, NEXT #3)
     grid += [(t, d) for t in ("fp16", "fp32") for d in (64, 128, 256, 512, 768, 1024)]
+    if args.sweep_cells:
+        grid = [(c.split(":")[0], int(c.split(":")[1])) for c in args.sweep_cells.split(",")]
+    else:
+        # every cell in a fresh process: after the 100+ GB tables of the large cells the allocator's
+        # physical memory is fragmented and a later table can land on small pages (measured: a 256 B
+        # cell at 0.58 after the 1.5 KB cell in the same process, 0.85 in a fresh one)
+        for dtype, dim in grid:
+            r = subprocess.run([sys.executable, os.path.abspath(__file__), "--sweep", "--sweep-cells", f"{dtype}:{dim}",
+                                "--steps", str(args.steps), "--sweep-rows", str(n), "--sweep-ids", str(R)],
+                               capture_output=True, text=True, timeout=900)
+            lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+            if r.returncode != 0 or not lines:
+                cells.append({"dtype": dtype, "dim": dim, "error": (r.stderr or r.stdout)[-300:]})
+                continue
+            cells += json.loads(lines[-1])["cells"]
+        grid = []
     for dtype, dim in grid:
         if True:
             rb = dim * sfeat.elt_bytes(dtype)
@@ -678,7 +695,9 @@ def bench_sweep(args):
             del out
             dsm.destroy()
             torch.cuda.empty_cache()
-    best = max((c for c in cells if "ms" in c), key=lambda c: c["frac_of_hbm_roofline"])
+    measured = [c for c in cells if "ms" in c]
+    best = max(measured, key=lambda c: c["frac_of_hbm_roofline"]) if measured else \
+        {"hbm_gbs_read_plus_write": None, "frac_of_hbm_roofline": None}
     line = {"metric": "feature gather GB/s vs HBM roofline (config 4 sweep, W=1)", "value": best["hbm_gbs_read_plus_write"],
             "unit": "GB/s", "n_gpus": 1, "steps": args.steps, "warmup": 3, "higher_is_better": True,
             "config": {"workload": "gather-sweep", "rows": n, "ids_per_rank": R, "ids": "uniform with replacement",
