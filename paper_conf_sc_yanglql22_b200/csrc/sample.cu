@@ -29,6 +29,9 @@
 namespace wg {
 
 constexpr int SAMPLE_THREADS = 256;
+#ifndef SAMPLE_MINB
+#define SAMPLE_MINB 6  // resident sampler blocks per SM the register allocation must allow
+#endif
 constexpr int SAMPLE_UNR_MAX = 4;
 // SAMPLE_UNR = rounds per warp, all in flight at once (1, 2 or 4; chosen per launch: small hops use
 // fewer rounds per warp and therefore more blocks / SMs)
@@ -75,7 +78,7 @@ __device__ __forceinline__ int64_t ld_rp(const int64_t* p, int keep) {
 }
 
 template <int SAMPLE_UNR, bool CLR>
-__global__ void __launch_bounds__(SAMPLE_THREADS) sample_kernel(const SampleArgs a) {
+__global__ void __launch_bounds__(SAMPLE_THREADS, SAMPLE_MINB) sample_kernel(const SampleArgs a) {
   pdl_enter();
   if (CLR) clear_table_if_cycle_restarts(a.hclear, a.hwords, a.ctrl);
   __shared__ unsigned sm_chain[SAMPLE_THREADS / 32][32];
