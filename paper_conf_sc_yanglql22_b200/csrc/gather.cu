@@ -20,6 +20,9 @@
 namespace wg {
 
 constexpr int GATHER_THREADS = 256;
+#ifndef GATHER_MINB
+#define GATHER_MINB 5  // resident gather blocks per SM the register allocation must allow
+#endif
 #ifndef V32_UNROLL
 #define V32_UNROLL 4  // 32 B loads in flight per thread (A/B: 2 was slower, 0.88 vs 0.93 for 512 B rows)
 #endif
@@ -137,7 +140,7 @@ __device__ __forceinline__ void st_out_hint(u32x8* p, const u32x8& r, int hint, 
 }
 
 template <typename V, int GATHER_UNROLL>
-__global__ void __launch_bounds__(GATHER_THREADS) gather_kernel(const GatherArgs a) {
+__global__ void __launch_bounds__(GATHER_THREADS, GATHER_MINB) gather_kernel(const GatherArgs a) {
   pdl_enter();
   int64_t n = a.cap;
   if (a.d_n) {
