@@ -23,6 +23,9 @@ constexpr int GATHER_THREADS = 256;
 #ifndef GATHER_MINB
 #define GATHER_MINB 5  // resident gather blocks per SM the register allocation must allow
 #endif
+#ifndef GATHER_LEAN_MINB
+#define GATHER_LEAN_MINB 6
+#endif
 #ifndef V32_UNROLL
 #define V32_UNROLL 4  // 32 B loads in flight per thread (A/B: 2 was slower, 0.88 vs 0.93 for 512 B rows)
 #endif
@@ -139,8 +142,11 @@ __device__ __forceinline__ void st_out_hint(u32x8* p, const u32x8& r, int hint, 
                  : "memory");
 }
 
-template <typename V, int GATHER_UNROLL>
-__global__ void __launch_bounds__(GATHER_THREADS, GATHER_MINB) gather_kernel(const GatherArgs a) {
+// MINB: resident blocks per SM the register allocation must allow -- GATHER_MINB for a gather that
+// fills the GPU alone; GATHER_LEAN_MINB (fewer registers, a few spills) for throughput-mode gathers
+// capped at a block or two per SM, whose register file the other streams' hop kernels then use.
+template <typename V, int GATHER_UNROLL, int MINB = GATHER_MINB>
+__global__ void __launch_bounds__(GATHER_THREADS, MINB) gather_kernel(const GatherArgs a) {
   pdl_enter();
   int64_t n = a.cap;
   if (a.d_n) {
@@ -520,6 +526,13 @@ cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int6
   blocks = blocks < 1 ? 1 : (blocks > max_blocks ? max_blocks : blocks);
   const unsigned gb = (unsigned)blocks;
   const cudaAccessPolicyWindow* w = &h->tail_window;  // num_bytes == 0 unless WG_TAIL_PERSIST=2
+  static int lean = -1;  // A/B knob WG_GATHER_LEAN=0: the full-occupancy kernel for capped launches too
+  if (lean < 0) {
+    const char* e = getenv("WG_GATHER_LEAN");
+    lean = (e && e[0] == '0') ? 0 : 1;
+  }
+  if (vb == 32 && lean && per_sm <= 2)
+    return launch_pdl_w(w, gather_kernel<u32x8, V32_UNROLL, GATHER_LEAN_MINB>, gb, GATHER_THREADS, 0, st, a);
   if (vb == 32) return launch_pdl_w(w, gather_kernel<u32x8, V32_UNROLL>, gb, GATHER_THREADS, 0, st, a);
   if (vb == 16) return launch_pdl_w(w, gather_kernel<uint4, 4>, gb, GATHER_THREADS, 0, st, a);
   if (vb == 4) return launch_pdl_w(w, gather_kernel<unsigned, 4>, gb, GATHER_THREADS, 0, st, a);
