@@ -23,8 +23,11 @@ constexpr int GATHER_THREADS = 256;
 #ifndef GATHER_MINB
 #define GATHER_MINB 5  // resident gather blocks per SM the register allocation must allow
 #endif
+#ifndef LEAN_UNROLL
+#define LEAN_UNROLL 2  // loads in flight per thread of the lean throughput-mode gather
+#endif
 #ifndef GATHER_LEAN_MINB
-#define GATHER_LEAN_MINB 6
+#define GATHER_LEAN_MINB 8
 #endif
 #ifndef V32_UNROLL
 #define V32_UNROLL 4  // 32 B loads in flight per thread (A/B: 2 was slower, 0.88 vs 0.93 for 512 B rows)
@@ -532,7 +535,7 @@ cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int6
     lean = (e && e[0] == '0') ? 0 : 1;
   }
   if (vb == 32 && lean && per_sm <= 2)
-    return launch_pdl_w(w, gather_kernel<u32x8, V32_UNROLL, GATHER_LEAN_MINB>, gb, GATHER_THREADS, 0, st, a);
+    return launch_pdl_w(w, gather_kernel<u32x8, LEAN_UNROLL, GATHER_LEAN_MINB>, gb, GATHER_THREADS, 0, st, a);
   if (vb == 32) return launch_pdl_w(w, gather_kernel<u32x8, V32_UNROLL>, gb, GATHER_THREADS, 0, st, a);
   if (vb == 16) return launch_pdl_w(w, gather_kernel<uint4, 4>, gb, GATHER_THREADS, 0, st, a);
   if (vb == 4) return launch_pdl_w(w, gather_kernel<unsigned, 4>, gb, GATHER_THREADS, 0, st, a);
