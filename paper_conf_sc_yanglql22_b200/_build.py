@@ -17,6 +17,8 @@ NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", "-O2", "--expt-relaxed-constexpr",
          "-I", INCLUDE]
+# extra compile-time knobs for A/B builds, e.g. WG_NVCC_DEFS="-DWG_LB_SLEEP_NS=0" (default build: none)
+FLAGS += os.environ.get("WG_NVCC_DEFS", "").split()
 
 
 def _stale(target, deps):

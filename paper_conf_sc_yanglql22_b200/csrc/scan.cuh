@@ -7,7 +7,18 @@
 
 #include "device_util.cuh"
 
+// Back-off between polls of a predecessor tile that has published nothing yet (ns; 0 = spin).
+#ifndef WG_LB_SLEEP_NS
+#define WG_LB_SLEEP_NS 32
+#endif
+
 namespace wg {
+
+__device__ __forceinline__ void lb_backoff() {
+#if WG_LB_SLEEP_NS > 0
+  __nanosleep(WG_LB_SLEEP_NS);
+#endif
+}
 
 template <int NT>
 struct LookbackSmem {
@@ -35,7 +46,7 @@ __device__ __forceinline__ unsigned long long block_lookback(unsigned long long*
     const long idx = tile - 1 - lane;
     unsigned long long s = idx >= 0 ? ld_volatile_u64(&status[idx]) : LB_PRE;
     while ((s >> 62) == 0) {
-      __nanosleep(32);
+      lb_backoff();
       s = ld_volatile_u64(&status[idx]);
     }
     const unsigned pm = __ballot_sync(FULL_MASK, (s >> 62) == 2);
@@ -55,7 +66,7 @@ __device__ __forceinline__ unsigned long long block_lookback(unsigned long long*
     const long idx = pred - tid;
     unsigned long long s = idx >= 0 ? ld_volatile_u64(&status[idx]) : LB_PRE;
     while ((s >> 62) == 0) {
-      __nanosleep(32);
+      lb_backoff();
       s = ld_volatile_u64(&status[idx]);
     }
     const unsigned pm = __ballot_sync(FULL_MASK, (s >> 62) == 2);
