@@ -32,9 +32,13 @@
 #include "hash.cuh"
 #include "scan.cuh"
 
+#ifndef WG_UQ_THREADS
+#define WG_UQ_THREADS 256  // threads per append-unique block (A/B knob via WG_NVCC_DEFS)
+#endif
+
 namespace wg {
 
-constexpr int UQ_THREADS = 256;
+constexpr int UQ_THREADS = WG_UQ_THREADS;
 // neighbour positions per thread of the flag scan: 1..8, chosen per launch so that small hops
 // spread over many SMs (latency-bound) and large hops keep several loads in flight per thread
 constexpr int CNT_BITS = 31;                    // packed scan value: (valid << 31) | first
