@@ -28,7 +28,10 @@
 
 namespace wg {
 
-constexpr int SAMPLE_THREADS = 256;
+#ifndef WG_SAMPLE_THREADS
+#define WG_SAMPLE_THREADS 256  // threads per sampler block (A/B knob via WG_NVCC_DEFS)
+#endif
+constexpr int SAMPLE_THREADS = WG_SAMPLE_THREADS;
 #ifndef SAMPLE_MINB
 #define SAMPLE_MINB 6  // resident sampler blocks per SM the register allocation must allow
 #endif
