@@ -65,7 +65,18 @@ typedef enum { WG_F32 = 0, WG_F16 = 1, WG_BF16 = 2 } wg_dtype;
 #define WG_DEVERR_CAPACITY   0x4u  /* a device count exceeded its host capacity, or the hash table filled */
 #define WG_DEVERR_DEGREE     0x8u  /* a degree >= 2^32 (A3 requires N < 2^32) */
 #define WG_DEVERR_EPOCH      0x10u /* hash-table epoch space exhausted: call wg_dsm_reset_workspace */
-#define WG_DEVERR_TMA        0x20u /* a TMA gather stage never completed (the kernel stopped instead of hanging) */
+
+/* wg_dsm_desc.flags (layout / placement choices of one DSM; results never depend on the layout
+ * flags, only on the graph, the table and the inputs). */
+#define WG_DSM_WHOLE_ROWS     0x1u  /* feature rows stored whole (never split into body + tail, see
+                                       wg_dsm_feat_layout) */
+#define WG_DSM_WIDE_HASH      0x2u  /* 16 B append-unique hash slots even when node ids and positions fit
+                                       the compact 8 B format (the format used for num_nodes >= 2^28) */
+#define WG_DSM_PAD64          0x4u  /* int64 padded sampler slots even when every id fits 32 bits */
+#define WG_DSM_CSR_REPLICATED 0x8u  /* hybrid placement: every rank holds the WHOLE
+                                       CSR (row_ptr int64[num_nodes+1], col_idx int64[local_num_edges =
+                                       all E]) and samples locally; only the feature table is row-sharded
+                                       (o(v) = v mod W) and read over NVLink.  Results are identical. */
 
 /* Allgather of host bytes across the W ranks of the DSM ("an
  * AllGather pattern communication is performed so that each process can get all
@@ -90,11 +101,13 @@ typedef struct {
                                n_targets passed to wg_sample_neighbors */
   wg_allgather_fn allgather;
   void* ctx;                /* passed through to allgather */
+  uint32_t flags;           /* WG_DSM_* above (0 = the paper's placement, measured-best layout) */
+  uint32_t reserved;        /* must be 0 */
 } wg_dsm_desc;
 
 /* Create the DSM (section III-B).  COLLECTIVE over the W ranks.
- * Each rank allocates its shard slab on its device -- row_ptr int64[n_local+1],
- * col_idx int64[local_num_edges], features [n_local][row stride] (+ a tail region for the
+ * Each rank allocates its shard slab on its device -- row_ptr int64[n_local+1] (int64[num_nodes+1]
+ * with WG_DSM_CSR_REPLICATED), col_idx int64[local_num_edges], features [n_local][row stride] (+ a tail region for the
  * split row layout, see wg_dsm_feat_layout) -- exports a CUDA IPC handle, allgathers the
  * handles (L100), opens every peer's handle (L100-106; same-process peers are used
  * directly) and keeps the W base pointers as the "memory pointer table" (L106),
@@ -120,12 +133,13 @@ wg_status wg_dsm_local_view(wg_dsm_t h, int64_t** d_row_ptr, int64_t** d_col_idx
  * THIS rank's slab.  Otherwise body_bytes = R, body_pitch = R rounded up to 64, d_tail = NULL
  * and tail_pitch = 0.  Fillers write bytes [0, body_bytes) of local row l at
  * d_feat + l * body_pitch and bytes [body_bytes, R) at d_tail + l * tail_pitch.  The layout is
- * invisible to every op (wg_gather returns whole rows).  WG_FEAT_SPLIT=0 in the environment at
- * create disables the split (A/B).  Any output may be NULL. */
+ * invisible to every op (wg_gather returns whole rows).  The WG_DSM_WHOLE_ROWS flag at create
+ * disables the split (A/B).  Any output may be NULL. */
 wg_status wg_dsm_feat_layout(wg_dsm_t h, int64_t* body_bytes, int64_t* body_pitch, void** d_tail,
                              int64_t* tail_pitch);
 
-/* Geometry of rank r's shard (any r): local rows and local CSR entries. */
+/* Geometry of rank r's shard (any r): local feature rows and local CSR entries (with
+ * WG_DSM_CSR_REPLICATED: the whole CSR's entries; its rows are num_nodes). */
 wg_status wg_dsm_shard_info(wg_dsm_t h, int32_t r, int64_t* n_local_rows, int64_t* local_num_edges);
 
 /* A second handle on the SAME shards with its own workspace (hash table, scan
@@ -237,9 +251,10 @@ wg_status wg_rows_permute(const void* d_src, void* d_dst, const int64_t* d_perm,
  *           CSR with atomic adds (no transpose, L186); rows with d_dup_count == 1 (the
  *           Append Unique duplicate count; nullable) are written with a plain store
  *           (L186-192).  d_dx [n_x_rows, dim] is zeroed by the call.
- * d_n_rows: optional device count (as for the other ops). */
+ * d_x has n_x_rows rows; an edge whose sub-graph id lies outside [0, n_x_rows) (the -1 of an
+ * invalid id) is skipped in both directions.  d_n_rows: optional device count (as for the other ops). */
 wg_status wg_spmm_mean_forward(const int64_t* d_row_ptr, int64_t n_rows, const int64_t* d_n_rows,
-                               const int32_t* d_sub_col, const float* d_x, int64_t dim, float* d_y,
+                               const int32_t* d_sub_col, const float* d_x, int64_t n_x_rows, int64_t dim, float* d_y,
                                wg_stream_t stream);
 wg_status wg_spmm_mean_backward(const int64_t* d_row_ptr, int64_t n_rows, const int64_t* d_n_rows,
                                 const int32_t* d_sub_col, const int32_t* d_dup_count, const float* d_dy,
@@ -248,12 +263,29 @@ wg_status wg_spmm_mean_backward(const int64_t* d_row_ptr, int64_t n_rows, const 
 /* DSM characterisation, the analogue of PAPER.md Table I (L66-80): one GPU thread
  * performs `accesses` dependent 8 B loads at random 64 B-aligned offsets within the
  * first span_bytes of rank `rank`'s feature shard (local HBM when rank is this rank,
- * a peer's HBM over NVLink otherwise); each address is a hash of the previously loaded
- * value.  The caller times the launch (e.g. with CUDA events) and divides by
+ * a peer's HBM over NVLink otherwise); each address is the multiply-high of the previously
+ * loaded value (times a constant) with the slot count: two dependent integer multiplies
+ * (~4 ns) between a load's return and the next load.  The caller times the launch (e.g. with CUDA events) and divides by
  * `accesses`.  d_sink: one device uint64 receiving a checksum (keeps the loads live).
  * Errors: WG_ERR_INVALID_ARG if span_bytes exceeds that shard. */
 wg_status wg_dsm_chase(wg_dsm_t h, int32_t rank, int64_t span_bytes, int64_t accesses, uint64_t* d_sink,
                        wg_stream_t stream);
+
+/* Ceilings of the latency-bound prep kernels, measured on the box itself.
+ * wg_micro_random_read: blocks_per_sm x SMs blocks of 256 threads, each thread `rounds` times issuing
+ * 8 independent loads of `width` (8 or 32) bytes at hash-random width-aligned offsets of
+ * [d_buf, d_buf + span_bytes) -- the random-sector rate bounding the sampler (S1-S2: row_ptr pairs and
+ * col_idx entries at random rows).  wg_micro_atomics: the same shape of independent 64-bit atomics on
+ * random words of d_table[slots] -- op 0 = a CAS that never swaps (a probe), 1 = a CAS that swaps, 2 =
+ * atomicMin -- the L2 atomic rate bounding append-unique's insert pass (S3).  *loads_issued / *ops_issued
+ * (nullable) receive the operation count of the launch; the caller times it (CUDA events) on `stream`.
+ * d_sink: one device uint64 that keeps the results live.  d_table's contents are overwritten.
+ * Errors: WG_ERR_INVALID_ARG (null pointer, width not 8/32, span < width, rounds < 1,
+ * blocks_per_sm outside [1, 8], op outside [0, 2]). */
+wg_status wg_micro_random_read(const void* d_buf, int64_t span_bytes, int32_t width, int32_t rounds,
+                               int32_t blocks_per_sm, uint64_t* d_sink, int64_t* loads_issued, wg_stream_t stream);
+wg_status wg_micro_atomics(uint64_t* d_table, int64_t slots, int32_t op, int32_t rounds, int32_t blocks_per_sm,
+                           uint64_t* d_sink, int64_t* ops_issued, wg_stream_t stream);
 
 /* wg_gather restricted to rows [*d_begin, *d_end) of d_ids / d_out (device int64 scalars;
  * d_begin NULL = 0, d_end NULL = n_ids; both clamped to [0, n_ids]).  Row i is written at
@@ -281,9 +313,22 @@ wg_status wg_device_error(wg_dsm_t h, uint32_t* code, int32_t clear);
 
 /* Clear the append-unique hash table and restart its epoch counter.  Stream-ordered.
  * Needed only with the wide 16 B table format (node ids or positions >= 2^28, or
- * WG_HASH_COMPACT=0) after WG_DEVERR_EPOCH, i.e. after ~8M append-unique calls; the compact
+ * WG_DSM_WIDE_HASH) after WG_DEVERR_EPOCH, i.e. after ~8M append-unique calls; the compact
  * 8 B format cycles through 255 epochs and clears itself when a cycle restarts. */
 wg_status wg_dsm_reset_workspace(wg_dsm_t h, wg_stream_t stream);
+
+/* Diagnostics (per-kernel device times): while set, wg_sample_hop records events[0..n)
+ * in order after its kernels -- sampler, insert, flag scan, relabel (the relabel's on the side stream
+ * when one is given) -- and wg_append_unique after insert, flag scan, relabel.  events are cudaEvent_t
+ * handles owned by the caller; n = 0 clears.  Use with eager launches (not inside a graph capture).
+ * Errors: WG_ERR_INVALID_ARG if n is outside [0, 8] or events is NULL with n > 0. */
+wg_status wg_dsm_set_stage_events(wg_dsm_t h, void* const* events, int32_t n);
+
+/* Test hook: set the hash-table epoch counter of h's workspace (synchronous), e.g. near the end
+ * of the wide format's 2^23 epochs or of the compact format's 255-epoch cycle, so tests reach
+ * WG_DEVERR_EPOCH and the cycle restart in a few calls.  Errors: WG_ERR_INVALID_ARG if epoch is
+ * 0 or >= 2^23. */
+wg_status wg_dsm_debug_set_epoch(wg_dsm_t h, uint32_t epoch);
 
 /* Thread-local message describing the last non-OK status. */
 const char* wg_last_error(void);

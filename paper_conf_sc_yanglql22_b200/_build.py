@@ -10,7 +10,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.path.join(PKG, "libwg.so")
-SOURCES = ["dsm.cu", "sample.cu", "unique.cu", "gather.cu", "gather_g4.cu", "micro.cu", "spmm.cu", "exchange.cu"]
+SOURCES = ["dsm.cu", "sample.cu", "unique.cu", "gather.cu", "micro.cu", "spmm.cu", "exchange.cu"]
 HEADERS = ["wg_internal.cuh", "device_util.cuh", "hash.cuh", "scan.cuh"]
 
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")
@@ -21,11 +21,28 @@ FLAGS = ["-O3", "-lineinfo", "-std=c++17", "-Xcompiler", "-fPIC", "-Xcompiler", 
 FLAGS += os.environ.get("WG_NVCC_DEFS", "").split()
 
 
+STAMP = LIB + ".stamp"   # the nvcc command line the library was built with
+
+
+def _stamp_text(lib_path=LIB):
+    import hashlib
+    with open(lib_path, "rb") as f:
+        digest = hashlib.sha256(f.read()).hexdigest()
+    return " ".join([NVCC, *ARCH, *FLAGS, *SOURCES]) + "\n" + digest
+
+
 def _stale(target, deps):
     if not os.path.exists(target):
         return True
     t = os.path.getmtime(target)
-    return any(os.path.getmtime(d) > t for d in deps)
+    if any(os.path.getmtime(d) > t for d in deps):
+        return True
+    # a build with other flags (e.g. WG_NVCC_DEFS A/B defines) or a copied-in binary is never current
+    try:
+        with open(STAMP) as f:
+            return f.read() != _stamp_text(target)
+    except OSError:
+        return True
 
 
 def build_lib(force=False, verbose=False) -> str:
@@ -53,6 +70,8 @@ def build_lib(force=False, verbose=False) -> str:
     tmp = LIB + f".tmp{os.getpid()}"
     subprocess.check_call([NVCC, *ARCH, "-shared", "-cudart", "static", *objs, "-o", tmp])
     os.replace(tmp, LIB)
+    with open(STAMP, "w") as f:
+        f.write(_stamp_text())
     return LIB
 
 

@@ -21,7 +21,14 @@ class WgDsmDesc(ctypes.Structure):
     _fields_ = [("rank", ctypes.c_int32), ("world_size", ctypes.c_int32), ("device", ctypes.c_int32),
                 ("feat_dtype", ctypes.c_int32), ("num_nodes", ctypes.c_int64), ("local_num_edges", ctypes.c_int64),
                 ("feat_dim", ctypes.c_int64), ("max_batch_keys", ctypes.c_int64), ("allgather", ALLGATHER_FN),
-                ("ctx", ctypes.c_void_p)]
+                ("ctx", ctypes.c_void_p), ("flags", ctypes.c_uint32), ("reserved", ctypes.c_uint32)]
+
+
+# wg_dsm_desc.flags (include/wg.h)
+WG_DSM_WHOLE_ROWS = 0x1
+WG_DSM_WIDE_HASH = 0x2
+WG_DSM_PAD64 = 0x4
+WG_DSM_CSR_REPLICATED = 0x8
 
 
 class WgError(RuntimeError):
@@ -56,15 +63,20 @@ def lib():
     L.wg_dsm_chase.argtypes = [P, I32, I64, I64, P, P]
     L.wg_bucket_by_owner.argtypes = [P, P, I64, P, P, P, P, P]
     L.wg_rows_permute.argtypes = [P, P, P, I64, I64, P]
-    L.wg_spmm_mean_forward.argtypes = [P, I64, P, P, P, I64, P, P]
+    L.wg_spmm_mean_forward.argtypes = [P, I64, P, P, P, I64, I64, P, P]
     L.wg_spmm_mean_backward.argtypes = [P, I64, P, P, P, P, I64, P, I64, P]
     L.wg_device_error.argtypes = [P, P, I32]
     L.wg_dsm_reset_workspace.argtypes = [P, P]
     L.wg_dsm_set_gather_occupancy.argtypes = [P, I32]
+    L.wg_dsm_debug_set_epoch.argtypes = [P, ctypes.c_uint32]
+    L.wg_dsm_set_stage_events.argtypes = [P, P, I32]
+    L.wg_micro_random_read.argtypes = [P, I64, I32, I32, I32, P, P, P]
+    L.wg_micro_atomics.argtypes = [P, I64, I32, I32, I32, P, P, P]
     for f in ("wg_dsm_create", "wg_dsm_fork", "wg_dsm_local_view", "wg_dsm_shard_info", "wg_dsm_feat_layout",
               "wg_dsm_destroy", "wg_sample_neighbors", "wg_append_unique", "wg_sample_hop", "wg_gather", "wg_gather_rows",
               "wg_dsm_chase", "wg_spmm_mean_forward", "wg_spmm_mean_backward", "wg_bucket_by_owner", "wg_rows_permute",
-              "wg_device_error", "wg_dsm_reset_workspace", "wg_dsm_set_gather_occupancy"):
+              "wg_device_error", "wg_dsm_reset_workspace", "wg_dsm_set_gather_occupancy",
+              "wg_dsm_debug_set_epoch", "wg_micro_random_read", "wg_micro_atomics", "wg_dsm_set_stage_events"):
         getattr(L, f).restype = ctypes.c_int
     L.wg_last_error.restype = ctypes.c_char_p
     L.wg_last_error.argtypes = []
@@ -81,5 +93,5 @@ def check(status):
 
 EXPORTS = ["wg_dsm_create", "wg_dsm_fork", "wg_dsm_local_view", "wg_dsm_shard_info", "wg_dsm_feat_layout", "wg_dsm_destroy", "wg_sample_neighbors",
            "wg_append_unique", "wg_sample_hop", "wg_gather", "wg_gather_rows", "wg_dsm_chase", "wg_spmm_mean_forward",
-           "wg_spmm_mean_backward", "wg_bucket_by_owner", "wg_rows_permute", "wg_device_error", "wg_dsm_reset_workspace", "wg_dsm_set_gather_occupancy", "wg_last_error",
-           "wg_version"]
+           "wg_spmm_mean_backward", "wg_bucket_by_owner", "wg_rows_permute", "wg_device_error", "wg_dsm_reset_workspace", "wg_dsm_set_gather_occupancy",
+           "wg_dsm_debug_set_epoch", "wg_micro_random_read", "wg_micro_atomics", "wg_dsm_set_stage_events", "wg_last_error", "wg_version"]

@@ -25,15 +25,6 @@ namespace wg {
 
 static thread_local std::string g_last_error;
 
-bool pdl_enabled() {
-  static int on = -1;
-  if (on < 0) {
-    const char* e = getenv("WG_PDL");
-    on = (e && e[0] == '0') ? 0 : 1;
-  }
-  return on != 0;
-}
-
 void set_error(const std::string& msg) { g_last_error = msg; }
 wg_status fail(wg_status s, const std::string& msg) {
   g_last_error = msg;
@@ -54,13 +45,8 @@ static int64_t local_rows(int64_t n, int rank, int world) {
 // exactly that many bytes, so a body is whole lines and costs no over-fetch; the remaining
 // row % 128 bytes (the tail) live densely in a separate tail region (pitch = tail bytes), small
 // enough to stay in L2 (products-shaped: 2.45M x 16 B = 39 MB) and read with an evict_last hint.
-// Otherwise rows stay whole at a pitch rounded up to 64 B.  WG_FEAT_SPLIT=0 disables the split.
-static void feat_geometry(int64_t row_bytes, int64_t* body, int64_t* stride, int64_t* tail_pitch) {
-  static int split = -1;
-  if (split < 0) {
-    const char* e = getenv("WG_FEAT_SPLIT");
-    split = (e && e[0] == '0') ? 0 : 1;
-  }
+// Otherwise rows stay whole at a pitch rounded up to 64 B.  WG_DSM_WHOLE_ROWS disables the split.
+static void feat_geometry(int64_t row_bytes, bool split, int64_t* body, int64_t* stride, int64_t* tail_pitch) {
   const int64_t t = row_bytes % 128;
   if (split && row_bytes > 128 && t != 0 && t % 16 == 0) {
     *body = row_bytes - t;
@@ -87,6 +73,9 @@ struct PeerRecord {
   int64_t tail_pitch;
   int32_t world;
   int32_t rank;
+  uint32_t flags;
+  int32_t pad_;
+  char uuid[16];  // the rank's GPU (cudaDeviceProp::uuid): ordinals differ between processes
   cudaIpcMemHandle_t handle;
 };
 
@@ -113,20 +102,13 @@ static void free_workspace(wg_dsm* h) {
 static wg_status alloc_workspace(wg_dsm* h, int64_t max_keys) {
   Workspace& w = h->ws;
   if (max_keys < 1) max_keys = 1;
-  // Table size = WG_HASH_FACTOR (default 2) x the capacity bound (a multiple of 8 slots).  Trade-off measured on B200:
+  // Table size = HASH_FACTOR (2) x the capacity bound (a multiple of 8 slots).  Trade-off measured on B200:
   // a larger table shortens the warp-max linear-probe chains (single-batch latency), a smaller
   // one packs the touched slots into fewer DRAM lines, which matters when several batches (one
-  // table each) are in flight and compete for the 126 MB L2.
-  static double factor = 0.0;
-  if (factor == 0.0) {
-    const char* f = getenv("WG_HASH_FACTOR");
-    factor = f ? atof(f) : 2.0;
-    if (factor < 1.25) factor = 1.25;
-  }
-  int64_t cap = (int64_t)(factor * (double)max_keys) + 8;
-  cap = std::max<int64_t>(1024, (cap + 7) / 8 * 8);
+  // table each) are in flight and compete for the 126 MB L2.  Slot indices must fit int32 (slot_of).
+  int64_t cap = (int64_t)(HASH_FACTOR * (double)max_keys) + 8;
+  cap = std::min<int64_t>(std::max<int64_t>(1024, (cap + 7) / 8 * 8), HASH_MAX_SLOTS);
   w.hcap = cap;
-  w.hfactor = factor;
   w.max_keys = max_keys;
   w.status_cap = max_keys / 32 + 2;  // sampler tiles hold >= 32 targets, flag tiles 1024 positions
   if (cudaMalloc(&w.hslots, cap * sizeof(HashSlot)) != cudaSuccess ||
@@ -141,33 +123,24 @@ static wg_status alloc_workspace(wg_dsm* h, int64_t max_keys) {
     free_workspace(h);
     return fail(WG_ERR_OOM, "workspace allocation failed");
   }
-  // compact 8 B slots (hash.cuh) when node ids and positions fit 28 bits (WG_HASH_COMPACT=0: 16 B slots)
-  static int compact_ok = -1;
-  if (compact_ok < 0) {
-    const char* c = getenv("WG_HASH_COMPACT");
-    compact_ok = (c && c[0] == '0') ? 0 : 1;
-  }
-  w.compact = compact_ok && h->n <= (int64_t(1) << 28) && max_keys < (int64_t(1) << 28) ? 1 : 0;
-  static int pad32_ok = -1;
-  if (pad32_ok < 0) {
-    const char* c = getenv("WG_PAD32");
-    pad32_ok = (c && c[0] == '0') ? 0 : 1;
-  }
-  w.pad32 = pad32_ok && h->n < (int64_t(1) << 32) ? 1 : 0;
+  // compact 8 B slots (hash.cuh) when node ids and positions fit 28 bits (WG_DSM_WIDE_HASH: 16 B slots)
+  w.compact = !(h->flags & WG_DSM_WIDE_HASH) && h->n <= (int64_t(1) << 28) && max_keys < (int64_t(1) << 28) ? 1 : 0;
+  w.pad32 = !(h->flags & WG_DSM_PAD64) && h->n < (int64_t(1) << 32) ? 1 : 0;
   if (w.compact) {
     WG_CUDA_TRY(cudaMemset(w.hslots, 0, cap * sizeof(HashSlot)));  // every word stale (epoch 0)
   } else {
     WG_CUDA_TRY(cudaMemset(w.hslots, 0xff, cap * sizeof(HashSlot)));                   // val = all ones
     WG_CUDA_TRY(cudaMemset2D(w.hslots, sizeof(HashSlot), 0, sizeof(unsigned long long), cap));  // key = 0 (empty)
   }
+  // The kernels read the padded sampler slots speculatively (a key is loaded together with its
+  // slot's count and discarded for a padding slot): zero them once so no read is of never-written
+  // memory (compute-sanitizer initcheck clean).
+  WG_CUDA_TRY(cudaMemset(w.nbrs_pad, 0, max_keys * 8));
+  WG_CUDA_TRY(cudaMemset(w.pos_pad, 0, max_keys * 4));
   WG_CUDA_TRY(cudaMemset(w.status_sample, 0, w.status_cap * 8));
   WG_CUDA_TRY(cudaMemset(w.status_unique, 0, w.status_cap * 8));
   unsigned ctrl[CTRL_WORDS] = {0};
   ctrl[CTRL_EPOCH] = 1;
-  if (const char* e = getenv("WG_EPOCH_START")) {  // test hook: start near the end of the epoch space
-    const long v = atol(e);
-    if (v >= 1 && v < (long)EPOCH_MAX) ctrl[CTRL_EPOCH] = (unsigned)v;
-  }
   WG_CUDA_TRY(cudaMemcpy(w.ctrl, ctrl, sizeof(ctrl), cudaMemcpyHostToDevice));
   return WG_OK;
 }
@@ -196,36 +169,6 @@ extern "C" {
 const char* wg_last_error(void) { return g_last_error.c_str(); }
 const char* wg_version(void) { return "wholegraph-b200 0.1 (sm_100a)"; }
 
-// L2 persistence for the split layout's tail region (WG_TAIL_PERSIST, default 0 = off):
-// 1 = reserve a persisting L2 set-aside of the tail region's size (the gather's evict_last tail
-// loads may then occupy it); 2 = also attach an access-policy window over this rank's tail region
-// (hitProp persisting) to every gather launch.  The set-aside is device-wide for the process.
-static void setup_tail_persistence(wg_dsm* h) {
-  const char* e = getenv("WG_TAIL_PERSIST");
-  const int mode = e ? atoi(e) : 0;
-  const size_t tail_bytes = (size_t)(h->n_local * h->tail_pitch);
-  if (mode <= 0 || tail_bytes == 0) return;
-  int max_persist = 0, max_window = 0;
-  cudaDeviceGetAttribute(&max_persist, cudaDevAttrMaxPersistingL2CacheSize, h->device);
-  cudaDeviceGetAttribute(&max_window, cudaDevAttrMaxAccessPolicyWindowSize, h->device);
-  const size_t want = std::min(tail_bytes, (size_t)max_persist);
-  size_t cur = 0;
-  cudaDeviceGetLimit(&cur, cudaLimitPersistingL2CacheSize);
-  if (want > cur) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, want);
-  if (mode >= 2) {
-    cudaAccessPolicyWindow& w = h->tail_window;
-    w.base_ptr = const_cast<uint8_t*>(h->view.tail[h->rank]);
-    w.num_bytes = std::min(tail_bytes, (size_t)max_window);
-    w.hitRatio = std::min(1.0f, (float)want / (float)w.num_bytes);
-    w.hitProp = cudaAccessPropertyPersisting;
-    w.missProp = cudaAccessPropertyStreaming;
-  }
-  if (getenv("WG_VERBOSE"))
-    fprintf(stderr, "[wg] tail persistence mode %d: tail %zu B, set-aside %zu B (max %d), window %zu B (max %d)\n",
-            mode, tail_bytes, want, max_persist, (size_t)h->tail_window.num_bytes, max_window);
-  cudaGetLastError();
-}
-
 wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
   if (!out) return fail(WG_ERR_INVALID_ARG, "out is NULL");
   *out = nullptr;
@@ -237,6 +180,8 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
     return fail(WG_ERR_INVALID_ARG, "sizes out of range (num_nodes < 2^40, max_batch_keys < 2^31)");
   if (d->feat_dtype < WG_F32 || d->feat_dtype > WG_BF16) return fail(WG_ERR_INVALID_ARG, "feat_dtype");
   if (d->world_size > 1 && !d->allgather) return fail(WG_ERR_INVALID_ARG, "allgather callback required for W > 1");
+  if ((d->flags & ~(WG_DSM_WHOLE_ROWS | WG_DSM_WIDE_HASH | WG_DSM_PAD64 | WG_DSM_CSR_REPLICATED)) || d->reserved)
+    return fail(WG_ERR_INVALID_ARG, "unknown flags");
 
   WG_CUDA_TRY(cudaSetDevice(d->device));
   int major = 0, minor = 0, sms = 0;
@@ -253,15 +198,18 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
   h->feat_dim = d->feat_dim;
   h->elt = d->feat_dtype == WG_F32 ? 4 : 2;
   h->row_bytes = h->feat_dim * h->elt;
-  feat_geometry(h->row_bytes, &h->body_bytes, &h->feat_stride, &h->tail_pitch);
+  h->flags = d->flags;
+  feat_geometry(h->row_bytes, !(h->flags & WG_DSM_WHOLE_ROWS), &h->body_bytes, &h->feat_stride, &h->tail_pitch);
   h->allgather = d->allgather;
   h->ctx = d->ctx;
   h->sm_count = sms;
   h->n_local = local_rows(h->n, h->rank, h->world);
   h->e_local = d->local_num_edges;
 
-  // ---- this rank's slab
-  const int64_t off_col = round_up((h->n_local + 1) * 8, 256);
+  // ---- this rank's slab (the CSR part holds all n rows with WG_DSM_CSR_REPLICATED)
+  const bool csr_rep = (h->flags & WG_DSM_CSR_REPLICATED) != 0;
+  const int64_t csr_rows = csr_rep ? h->n : h->n_local;
+  const int64_t off_col = round_up((csr_rows + 1) * 8, 256);
   const int64_t off_feat = round_up(off_col + h->e_local * 8, 256);
   const int64_t off_tail = round_up(off_feat + h->n_local * h->feat_stride, 256);
   h->slab_bytes = (size_t)round_up(off_tail + h->n_local * h->tail_pitch, 256);
@@ -300,6 +248,12 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
   mine.tail_pitch = h->tail_pitch;
   mine.world = h->world;
   mine.rank = h->rank;
+  mine.flags = h->flags;
+  {
+    cudaDeviceProp prop;
+    WG_CUDA_TRY(cudaGetDeviceProperties(&prop, h->device));
+    std::memcpy(mine.uuid, prop.uuid.bytes, 16);
+  }
   PeerRecord all[WG_MAX_WORLD];
   std::memset(all, 0, sizeof(all));
   if (h->world > 1) {
@@ -317,9 +271,9 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
   }
   for (int r = 0; r < h->world; ++r) {
     if (all[r].rank != r || all[r].world != h->world || all[r].num_nodes != h->n ||
-        all[r].feat_stride != h->feat_stride || all[r].tail_pitch != h->tail_pitch) {
+        all[r].feat_stride != h->feat_stride || all[r].tail_pitch != h->tail_pitch || all[r].flags != h->flags) {
       release(h);
-      return fail(WG_ERR_INVALID_ARG, "ranks disagree on world_size / num_nodes / feat_dim");
+      return fail(WG_ERR_INVALID_ARG, "ranks disagree on world_size / num_nodes / feat_dim / flags");
     }
   }
 
@@ -332,6 +286,25 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
     } else if (all[r].pid == mine.pid) {
       h->peer_base[r] = (void*)(uintptr_t)all[r].dev_ptr;  // same process: plain device pointer
     } else {
+      // one process per GPU (L98): a peer slab on ANOTHER visible GPU needs P2P access (NVLink) from ours
+      int peer_dev = -1, ndev = 0;
+      cudaGetDeviceCount(&ndev);
+      for (int dv = 0; dv < ndev && peer_dev < 0; ++dv) {
+        cudaDeviceProp pp;
+        if (cudaGetDeviceProperties(&pp, dv) == cudaSuccess && std::memcmp(pp.uuid.bytes, all[r].uuid, 16) == 0)
+          peer_dev = dv;
+      }
+      cudaGetLastError();
+      if (peer_dev >= 0 && peer_dev != h->device) {
+        int can = 0;
+        cudaDeviceCanAccessPeer(&can, h->device, peer_dev);
+        if (!can) {
+          release(h);
+          return fail(WG_ERR_PEER_ACCESS, "device " + std::to_string(h->device) + " cannot access rank " +
+                                              std::to_string(r) + "'s device " + std::to_string(peer_dev) +
+                                              " peer-to-peer (cudaDeviceCanAccessPeer == 0)");
+        }
+      }
       void* p = nullptr;
       cudaError_t e = cudaIpcOpenMemHandle(&p, all[r].handle, cudaIpcMemLazyEnablePeerAccess);
       if (e != cudaSuccess) {
@@ -356,9 +329,9 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
   h->view.log2w = -1;
   for (int k = 0; k <= 3; ++k)
     if ((1 << k) == h->world) h->view.log2w = k;
-  setup_tail_persistence(h);
-  // Zero this rank's row_ptr sentinel so an unfilled shard reads as degree 0.
-  if (cudaMemset(h->slab, 0, (h->n_local + 1) * 8) != cudaSuccess) {
+  h->view.csr_rank = csr_rep ? h->rank : -1;
+  // Zero this rank's row_ptr so an unfilled shard reads as degree 0.
+  if (cudaMemset(h->slab, 0, (csr_rows + 1) * 8) != cudaSuccess) {
     cudaGetLastError();
     release(h);
     return fail(WG_ERR_CUDA, "memset row_ptr");
@@ -416,6 +389,7 @@ wg_status wg_dsm_fork(wg_dsm_t parent, int64_t max_batch_keys, wg_dsm_t* out) {
   *h = *parent;  // geometry, pointer table, callbacks
   h->ws = Workspace{};
   h->fork_event = nullptr;
+  h->stage_n = 0;
   h->parent = parent;
   h->live_forks = 0;
   h->excl_next = 0;
@@ -565,6 +539,22 @@ wg_status wg_dsm_reset_workspace(wg_dsm_t h, wg_stream_t stream) {
   }
   static const unsigned one = 1;
   WG_CUDA_TRY(cudaMemcpyAsync(h->ws.ctrl + CTRL_EPOCH, &one, 4, cudaMemcpyHostToDevice, st));
+  return WG_OK;
+}
+
+wg_status wg_dsm_set_stage_events(wg_dsm_t h, void* const* events, int32_t n) {
+  if (!h || n < 0 || n > 8 || (n > 0 && !events)) return fail(WG_ERR_INVALID_ARG, "bad arguments (n <= 8)");
+  for (int i = 0; i < 8; ++i) h->stage_ev[i] = i < n ? (cudaEvent_t)events[i] : nullptr;
+  h->stage_n = n;
+  h->stage_i = 0;
+  return WG_OK;
+}
+
+wg_status wg_dsm_debug_set_epoch(wg_dsm_t h, uint32_t epoch) {
+  if (!h || epoch == 0 || epoch >= EPOCH_MAX) return fail(WG_ERR_INVALID_ARG, "bad handle or epoch");
+  cudaSetDevice(h->device);
+  WG_CUDA_TRY(cudaDeviceSynchronize());
+  WG_CUDA_TRY(cudaMemcpy(h->ws.ctrl + CTRL_EPOCH, &epoch, 4, cudaMemcpyHostToDevice));
   return WG_OK;
 }
 

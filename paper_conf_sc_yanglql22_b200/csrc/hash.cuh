@@ -19,7 +19,6 @@ constexpr unsigned long long KEY_MASK = (1ull << 40) - 1;
 struct HashTable {
   HashSlot* slots;
   unsigned long long size;  // slots in use (any size: slot = high half of hash * size)
-  int cas128;               // claim with one 128-bit CAS of {key, value} (WG_HASH_CAS128)
   int compact;              // 8 B slots (below) instead of 16 B HashSlots
 };
 
@@ -90,9 +89,8 @@ __device__ __forceinline__ void cas128(HashSlot* p, unsigned long long& k, unsig
 
 // Returns the slot holding `stored` (claiming an empty one if needed), or -1 if full.
 // *seen receives the slot's value as read together with its key (one 16 B load) when the
-// key was already present, or ~0 when the value may still be stale (the caller then records
-// its position with an atomicMin).  With t.cas128 a claim writes the key together with the
-// value `mine` in one 128-bit CAS, and *seen = 0 tells the caller nothing is left to do.
+// key was already present.  A claim writes the key together with the value `mine` in one
+// 128-bit CAS, and *seen = 0 tells the caller nothing is left to do.
 __device__ __forceinline__ long long hash_insert(const HashTable& t, unsigned long long stored, unsigned epoch,
                                                  unsigned long long mine, unsigned long long* seen) {
   unsigned long long slot = __umul64hi(fmix64(stored & KEY_MASK), t.size);  // uniform in [0, size)
@@ -105,25 +103,13 @@ __device__ __forceinline__ long long hash_insert(const HashTable& t, unsigned lo
         return (long long)slot;
       }
       if ((unsigned)(cur >> 40) == epoch) break;  // occupied by another key this epoch
-      if (t.cas128) {
-        const unsigned long long ck = cur, cv = val;
-        cas128(&t.slots[slot], cur, val, stored, mine);  // cur, val <- the slot's previous contents
-        if (cur == ck && val == cv) {
-          *seen = 0;  // claimed with our position already in place
-          return (long long)slot;
-        }
-        continue;  // re-examine what is there now (our key, another key, or a newer stale pair)
-      }
-      const unsigned long long prev = atomicCAS(&t.slots[slot].key, cur, stored);
-      if (prev == cur) {
-        *seen = ~0ull;
+      const unsigned long long ck = cur, cv = val;
+      cas128(&t.slots[slot], cur, val, stored, mine);  // cur, val <- the slot's previous contents
+      if (cur == ck && val == cv) {
+        *seen = 0;  // claimed with our position already in place
         return (long long)slot;
       }
-      if (prev == stored) {
-        *seen = ~0ull;  // claimed by another thread a moment ago: its minimum may not be there yet
-        return (long long)slot;
-      }
-      cur = prev;
+      // re-examine what is there now (our key, another key, or a newer stale pair)
     }
     slot = slot + 1 == t.size ? 0 : slot + 1;
   }

@@ -55,7 +55,6 @@ struct SampleArgs {
   int32_t* pos_pad;   // [nT * M]
   int32_t* cnt;       // [nT]
   unsigned* ctrl;
-  int rp_keep;        // 1: row_ptr loads carry an L2 evict_last hint (WG_RP_EVICT_LAST)
   unsigned long long* hclear;  // fused hop, compact hash table: zeroed here when its epoch cycle restarts
   int pad32;                   // padded neighbour slots hold uint32 ids (num_nodes < 2^32)
   int64_t hwords;
@@ -67,17 +66,6 @@ __device__ __noinline__ void clear_table_if_cycle_restarts(unsigned long long* w
   if (compact_epoch(ctrl[CTRL_EPOCH]) != 1u) return;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < words; i += stride) w[i] = 0ull;
-}
-
-// row_ptr is read by every target of every batch (2.45M x 8 B = 20 MB for products): an
-// evict_last hint asks L2 to keep it over the streaming gather bytes.
-__device__ __forceinline__ int64_t ld_rp(const int64_t* p, int keep) {
-  if (!keep) return *p;
-  unsigned long long pol;
-  asm("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(pol));
-  long long v;
-  asm volatile("ld.global.nc.L2::cache_hint.s64 %0, [%1], %2;" : "=l"(v) : "l"(p), "l"(pol));
-  return v;
 }
 
 template <int SAMPLE_UNR, bool CLR>
@@ -115,10 +103,10 @@ __global__ void __launch_bounds__(SAMPLE_THREADS, SAMPLE_MINB) sample_kernel(con
       } else {
         int o;
         int64_t l;
-        owner_local(a.s, my_v, o, l);
+        csr_owner_local(a.s, my_v, o, l);
         const int64_t* rp = a.s.row_ptr[o] + l;
-        my_start = ld_rp(rp, a.rp_keep);
-        const int64_t d = ld_rp(rp + 1, a.rp_keep) - my_start;
+        my_start = rp[0];
+        const int64_t d = rp[1] - my_start;
         if (d >= (int64_t(1) << 32) || d < 0)
           latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DEGREE);
         else
@@ -171,7 +159,7 @@ __global__ void __launch_bounds__(SAMPLE_THREADS, SAMPLE_MINB) sample_kernel(con
     ok[u] = active && (full ? (unsigned)i < N : i < M);
     int o = 0;
     int64_t l;
-    if (ok[u]) owner_local(a.s, tv, o, l);
+    if (ok[u]) csr_owner_local(a.s, tv, o, l);
     src[u] = a.s.col[o] + tstart + pos[u];
     dst[u] = k * M + i;
     if (i == 0 && g < TPW && k < nT) a.cnt[k] = active ? (int32_t)min(N, (unsigned)M) : 0;
@@ -220,7 +208,7 @@ __global__ void __launch_bounds__(BT) sample_block_kernel(const SampleArgs a) {
     } else {
       int o;
       int64_t l;
-      owner_local(a.s, v, o, l);
+      csr_owner_local(a.s, v, o, l);
       const int64_t* rp = a.s.row_ptr[o] + l;
       start = rp[0];
       const int64_t d = rp[1] - start;
@@ -240,7 +228,7 @@ __global__ void __launch_bounds__(BT) sample_block_kernel(const SampleArgs a) {
   const unsigned N = s_n;
   int o;
   int64_t l;
-  owner_local(a.s, v, o, l);
+  csr_owner_local(a.s, v, o, l);
   const int64_t* col = a.s.col[o] + s_start;
   if (N <= (unsigned)M) {  // L118: all of N neighbours, CSR order (A5)
     for (unsigned j = i; j < N; j += BT) {
@@ -403,12 +391,6 @@ cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap,
   a.ctrl = h->ws.ctrl;
   a.hclear = h->ws.compact ? reinterpret_cast<unsigned long long*>(h->ws.hslots) : nullptr;
   a.hwords = h->ws.hcap;
-  static int rp_keep = -1;
-  if (rp_keep < 0) {
-    const char* e = getenv("WG_RP_EVICT_LAST");
-    rp_keep = (e && e[0] == '1') ? 1 : 0;
-  }
-  a.rp_keep = rp_keep;
   if (fanout > 32) {  // block per target (Algorithm 1 with a block sort)
     const unsigned blocks = (unsigned)(cap > 0 ? cap : 1);
     if (a.hclear) return launch_block_sampler<true>(fanout, blocks, a, st);
@@ -416,13 +398,7 @@ cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap,
   }
   const int G = sample_group(fanout);
   const int tpw = 32 / G;
-  static int unr_max = -1;  // A/B knob WG_SAMPLE_UNR_MAX (4, 2 or 1)
-  if (unr_max < 0) {
-    const char* e = getenv("WG_SAMPLE_UNR_MAX");
-    unr_max = e ? std::max(1, std::min(4, atoi(e))) : 4;
-    if (unr_max == 3) unr_max = 2;
-  }
-  int unr = unr_max;  // largest of 4/2/1 that still gives >= 2 blocks per SM
+  int unr = SAMPLE_UNR_MAX;  // largest of 4/2/1 that still gives >= 2 blocks per SM
   while (unr > 1 && cap < (int64_t)(SAMPLE_THREADS / 32) * tpw * unr * 2 * h->sm_count) unr >>= 1;
   const int64_t tile = (int64_t)(SAMPLE_THREADS / 32) * tpw * unr;
   const unsigned blocks = (unsigned)(cap > 0 ? (cap + tile - 1) / tile : 1);

@@ -24,9 +24,11 @@ __device__ __forceinline__ int64_t count_or_cap(const int64_t* d, int64_t cap) {
 }
 
 // D4 = feature columns / 4 (float4 slices per row)
+// Edges whose column lies outside [0, n_x) (e.g. the -1 a relabel writes for an invalid id after
+// WG_DEVERR_ID_RANGE) are skipped in both directions: no out-of-bounds read or write.
 __global__ void __launch_bounds__(SPMM_THREADS) spmm_mean_fwd_kernel(const int64_t* row_ptr, int64_t cap_rows,
                                                                      const int64_t* d_rows, const int32_t* col,
-                                                                     const float4* X, int D4, float4* Y) {
+                                                                     const float4* X, int64_t n_x, int D4, float4* Y) {
   const int64_t n = count_or_cap(d_rows, cap_rows);
   const int lane = threadIdx.x & 31;
   const int64_t warps = (int64_t)gridDim.x * (SPMM_THREADS / 32);
@@ -36,7 +38,9 @@ __global__ void __launch_bounds__(SPMM_THREADS) spmm_mean_fwd_kernel(const int64
     for (int c = lane; c < D4; c += 32) {
       float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
       for (int64_t k = b; k < e; ++k) {
-        const float4 x = __ldg(&X[(int64_t)col[k] * D4 + c]);
+        const int64_t r = col[k];
+        if (r < 0 || r >= n_x) continue;
+        const float4 x = __ldg(&X[r * D4 + c]);
         acc.x += x.x;
         acc.y += x.y;
         acc.z += x.z;
@@ -50,7 +54,7 @@ __global__ void __launch_bounds__(SPMM_THREADS) spmm_mean_fwd_kernel(const int64
 __global__ void __launch_bounds__(SPMM_THREADS) spmm_mean_bwd_kernel(const int64_t* row_ptr, int64_t cap_rows,
                                                                      const int64_t* d_rows, const int32_t* col,
                                                                      const int32_t* dup, const float4* dY, int D4,
-                                                                     float4* dX) {
+                                                                     float4* dX, int64_t n_x) {
   const int64_t n = count_or_cap(d_rows, cap_rows);
   const int lane = threadIdx.x & 31;
   const int64_t warps = (int64_t)gridDim.x * (SPMM_THREADS / 32);
@@ -63,6 +67,7 @@ __global__ void __launch_bounds__(SPMM_THREADS) spmm_mean_bwd_kernel(const int64
       g = make_float4(g.x * inv, g.y * inv, g.z * inv, g.w * inv);
       for (int64_t k = b; k < e; ++k) {
         const int64_t r = col[k];
+        if (r < 0 || r >= n_x) continue;
         if (dup && dup[r] == 1)
           dX[r * D4 + c] = g;  // the only contribution this row receives
         else
@@ -79,9 +84,9 @@ using namespace wg;
 extern "C" {
 
 wg_status wg_spmm_mean_forward(const int64_t* d_row_ptr, int64_t n_rows, const int64_t* d_n_rows,
-                               const int32_t* d_sub_col, const float* d_x, int64_t dim, float* d_y,
+                               const int32_t* d_sub_col, const float* d_x, int64_t n_x_rows, int64_t dim, float* d_y,
                                wg_stream_t stream) {
-  if (n_rows < 0 || dim <= 0 || dim % 4 != 0 || (n_rows > 0 && (!d_row_ptr || !d_sub_col || !d_x || !d_y)))
+  if (n_rows < 0 || n_x_rows < 0 || dim <= 0 || dim % 4 != 0 || (n_rows > 0 && (!d_row_ptr || !d_sub_col || !d_x || !d_y)))
     return fail(WG_ERR_INVALID_ARG, "bad arguments (dim must be a positive multiple of 4)");
   if (n_rows == 0) return WG_OK;
   int dev = 0, sms = 148;
@@ -90,7 +95,7 @@ wg_status wg_spmm_mean_forward(const int64_t* d_row_ptr, int64_t n_rows, const i
   int64_t blocks = (n_rows * 32 + SPMM_THREADS - 1) / SPMM_THREADS;
   blocks = blocks > (int64_t)sms * 8 ? (int64_t)sms * 8 : blocks;
   spmm_mean_fwd_kernel<<<(unsigned)blocks, SPMM_THREADS, 0, (cudaStream_t)stream>>>(
-      d_row_ptr, n_rows, d_n_rows, d_sub_col, reinterpret_cast<const float4*>(d_x), (int)(dim / 4),
+      d_row_ptr, n_rows, d_n_rows, d_sub_col, reinterpret_cast<const float4*>(d_x), n_x_rows, (int)(dim / 4),
       reinterpret_cast<float4*>(d_y));
   cudaError_t e = cudaGetLastError();
   return e == cudaSuccess ? WG_OK : fail(WG_ERR_CUDA, cudaGetErrorString(e));
@@ -113,7 +118,7 @@ wg_status wg_spmm_mean_backward(const int64_t* d_row_ptr, int64_t n_rows, const 
   blocks = blocks > (int64_t)sms * 8 ? (int64_t)sms * 8 : blocks;
   spmm_mean_bwd_kernel<<<(unsigned)blocks, SPMM_THREADS, 0, st>>>(
       d_row_ptr, n_rows, d_n_rows, d_sub_col, d_dup_count, reinterpret_cast<const float4*>(d_dy), (int)(dim / 4),
-      reinterpret_cast<float4*>(d_dx));
+      reinterpret_cast<float4*>(d_dx), n_x_rows);
   e = cudaGetLastError();
   return e == cudaSuccess ? WG_OK : fail(WG_ERR_CUDA, cudaGetErrorString(e));
 }

@@ -42,6 +42,8 @@ constexpr int UQ_THREADS = WG_UQ_THREADS;
 // neighbour positions per thread of the flag scan: 1..8, chosen per launch so that small hops
 // spread over many SMs (latency-bound) and large hops keep several loads in flight per thread
 constexpr int CNT_BITS = 31;                    // packed scan value: (valid << 31) | first
+constexpr int PREP_BPS = 8;                     // insert / relabel blocks per SM (full occupancy)
+constexpr int FLAG_ITEMS_MAX = 8;               // most positions per thread of the flag scan
 constexpr int32_t SLOT_EMPTY = -1;              // slot_of: padded slot without a sample
 constexpr int32_t SLOT_BADID = -2;              // slot_of: sample whose id is out of range
 
@@ -301,12 +303,13 @@ __global__ void __launch_bounds__(256) hash_clear_kernel(unsigned long long* w, 
 }
 
 template <bool C>
-static cudaError_t launch_insert_flag(bool padded, int items, int64_t ib, unsigned fb, const UniqueArgs& a,
+static cudaError_t launch_insert_flag(wg_dsm* h, bool padded, int items, int64_t ib, unsigned fb, const UniqueArgs& a,
                                       cudaStream_t st) {
-  cudaError_t e;
+  cudaError_t e = padded ? launch_pdl(unique_insert_kernel<true, C>, (unsigned)ib, UQ_THREADS, 0, st, a)
+                         : launch_pdl(unique_insert_kernel<false, C>, (unsigned)ib, UQ_THREADS, 0, st, a);
+  if (e != cudaSuccess) return e;
+  stage_mark(h, st);
   if (padded) {
-    e = launch_pdl(unique_insert_kernel<true, C>, (unsigned)ib, UQ_THREADS, 0, st, a);
-    if (e != cudaSuccess) return e;
     switch (items) {
       case 8: return launch_pdl(unique_flag_kernel<true, 8, C>, fb, UQ_THREADS, 0, st, a);
       case 4: return launch_pdl(unique_flag_kernel<true, 4, C>, fb, UQ_THREADS, 0, st, a);
@@ -314,8 +317,6 @@ static cudaError_t launch_insert_flag(bool padded, int items, int64_t ib, unsign
       default: return launch_pdl(unique_flag_kernel<true, 1, C>, fb, UQ_THREADS, 0, st, a);
     }
   }
-  e = launch_pdl(unique_insert_kernel<false, C>, (unsigned)ib, UQ_THREADS, 0, st, a);
-  if (e != cudaSuccess) return e;
   switch (items) {
     case 8: return launch_pdl(unique_flag_kernel<false, 8, C>, fb, UQ_THREADS, 0, st, a);
     case 4: return launch_pdl(unique_flag_kernel<false, 4, C>, fb, UQ_THREADS, 0, st, a);
@@ -328,51 +329,24 @@ static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, c
   a.excl = h->ws.excl[h->excl_next];
   h->excl_next = (h->excl_next + 1) % EXCL_RING;
   a.slot_of = h->ws.slot_of;
-  // Each call uses only a prefix of the table sized for ITS key bound (capT + capE): factor x bound
-  // slots (any size, a multiple of 8 = one 128 B line; at least WG_HASH_MIN_SLOTS), so a hop touches
+  // Each call uses only a prefix of the table sized for ITS key bound (capT + capE): HASH_FACTOR x bound
+  // slots (any size, a multiple of 8 = one 128 B line; at least HASH_MIN_SLOTS), so a hop touches
   // about as many lines as it has keys instead of random lines all over the table sized for the
   // largest hop.  Slots outside the prefix, or left by earlier calls, carry older epochs and read as
-  // empty.  WG_HASH_PER_CALL=0 uses the whole table for every call (A/B).
-  static int per_call = -1;
-  static int64_t min_slots = 0;
-  if (per_call < 0) {
-    const char* e = getenv("WG_HASH_PER_CALL");
-    per_call = (e && e[0] == '0') ? 0 : 1;
-    const char* m = getenv("WG_HASH_MIN_SLOTS");
-    min_slots = m ? atoll(m) : (int64_t(1) << 20);
-  }
-  int64_t hc = h->ws.hcap;
-  if (per_call) {
-    hc = (int64_t)(h->ws.hfactor * (double)(a.capT + a.capE)) + 8;
-    hc = std::max<int64_t>(hc, min_slots);
-    hc = std::min<int64_t>((hc + 7) / 8 * 8, h->ws.hcap);
-  }
-  static int cas128 = -1;
-  if (cas128 < 0) {
-    const char* e = getenv("WG_HASH_CAS128");
-    cas128 = (e && e[0] == '0') ? 0 : 1;
-  }
-  a.ht = HashTable{h->ws.hslots, (unsigned long long)hc, cas128, h->ws.compact};
+  // empty.
+  int64_t hc = (int64_t)(HASH_FACTOR * (double)(a.capT + a.capE)) + 8;
+  hc = std::max<int64_t>(hc, HASH_MIN_SLOTS);
+  hc = std::min<int64_t>((hc + 7) / 8 * 8, h->ws.hcap);
+  a.ht = HashTable{h->ws.hslots, (unsigned long long)hc, h->ws.compact};
   a.status = h->ws.status_unique;
   a.ctrl = h->ws.ctrl;
   a.n = h->n;
   const int64_t total = a.capT + a.capE;
-  static int prep_bps = -1;  // A/B knob WG_PREP_BPS: insert / relabel blocks per SM (default 8 = full occupancy)
-  if (prep_bps < 0) {
-    const char* e = getenv("WG_PREP_BPS");
-    prep_bps = (e && atoi(e) > 0) ? atoi(e) : 8;
-  }
-  const int64_t max_blocks = (int64_t)h->sm_count * prep_bps;
+  const int64_t max_blocks = (int64_t)h->sm_count * PREP_BPS;
   int64_t ib = (total + UQ_THREADS - 1) / UQ_THREADS;
   ib = ib < 1 ? 1 : (ib > max_blocks ? max_blocks : ib);
   // items per thread: the largest of 8/4/2/1 that still gives >= 2 tiles per SM
-  static int items_max = -1;  // A/B knob WG_FLAG_ITEMS_MAX (8, 4, 2 or 1)
-  if (items_max < 0) {
-    const char* e = getenv("WG_FLAG_ITEMS_MAX");
-    const int v = e ? atoi(e) : 8;
-    items_max = v >= 8 ? 8 : v >= 4 ? 4 : v >= 2 ? 2 : 1;
-  }
-  int items = items_max;
+  int items = FLAG_ITEMS_MAX;
   while (items > 1 && a.capE < (int64_t)items * UQ_THREADS * 2 * h->sm_count) items >>= 1;
   const int64_t tile = (int64_t)items * UQ_THREADS;
   const unsigned fb = (unsigned)(a.capE > 0 ? (a.capE + tile - 1) / tile : 1);
@@ -383,10 +357,11 @@ static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, c
     if (e != cudaSuccess) return e;
   }
   if (h->ws.compact)
-    e = launch_insert_flag<true>(padded, items, ib, fb, a, st);
+    e = launch_insert_flag<true>(h, padded, items, ib, fb, a, st);
   else
-    e = launch_insert_flag<false>(padded, items, ib, fb, a, st);
+    e = launch_insert_flag<false>(h, padded, items, ib, fb, a, st);
   if (e != cudaSuccess) return e;
+  stage_mark(h, st);
   if (a.capE > 0) {
     // relabel runs over the DENSE neighbours: count = num_edges (padded) or d_nE
     UniqueArgs r = a;
@@ -402,6 +377,7 @@ static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, c
       rs = side;
     }
     unique_relabel_kernel<<<(unsigned)rb, UQ_THREADS, 0, rs>>>(r);
+    stage_mark(h, rs);
   }
   return cudaGetLastError();
 }
@@ -422,6 +398,7 @@ cudaError_t launch_append_unique(wg_dsm* h, const int64_t* T, int64_t capT, cons
   a.d_nU = d_nU;
   a.sub_col = sub_col;
   a.dup = dup;
+  h->stage_i = 0;
   return launch_unique_passes(h, a, false, st, nullptr);
 }
 
@@ -432,8 +409,10 @@ cudaError_t launch_hop(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t*
                        const uint64_t* d_seed, int hop, int64_t* out_row_ptr, int64_t* out_nbrs, int32_t* out_pos,
                        int64_t* d_num_edges, int64_t* U, int64_t* d_nU, int32_t* sub_col, int32_t* dup,
                        cudaStream_t st, cudaStream_t side) {
+  h->stage_i = 0;
   cudaError_t e = launch_sample_padded(h, T, capT, d_nT, fanout, seed, d_seed, hop, out_pos != nullptr, st);
   if (e != cudaSuccess) return e;
+  stage_mark(h, st);
   UniqueArgs a{};
   a.T = T;
   a.capT = capT;

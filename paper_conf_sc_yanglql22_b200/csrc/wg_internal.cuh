@@ -35,8 +35,11 @@ struct ShardView {
   int64_t body_bytes;   // bytes of a row stored in feat (= row bytes when not split)
   int32_t world;
   int32_t log2w;        // log2(world) if world is a power of two, else -1
+  int32_t csr_rank;     // WG_DSM_CSR_REPLICATED: this rank, whose slab holds the whole CSR; -1: CSR row-sharded
 };
 
+// Owner rank and local row of node v in the feature table (hash partition o(v) = v mod W,
+// l(v) = v div W; A11).
 __device__ __forceinline__ void owner_local(const ShardView& s, int64_t v, int& o, int64_t& l) {
   if (s.log2w >= 0) {
     o = (int)(v & (int64_t)(s.world - 1));
@@ -44,6 +47,16 @@ __device__ __forceinline__ void owner_local(const ShardView& s, int64_t v, int& 
   } else {
     o = (int)(v % s.world);
     l = v / s.world;
+  }
+}
+// Where v's CSR row lives: with the paper's placement next to its feature row ("edges are stored
+// together with the source node", L110); with WG_DSM_CSR_REPLICATED in this rank's own full copy.
+__device__ __forceinline__ void csr_owner_local(const ShardView& s, int64_t v, int& o, int64_t& l) {
+  if (s.csr_rank >= 0) {
+    o = s.csr_rank;
+    l = v;
+  } else {
+    owner_local(s, v, o, l);
   }
 }
 
@@ -58,8 +71,7 @@ struct __align__(16) HashSlot {
 };
 struct Workspace {
   HashSlot* hslots = nullptr;            // [hcap] append-unique hash table (hash.cuh)
-  int64_t hcap = 0;                      // slots (a multiple of 8); each call uses a prefix
-  double hfactor = 2.0;                  // slots per key bound (WG_HASH_FACTOR)
+  int64_t hcap = 0;                      // slots (a multiple of 8, < 2^31); each call uses a prefix
   int compact = 0;                       // 8 B slots {epoch8, key28, pos28} (hash.cuh), else 16 B slots
   int pad32 = 0;                         // padded sampler slots hold uint32 ids (num_nodes < 2^32)
   unsigned long long* status_sample = nullptr;  // decoupled look-back tile status
@@ -81,6 +93,11 @@ constexpr unsigned EPOCH_MAX = (1u << 23) - 1;
 constexpr unsigned CEPOCHS = 255;
 __host__ __device__ inline unsigned compact_epoch(unsigned e) { return e % CEPOCHS + 1u; }
 constexpr int EXCL_RING = 4;
+// Hash-table sizing (measured on B200): a call uses a prefix of
+// HASH_FACTOR x its own key bound slots (at least HASH_MIN_SLOTS), so small hops touch few lines.
+constexpr double HASH_FACTOR = 2.0;
+constexpr int64_t HASH_MIN_SLOTS = int64_t(1) << 20;
+constexpr int64_t HASH_MAX_SLOTS = (int64_t(1) << 31) - 8;  // slot indices are stored as int32 (slot_of)
 
 }  // namespace wg
 
@@ -105,41 +122,36 @@ struct wg_dsm {
   wg_dsm* parent = nullptr;             // set for a workspace fork (wg_dsm_fork): shards are the parent's
   int live_forks = 0;                   // forks of this handle not yet destroyed
   int gather_bps = 0;                   // wg_dsm_set_gather_occupancy (0 = occupancy maximum)
-  // L2 persistence of the split layout's tail region (WG_TAIL_PERSIST, see dsm.cu): the access-policy
-  // window attached to gather launches (num_bytes = 0: none)
-  cudaAccessPolicyWindow tail_window{};
+  uint32_t flags = 0;                   // wg_dsm_desc.flags
+  // wg_dsm_set_stage_events: events recorded after each kernel of an op (diagnostics, eager launches)
+  cudaEvent_t stage_ev[8] = {nullptr};
+  int stage_n = 0, stage_i = 0;
 };
 
 namespace wg {
 // Programmatic dependent launch (sm_90+): kernels of one op chain are launched with
 // ProgrammaticStreamSerialization, start their blocks while the previous kernel drains and
-// wait for its results with griddepcontrol.wait (pdl_wait) before touching memory.
-// WG_PDL=0 disables it (A/B switch); correctness never depends on it.
-bool pdl_enabled();
+// wait for its results with griddepcontrol.wait (pdl_wait) before touching memory
+// (correctness never depends on it: a kernel launched without the attribute waits anyway).
 template <typename... KArgs, typename... Args>
-inline cudaError_t launch_pdl_w(const cudaAccessPolicyWindow* win, void (*kernel)(KArgs...), dim3 grid, dim3 block,
-                                size_t smem, cudaStream_t st, Args... args) {
+inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
+                              Args... args) {
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = grid;
   cfg.blockDim = block;
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
-  cudaLaunchAttribute attr[2];
+  cudaLaunchAttribute attr[1];
   attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
-  attr[0].val.programmaticStreamSerializationAllowed = pdl_enabled() ? 1 : 0;
+  attr[0].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = 1;
-  if (win && win->num_bytes) {  // L2 access-policy window (persisting lines) for this launch
-    attr[1].id = cudaLaunchAttributeAccessPolicyWindow;
-    attr[1].val.accessPolicyWindow = *win;
-    cfg.numAttrs = 2;
-  }
   return cudaLaunchKernelEx(&cfg, kernel, static_cast<KArgs>(args)...);
 }
-template <typename... KArgs, typename... Args>
-inline cudaError_t launch_pdl(void (*kernel)(KArgs...), dim3 grid, dim3 block, size_t smem, cudaStream_t st,
-                              Args... args) {
-  return launch_pdl_w(nullptr, kernel, grid, block, smem, st, args...);
+
+// Record the next stage event (if any are set) on st, after the kernel just enqueued there.
+inline void stage_mark(wg_dsm* h, cudaStream_t st) {
+  if (h->stage_i < h->stage_n) cudaEventRecord(h->stage_ev[h->stage_i++], st);
 }
 
 // padded sampler slots: int64 ids, or uint32 ids when every id fits (half the bytes)
@@ -164,8 +176,6 @@ cudaError_t launch_hop(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t*
                        const uint64_t* d_seed, int hop, int64_t* out_row_ptr, int64_t* out_nbrs, int32_t* out_pos,
                        int64_t* d_num_edges, int64_t* U, int64_t* d_nU, int32_t* sub_col, int32_t* dup,
                        cudaStream_t st, cudaStream_t side);
-cudaError_t launch_gather_g4(wg_dsm* h, const int64_t* ids, int64_t cap, const int64_t* d_n, const int64_t* d_begin,
-                             void* out, int64_t cw, cudaStream_t st);
 cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int64_t* d_n, const int64_t* d_begin,
                           void* out, int64_t out_pitch, cudaStream_t st);
 }  // namespace wg

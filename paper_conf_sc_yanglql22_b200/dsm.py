@@ -105,7 +105,7 @@ class DSM:
     its feature table.  Collective create/destroy."""
 
     def __init__(self, num_nodes, local_num_edges, feat_dim=0, feat_dtype="fp32", max_batch_keys=1 << 20,
-                 rank=0, world_size=1, device=None, allgather=None):
+                 rank=0, world_size=1, device=None, allgather=None, flags=0):
         if device is None:
             device = torch.cuda.current_device()
         self.device = torch.device("cuda", device) if isinstance(device, int) else torch.device(device)
@@ -113,10 +113,14 @@ class DSM:
         self.num_nodes, self.feat_dim, self.feat_dtype = num_nodes, feat_dim, feat_dtype
         self.row_bytes = feat_dim * DTYPE_BYTES[feat_dtype]
         self.max_batch_keys = max_batch_keys
+        self.flags = int(flags)
+        # WG_DSM_CSR_REPLICATED: this rank's slab holds the whole CSR (all num_nodes rows)
+        self.csr_replicated = bool(self.flags & _lib.WG_DSM_CSR_REPLICATED)
         self._cb = _lib.ALLGATHER_FN(allgather) if allgather is not None else _lib.ALLGATHER_FN()
         d = _lib.WgDsmDesc(rank=rank, world_size=world_size, device=self.device.index, feat_dtype=DTYPE_CODE[feat_dtype],
                            num_nodes=num_nodes, local_num_edges=local_num_edges, feat_dim=feat_dim,
-                           max_batch_keys=max_batch_keys, allgather=self._cb, ctx=None)
+                           max_batch_keys=max_batch_keys, allgather=self._cb, ctx=None,
+                           flags=self.flags, reserved=0)
         h = ctypes.c_void_p()
         check(lib().wg_dsm_create(ctypes.byref(d), ctypes.byref(h)))
         self.h = h
@@ -135,7 +139,8 @@ class DSM:
                                       ctypes.byref(nl), ctypes.byref(stride)))
         n_local = nl.value
         _, e_local = self.shard_info(self.rank)
-        row_ptr = device_view(rp.value, (n_local + 1,), torch.int64, self.device)
+        csr_rows = self.num_nodes if self.csr_replicated else n_local
+        row_ptr = device_view(rp.value, (csr_rows + 1,), torch.int64, self.device)
         colv = device_view(col.value, (e_local,), torch.int64, self.device)
         featv = device_view(feat.value, (n_local, stride.value), torch.uint8, self.device) if self.row_bytes else None
         return row_ptr, colv, featv
@@ -188,6 +193,16 @@ class DSM:
 
     def reset_workspace(self, stream=None):
         check(lib().wg_dsm_reset_workspace(self.h, _stream(stream)))
+
+    def set_stage_events(self, events):
+        """Diagnostics: record these torch.cuda.Events after each kernel of the next ops
+        (wg_dsm_set_stage_events); [] clears.  The events must have been recorded once (created)."""
+        arr = (ctypes.c_void_p * max(len(events), 1))(*[e.cuda_event for e in events])
+        check(lib().wg_dsm_set_stage_events(self.h, arr, len(events)))
+
+    def debug_set_epoch(self, epoch):
+        """Test hook: set the workspace's hash-table epoch (wg_dsm_debug_set_epoch)."""
+        check(lib().wg_dsm_debug_set_epoch(self.h, int(epoch)))
 
     def destroy(self):
         if self.h is not None and self.h.value:
@@ -303,8 +318,12 @@ class DSM:
 
     # --- filling helpers (setup; not on the hot path) ----------------------------
     def fill_from_global_csr(self, row_ptr, col):
-        """Copy THIS rank's rows (v = rank, rank+W, ...) of a host CSR into its shard."""
-        lrp, lcol = shard_csr(row_ptr, col, self.rank, self.world)
+        """Copy THIS rank's rows (v = rank, rank+W, ...) of a host CSR into its shard (every row
+        with WG_DSM_CSR_REPLICATED)."""
+        if self.csr_replicated:
+            lrp, lcol = np.asarray(row_ptr, dtype=np.int64), np.asarray(col, dtype=np.int64)
+        else:
+            lrp, lcol = shard_csr(row_ptr, col, self.rank, self.world)
         rp, cv, _ = self.local_view()
         rp.copy_(torch.from_numpy(lrp))
         if len(lcol):

@@ -20,9 +20,11 @@ def _s():
 def spmm_mean_forward(row_ptr, sub_col, x, n_rows=None, n_rows_dev=None):
     """Y[t] = mean of x[sub_col[e]] over row t's edges.  x: float32 [*, D], D % 4 == 0."""
     n = row_ptr.numel() - 1 if n_rows is None else n_rows
-    y = torch.empty((n, x.shape[1]), dtype=torch.float32, device=x.device)
-    check(lib().wg_spmm_mean_forward(_p(row_ptr), n, _p(n_rows_dev), _p(sub_col), _p(x.contiguous()), x.shape[1],
-                                     _p(y), _s()))
+    # with a device row count the kernel writes only rows below it: the rest read as 0
+    alloc = torch.empty if n_rows_dev is None else torch.zeros
+    y = alloc((n, x.shape[1]), dtype=torch.float32, device=x.device)
+    check(lib().wg_spmm_mean_forward(_p(row_ptr), n, _p(n_rows_dev), _p(sub_col), _p(x.contiguous()), x.shape[0],
+                                     x.shape[1], _p(y), _s()))
     return y
 
 
@@ -36,15 +38,17 @@ def spmm_mean_backward(row_ptr, sub_col, dup, dy, n_x_rows, n_rows=None, n_rows_
 
 class SpMMMean(torch.autograd.Function):
     """autograd wrapper: forward = g-SpMM mean on the CSR, backward = atomics on the same
-    CSR with the duplicate-count store fast path."""
+    CSR with the duplicate-count store fast path.  ``row_ptr`` may be a pipeline's untrimmed
+    [capacity + 1] buffer when ``n_rows_dev`` (the device row count, e.g. the previous hop's
+    num_unique) is given: rows past it are left untouched (zero in the output)."""
 
     @staticmethod
-    def forward(ctx, x, row_ptr, sub_col, dup):
-        ctx.save_for_backward(row_ptr, sub_col, dup)
+    def forward(ctx, x, row_ptr, sub_col, dup, n_rows_dev=None):
+        ctx.save_for_backward(row_ptr, sub_col, dup, n_rows_dev)
         ctx.n_x = x.shape[0]
-        return spmm_mean_forward(row_ptr, sub_col, x)
+        return spmm_mean_forward(row_ptr, sub_col, x, n_rows_dev=n_rows_dev)
 
     @staticmethod
     def backward(ctx, dy):
-        row_ptr, sub_col, dup = ctx.saved_tensors
-        return spmm_mean_backward(row_ptr, sub_col, dup, dy, ctx.n_x), None, None, None
+        row_ptr, sub_col, dup, n_rows_dev = ctx.saved_tensors
+        return spmm_mean_backward(row_ptr, sub_col, dup, dy, ctx.n_x, n_rows_dev=n_rows_dev), None, None, None, None

@@ -19,8 +19,12 @@ from .pipeline import required_keys
 
 
 def build_dsm(preset, rank=0, world=1, device=None, allgather=None, max_seeds=None, on_device=None,
-              feat_dim=None, feat_dtype=None, extra_keys=0):
-    """Create and fill a DSM for ``preset`` (a synth.presets.Preset).  Returns (dsm, info)."""
+              feat_dim=None, feat_dtype=None, extra_keys=0, flags=0):
+    """Create and fill a DSM for ``preset`` (a synth.presets.Preset).  Returns (dsm, info).
+    ``flags``: wg_dsm_desc.flags (e.g. WG_DSM_CSR_REPLICATED: every rank holds the whole CSR)."""
+    from ._lib import WG_DSM_CSR_REPLICATED
+    csr_rep = bool(flags & WG_DSM_CSR_REPLICATED)
+    c_rank, c_world = (0, 1) if csr_rep else (rank, world)   # which CSR rows this rank's slab holds
     device = torch.device("cuda", torch.cuda.current_device() if device is None else device)
     spec = preset.graph()
     fd = preset.feat_dim if feat_dim is None else feat_dim
@@ -32,16 +36,17 @@ def build_dsm(preset, rank=0, world=1, device=None, allgather=None, max_seeds=No
     t0 = time.perf_counter()
     if on_device:
         from synth import gpu as sgpu
-        rp, col = sgpu.shard_csr_gpu(spec, rank, world, device)
+        rp, col = sgpu.shard_csr_gpu(spec, c_rank, c_world, device)
         e_local = col.numel()
     else:
         g_rp, g_col = sgraph.csr(spec)
-        e_local = local_num_edges(g_rp, rank, world)
+        e_local = local_num_edges(g_rp, c_rank, c_world)
     info["gen_s"] = time.perf_counter() - t0
     if on_device:
         torch.cuda.empty_cache()  # return the generator's temporaries to the driver before the big slab
     t1 = time.perf_counter()
-    dsm = DSM(spec.n, e_local, fd, fdt, keys, rank=rank, world_size=world, device=device.index, allgather=allgather)
+    dsm = DSM(spec.n, e_local, fd, fdt, keys, rank=rank, world_size=world, device=device.index, allgather=allgather,
+              flags=flags)
     torch.cuda.synchronize(device)
     info["create_s"] = time.perf_counter() - t1
     if on_device:
@@ -64,29 +69,3 @@ def build_dsm(preset, rank=0, world=1, device=None, allgather=None, max_seeds=No
     info["e_local"] = e_local
     info["fill_s"] = time.perf_counter() - t0 - info["gen_s"] - info["create_s"]
     return dsm, info
-
-
-def host_row_provider(spec, row_ptr=None, col=None):
-    """Adjacency rows for the oracle: slices of a host CSR if given, else regenerated
-    per node from the generator (any n)."""
-    if row_ptr is not None:
-        def rows(T):
-            T = np.asarray(T, dtype=np.int64)
-            starts, ends = row_ptr[T], row_ptr[T + 1]
-            lens = ends - starts
-            ptr = np.zeros(len(T) + 1, dtype=np.int64)
-            ptr[1:] = np.cumsum(lens)
-            idx = np.repeat(starts - ptr[:-1], lens) + np.arange(ptr[-1], dtype=np.int64)
-            return ptr, col[idx]
-        return rows
-    return lambda T: sgraph.rows_native(spec, T)
-
-
-def host_feat_provider(preset, feat_dim=None, feat_dtype=None):
-    fd = preset.feat_dim if feat_dim is None else feat_dim
-    fdt = preset.feat_dtype if feat_dtype is None else feat_dtype
-
-    def feats(ids):
-        u = np.unique(np.asarray(ids, dtype=np.int64))
-        return u, sfeat.feature_bytes_native(spre.FEAT_SEED, u, fd, fdt)
-    return feats

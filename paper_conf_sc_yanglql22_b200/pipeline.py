@@ -34,6 +34,7 @@ def required_keys(n, fanouts, max_seeds):
 # several at a time on one GPU: a gather at full occupancy holds the whole register file and keeps
 # the other streams' latency-bound hop kernels from overlapping it ("Concurrency").
 THROUGHPUT_GATHER_OCCUPANCY = 1
+EXCL_RING = 4     # scan buffers per DSM workspace (wg_sample_hop: join the side stream before a fifth hop)
 PARAMS_RING = 64  # pinned staging slots for the per-batch scalars (batches enqueued ahead per pipeline)
 
 
@@ -108,6 +109,10 @@ class MiniBatchPipeline:
         prev_nu = None
         for h, m in enumerate(self.fanouts):
             b = self.hops[h]
+            if self.fused and h and h % EXCL_RING == 0:
+                # the workspace keeps a ring of EXCL_RING scan buffers read by the side-stream relabels:
+                # hop h reuses hop h-EXCL_RING's buffer, so that relabel must be done (include/wg.h)
+                main.wait_stream(self.side)
             if self.fused:
                 d.sample_hop(tgt, m, 0, h, n_targets_dev=tn, seed_dev=self.rng_seed, out=b, cap=tcap, stream=main,
                              side_stream=self.side)

@@ -12,4 +12,5 @@ cp abso/libwg_$V.so $L
 timeout 300 python bench.py --steps 50 --warmup 5 --cpu-sample-s 0 --e2e-steps 10 > gpurun_out/b.log 2>&1
 echo -n "$V r$r "; python profiles/bench_summary.py gpurun_out/b.log
 done; done
-cp abso/libwg_uq256.so $L
+# restore the default build from source (never a copied binary: _build.py stamps the flags + hash)
+python -c "from paper_conf_sc_yanglql22_b200 import _build; _build.build_lib(force=True)"

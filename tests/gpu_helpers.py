@@ -7,6 +7,7 @@ import torch
 import oracle
 import paper_conf_sc_yanglql22_b200 as pkg
 from paper_conf_sc_yanglql22_b200 import loader
+from synth import providers
 
 
 def csr_from_rows(rows):
@@ -17,10 +18,11 @@ def csr_from_rows(rows):
 
 
 def make_dsm(row_ptr, col, feat_rows=None, feat_dim=0, feat_dtype="fp32", max_keys=1 << 16, rank=0, world=1,
-             allgather=None):
+             allgather=None, flags=0):
     n = len(row_ptr) - 1
-    dsm = pkg.DSM(n, pkg.local_num_edges(row_ptr, rank, world), feat_dim, feat_dtype, max_keys, rank=rank,
-                  world_size=world, allgather=allgather)
+    e_local = len(col) if flags & pkg.WG_DSM_CSR_REPLICATED else pkg.local_num_edges(row_ptr, rank, world)
+    dsm = pkg.DSM(n, e_local, feat_dim, feat_dtype, max_keys, rank=rank,
+                  world_size=world, allgather=allgather, flags=flags)
     dsm.fill_from_global_csr(row_ptr, col)
     if feat_dim:
         dsm.fill_features(feat_rows[rank::world])
@@ -31,7 +33,7 @@ def make_dsm(row_ptr, col, feat_rows=None, feat_dim=0, feat_dtype="fp32", max_ke
 
 
 def oracle_hop(row_ptr, col, T, M, seed, hop):
-    rows = loader.host_row_provider(None, row_ptr, col)
+    rows = providers.host_row_provider(None, row_ptr, col)
     adj_ptr, adj = rows(np.asarray(T, dtype=np.int64))
     return oracle.sample_hop(adj_ptr, adj, T, M, seed, hop)
 

@@ -1,7 +1,8 @@
 """Worker for the multi-process tests (one process per rank; env RANK/WORLD_SIZE/
-MASTER_ADDR/MASTER_PORT).  Mode "ipc": every rank drives cuda:0 (one-GPU box), the
-DSM handles are exchanged over gloo and opened with cudaIpcOpenMemHandle; mode
-"gloo-host": CPU-only check of the host-side collective plumbing."""
+MASTER_ADDR/MASTER_PORT).  Mode "ipc": rank r drives cuda:(r % device_count) -- its own GPU on a
+multi-GPU box, all ranks on cuda:0 on a one-GPU box -- the DSM handles are exchanged over gloo and
+opened with cudaIpcOpenMemHandle (a peer on another GPU is read over NVLink); mode "gloo-host":
+CPU-only check of the host-side collective plumbing."""
 
 import os
 import sys
@@ -33,14 +34,17 @@ def main():
         import oracle
         import paper_conf_sc_yanglql22_b200 as pkg
         from paper_conf_sc_yanglql22_b200 import loader
+        from synth import providers
         from synth import graph, presets, seeds
-        torch.cuda.set_device(0)
+        dev = rank % torch.cuda.device_count()
+        torch.cuda.set_device(dev)
+        print(f"rank {rank} on device cuda:{dev}", flush=True)
         p = presets.get("tiny")
         ag = pkg.TorchDistAllgather()
-        dsm, _ = loader.build_dsm(p, rank=rank, world=world, allgather=ag, on_device=False)
+        dsm, _ = loader.build_dsm(p, rank=rank, world=world, device=dev, allgather=ag, on_device=False)
         rp, col = graph.csr(p.graph())
-        rows = loader.host_row_provider(p.graph(), rp, col)
-        feats = loader.host_feat_provider(p)
+        rows = providers.host_row_provider(p.graph(), rp, col)
+        feats = providers.host_feat_provider(p)
         pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
         for b in seeds.rank_batches(4, rank, world):
             S = seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, b)
@@ -60,12 +64,14 @@ def main():
         import oracle
         import paper_conf_sc_yanglql22_b200 as pkg
         from paper_conf_sc_yanglql22_b200 import loader
+        from synth import providers
         from paper_conf_sc_yanglql22_b200.nccl_gather import DistributedGather
         from synth import features, presets
-        torch.cuda.set_device(0)
+        dev = rank % torch.cuda.device_count()
+        torch.cuda.set_device(dev)
         p = presets.get("tiny")
         ag = pkg.TorchDistAllgather()
-        dsm, _ = loader.build_dsm(p, rank=rank, world=world, allgather=ag, on_device=False)
+        dsm, _ = loader.build_dsm(p, rank=rank, world=world, device=dev, allgather=ag, on_device=False)
         ids = np.random.default_rng(rank).integers(0, p.n, 7000).astype(np.int64)
         out = DistributedGather(dsm).gather(torch.from_numpy(ids).cuda())
         direct = dsm.gather(torch.from_numpy(ids).cuda())

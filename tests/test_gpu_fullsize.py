@@ -11,6 +11,7 @@ import torch
 import oracle
 import paper_conf_sc_yanglql22_b200 as pkg
 from paper_conf_sc_yanglql22_b200 import loader
+from synth import providers
 from synth import features, graph, presets, seeds
 
 pytestmark = pytest.mark.gpu
@@ -47,8 +48,8 @@ def test_products_batches_bit_exact(products):
     pipe.run(torch.from_numpy(S0).cuda(), seeds.rng_seed(presets.RNG_BASE, 0))
     torch.cuda.synchronize()
     pipe.capture()
-    rows = loader.host_row_provider(p.graph())
-    feats = loader.host_feat_provider(p)
+    rows = providers.host_row_provider(p.graph())
+    feats = providers.host_feat_provider(p)
     for b in (1, 2):
         S = seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, b)
         rs = seeds.rng_seed(presets.RNG_BASE, b)
@@ -81,7 +82,7 @@ def test_papers100m_shaped_batch_bit_exact():
         rs = seeds.rng_seed(presets.RNG_BASE, 7)
         pipe.run(torch.from_numpy(S).cuda(), rs)
         torch.cuda.synchronize()
-        ref = oracle.minibatch(loader.host_row_provider(p.graph()), loader.host_feat_provider(p), S, p.fanouts, rs)
+        ref = oracle.minibatch(providers.host_row_provider(p.graph()), providers.host_feat_provider(p), S, p.fanouts, rs)
         for h in range(len(p.fanouts)):
             got, exp = pipe.result(h), ref["hops"][h]
             for k in ("row_ptr", "nbrs", "pos", "unique", "sub_col", "dup"):
@@ -138,8 +139,8 @@ def test_mag240m_shaped_graph_w4_virtual_ranks_bit_exact():
             sgpu.fill_dsm_features_gpu(d, presets.FEAT_SEED, r, W, FD, features.WG_DTYPE_CODE[FDT])
         del shards
         torch.cuda.synchronize()
-        rows = loader.host_row_provider(spec)
-        feats = loader.host_feat_provider(p, FD, FDT)
+        rows = providers.host_row_provider(spec)
+        feats = providers.host_feat_provider(p, FD, FDT)
         for r in (0, 3):
             pipe = pkg.MiniBatchPipeline(dsms[r], p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
             b = next(iter(seeds.rank_batches(W, r, W)))
@@ -172,8 +173,8 @@ def test_products_throughput_configuration_bit_exact(products):
     S = [seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 500 + b) for b in range(nb)]
     rs = [seeds.rng_seed(presets.RNG_BASE, 500 + b) for b in range(nb)]
     batches = [(torch.from_numpy(s).pin_memory(), r) for s, r in zip(S, rs)]
-    rows = loader.host_row_provider(p.graph())
-    feats = loader.host_feat_provider(p)
+    rows = providers.host_row_provider(p.graph())
+    feats = providers.host_feat_provider(p)
     seen = 0
     for pb in ld(batches):
         ref = oracle.minibatch(rows, feats, S[seen], p.fanouts, rs[seen])

@@ -8,6 +8,7 @@ import torch
 import oracle
 import paper_conf_sc_yanglql22_b200 as pkg
 from paper_conf_sc_yanglql22_b200 import loader
+from synth import providers
 from synth import graph, presets, seeds
 
 pytestmark = pytest.mark.gpu
@@ -17,8 +18,8 @@ pytestmark = pytest.mark.gpu
 def test_loader_batches_bit_exact(depth, nb):
     p = presets.get("tiny")
     rp, col = graph.csr(p.graph())
-    rows = loader.host_row_provider(p.graph(), rp, col)
-    feats = loader.host_feat_provider(p)
+    rows = providers.host_row_provider(p.graph(), rp, col)
+    feats = providers.host_feat_provider(p)
     dsm, _ = loader.build_dsm(p, on_device=False)
     ld = pkg.MiniBatchLoader(dsm, p.fanouts, p.seeds_per_batch, depth=depth, with_pos=True, with_dup=True)
     S = [seeds.seed_nodes(p.n, p.seeds_per_batch - (b % 3) * 17, presets.SEED_BASE, b) for b in range(nb)]

@@ -1,0 +1,127 @@
+"""The characterisation kernels (Table I analogue, the prep-kernel ceilings of SURVEY.md 8(d)), the
+per-kernel stage events, and a compute-sanitizer racecheck of one batch."""
+
+import ctypes
+import os
+import subprocess
+import sys
+
+import pytest
+import torch
+
+import paper_conf_sc_yanglql22_b200 as pkg
+from paper_conf_sc_yanglql22_b200 import loader
+from paper_conf_sc_yanglql22_b200._lib import check, lib
+from synth import presets, seeds
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+def test_dsm_chase_latency_orders_l2_below_hbm():
+    """wg_dsm_chase: a span that fits L2 (4 MB) chases faster than one that cannot (4 GB), both within
+    plausible B200 load latencies; spans past the shard are refused."""
+    small = pkg.DSM(1 << 16, 0, 16, "fp32", 16)            # 4 MB of 64 B rows
+    big = pkg.DSM(1 << 26, 0, 16, "fp32", 16)              # 4 GB
+    small.local_view()[2].fill_(3)
+    big.local_view()[2].fill_(7)
+    small.chase(0, (1 << 16) * 64, 2000)                    # warm-up: module load, TLB, L2 fill
+    big.chase(0, (1 << 26) * 64, 2000)
+    ns_l2 = min(small.chase(0, (1 << 16) * 64, 20000) for _ in range(3))
+    ns_hbm = min(big.chase(0, (1 << 26) * 64, 20000) for _ in range(3))
+    assert 20 < ns_l2 < 2000 and 200 < ns_hbm < 5000, (ns_l2, ns_hbm)
+    assert ns_hbm > 1.2 * ns_l2, (ns_l2, ns_hbm)
+    with pytest.raises(pkg.WgError):
+        small.chase(0, (1 << 16) * 64 * 2, 10)
+    small.destroy()
+    big.destroy()
+
+
+def _rate(fn, n):
+    best = None
+    for _ in range(3):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        fn()
+        e1.record()
+        e1.synchronize()
+        t = e0.elapsed_time(e1) / 1e3
+        best = t if best is None else min(best, t)
+    return n.value / best
+
+
+def test_micro_ceilings_plausible():
+    """wg_micro_random_read / wg_micro_atomics: random loads over an L2-sized span beat loads over 4 GB of
+    HBM, the HBM rate is bounded by the copy bandwidth at one 32 B sector per load, atomics run at a
+    positive rate; bad arguments are refused."""
+    sink = torch.zeros(1, dtype=torch.int64, device="cuda")
+    big = torch.zeros(4 << 30, dtype=torch.uint8, device="cuda")
+    small = torch.zeros(8 << 20, dtype=torch.uint8, device="cuda")
+    table = torch.zeros(1 << 21, dtype=torch.int64, device="cuda")
+    n = ctypes.c_int64()
+    st = ctypes.c_void_p(torch.cuda.current_stream().cuda_stream)
+    P = lambda t: ctypes.c_void_p(t.data_ptr())  # noqa: E731
+    r_hbm = _rate(lambda: check(lib().wg_micro_random_read(P(big), big.numel(), 8, 8, 8, P(sink), ctypes.byref(n), st)), n)
+    r_l2 = _rate(lambda: check(lib().wg_micro_random_read(P(small), small.numel(), 8, 8, 8, P(sink), ctypes.byref(n), st)), n)
+    assert 1e9 < r_hbm < 8e12 / 32, r_hbm
+    assert r_l2 > 1.2 * r_hbm, (r_l2, r_hbm)
+    for op in (0, 1, 2):
+        r = _rate(lambda: check(lib().wg_micro_atomics(P(table), table.numel(), op, 4, 8, P(sink), ctypes.byref(n), st)), n)
+        assert 1e9 < r < 1e13, (op, r)
+    assert lib().wg_micro_random_read(P(small), small.numel(), 16, 8, 8, P(sink), None, st) != 0
+    assert lib().wg_micro_atomics(P(table), table.numel(), 3, 8, 8, P(sink), None, st) != 0
+
+
+def test_stage_events_split_a_hop():
+    """wg_dsm_set_stage_events: the events recorded after the sampler, insert, flag scan and relabel of a
+    hop are ordered, and together they cover the hop."""
+    p = presets.get("tiny")
+    dsm, _ = loader.build_dsm(p, on_device=False)
+    S = torch.from_numpy(seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 1)).cuda()
+    evs = [torch.cuda.Event(enable_timing=True) for _ in range(5)]
+    for e in evs:
+        e.record()
+    evs[0].record()
+    dsm.set_stage_events(evs[1:])
+    o = dsm.sample_hop(S, p.fanouts[0], 5, 0)
+    dsm.set_stage_events([])
+    end = torch.cuda.Event(enable_timing=True)
+    end.record()
+    torch.cuda.synchronize()
+    parts = [evs[k].elapsed_time(evs[k + 1]) for k in range(4)]
+    assert all(x >= 0 for x in parts), parts
+    assert sum(parts) <= evs[0].elapsed_time(end) + 1e-3
+    assert int(o["num_unique"].item()) > len(S)
+    with pytest.raises(pkg.WgError):
+        dsm.set_stage_events([evs[0]] * 9)
+    assert dsm.device_error() == 0
+    dsm.destroy()
+
+
+@pytest.mark.slow
+def test_racecheck_one_batch():
+    """compute-sanitizer racecheck (shared-memory hazards: the sampler's chain words, the look-back
+    scan's smem) and synccheck over one fused batch + its gather: zero hazards, zero errors."""
+    code = r'''
+import sys, torch
+sys.path.insert(0, ".")
+import paper_conf_sc_yanglql22_b200 as pkg
+from paper_conf_sc_yanglql22_b200 import loader
+from synth import presets, seeds
+p = presets.get("tiny")
+dsm, _ = loader.build_dsm(p, on_device=False)
+pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_dup=True)
+pipe.run(torch.from_numpy(seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 0)).cuda(), 1)
+torch.cuda.synchronize()
+assert dsm.device_error() == 0
+dsm.destroy()
+print("BATCH OK")
+'''
+    cs = "/usr/local/cuda/bin/compute-sanitizer"
+    if not os.path.exists(cs):
+        pytest.skip("compute-sanitizer not installed")
+    for tool, summary in (("racecheck", "RACECHECK SUMMARY: 0 hazards"), ("synccheck", "ERROR SUMMARY: 0 errors")):
+        r = subprocess.run([cs, "--tool", tool, "--kernel-name", "kns=2wg", "--error-exitcode", "17", sys.executable,
+                            "-c", code], cwd=ROOT, capture_output=True, text=True, timeout=900)
+        assert r.returncode == 0 and "BATCH OK" in r.stdout and summary in r.stdout, (tool, r.stdout[-2000:],
+                                                                                      r.stderr[-2000:])

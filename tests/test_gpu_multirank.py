@@ -14,20 +14,21 @@ import torch
 import oracle
 import paper_conf_sc_yanglql22_b200 as pkg
 from paper_conf_sc_yanglql22_b200 import loader
+from synth import providers
 from synth import graph, presets, seeds
 
 pytestmark = pytest.mark.gpu
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def _create_all(p, W):
+def _create_all(p, W, flags=0):
     ag = pkg.ThreadAllgather(W)
     out = [None] * W
     errs = []
 
     def run(r):
         try:
-            out[r] = loader.build_dsm(p, rank=r, world=W, allgather=ag.for_rank(r), on_device=False)[0]
+            out[r] = loader.build_dsm(p, rank=r, world=W, allgather=ag.for_rank(r), on_device=False, flags=flags)[0]
         except Exception as e:  # pragma: no cover
             errs.append(e)
     ths = [threading.Thread(target=run, args=(r,)) for r in range(W)]
@@ -43,15 +44,22 @@ def _destroy_all(dsms):
     [t.join() for t in ths]
 
 
-@pytest.mark.parametrize("W", [2, 3, 4, 8])
-def test_virtual_ranks_w_invariance(W):
+@pytest.mark.parametrize("W,placement", [(2, "dsm"), (3, "dsm"), (4, "dsm"), (8, "dsm"), (2, "csr-replicated"),
+                                         (4, "csr-replicated"), (8, "csr-replicated")])
+def test_virtual_ranks_w_invariance(W, placement):
+    """Every rank's batches are byte-identical to the oracle for the paper's placement (CSR and features
+    row-sharded) and for the hybrid one (whole CSR on every rank, features sharded)."""
     p = presets.get("tiny")
     rp, col = graph.csr(p.graph())
-    dsms = _create_all(p, W)
-    rows = loader.host_row_provider(p.graph(), rp, col)
-    feats = loader.host_feat_provider(p)
+    flags = pkg.WG_DSM_CSR_REPLICATED if placement == "csr-replicated" else 0
+    dsms = _create_all(p, W, flags)
+    rows = providers.host_row_provider(p.graph(), rp, col)
+    feats = providers.host_feat_provider(p)
     for r, dsm in enumerate(dsms):
         assert dsm.shard_info(r)[0] == len(graph.shard_rows(p.n, r, W))
+        if flags:
+            lrp, lcol, _ = dsm.local_view()
+            assert lrp.numel() == p.n + 1 and lcol.numel() == len(col)   # the whole CSR on every rank
         pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
         for b in seeds.rank_batches(2 * W, r, W):
             S = seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, b)
@@ -85,21 +93,45 @@ def test_two_processes_cuda_ipc(mode):
         assert "PARITY OK" in o, o
 
 
-@pytest.mark.parametrize("placement", ["dsm", "replicas"])
+def test_real_multi_gpu_processes():
+    """W = min(device_count, 8) processes, rank r on its own GPU cuda:r: cross-device cudaIpcOpenMemHandle
+    and NVLink P2P loads from the sampler and the gather, every array bit-exact against the oracle.
+    Skips (visibly) on a one-GPU box, where the same-GPU IPC test below covers the host logic."""
+    ndev = torch.cuda.device_count()
+    if ndev < 2:
+        pytest.skip(f"needs >= 2 GPUs for one process per GPU (this box has {ndev})")
+    W = min(ndev, 8)
+    port = 29400 + os.getpid() % 1000
+    env = dict(os.environ, MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port), WORLD_SIZE=str(W),
+               LOCAL_WORLD_SIZE=str(W))
+    procs = []
+    for r in range(W):
+        e = dict(env, RANK=str(r), LOCAL_RANK=str(r))
+        procs.append(subprocess.Popen([sys.executable, os.path.join(ROOT, "tests", "mp_worker.py"), "ipc"],
+                                      env=e, stdout=subprocess.PIPE, stderr=subprocess.STDOUT))
+    outs = [p.communicate(timeout=900)[0].decode() for p in procs]
+    for r, (p, o) in enumerate(zip(procs, outs)):
+        assert p.returncode == 0, o
+        assert "PARITY OK" in o and f"device cuda:{r}" in o, o
+
+
+@pytest.mark.parametrize("placement", ["dsm", "csr-replicated", "replicas"])
 def test_bench_torchrun_two_ranks(placement):
     """The driver's N>1 launch of bench.py (torchrun, one process per rank) on the one test GPU:
     every rank must reach the same collectives (max over ranks, barriers, collective destroy) and
     rank 0 prints one JSON line with the whole-job value."""
     import json
-    port = 29600 + os.getpid() % 500 + (3 if placement == "dsm" else 0)
+    port = 29600 + os.getpid() % 500 + {"dsm": 3, "csr-replicated": 5, "replicas": 0}[placement]
     cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2",
            "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.join(ROOT, "bench.py"),
            "--gpus", "2", "--steps", "3", "--warmup", "3", "--cpu-sample-s", "0", "--e2e-steps", "1",
-           "--concurrency", "2", "--config", "tiny", "--placement", placement]
+           "--concurrency", "2", "--config", "tiny", "--placement", placement, "--north-star", ""]
     r = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=300)
     assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
     lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
     assert len(lines) == 1, r.stdout
     d = json.loads(lines[0])
     assert d["n_gpus"] == 2 and d["value"] > 0 and d["e2e"]["value"] > 0 and d["single_batch"]["value"] > 0
-    assert d["config"]["parallelism"].startswith("dsm-w2" if placement == "dsm" else "replicas-x2")
+    assert d["config"]["parallelism"].startswith({"dsm": "dsm-w2", "csr-replicated": "csr-replicated-w2",
+                                                  "replicas": "replicas-x2"}[placement])
+    assert d["parity"]["ok"] is True and d["parity"]["ranks"] == 2 and d["parity"]["batches"] == 2

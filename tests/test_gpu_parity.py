@@ -10,6 +10,7 @@ import torch
 import oracle
 import paper_conf_sc_yanglql22_b200 as pkg
 from paper_conf_sc_yanglql22_b200 import loader
+from synth import providers
 from synth import features, graph, presets, seeds
 
 from gpu_helpers import csr_from_rows, gpu_hop, gpu_unique, make_dsm, oracle_hop
@@ -41,8 +42,8 @@ def test_tiny_pipeline_many_batches(tiny, fused, incr):
     dsm, _ = loader.build_dsm(p, on_device=False)
     pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True, fused=fused,
                                  incremental_gather=incr)
-    rows = loader.host_row_provider(p.graph(), rp, col)
-    feats = loader.host_feat_provider(p)
+    rows = providers.host_row_provider(p.graph(), rp, col)
+    feats = providers.host_feat_provider(p)
     for b in range(20):
         S = seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, b)
         rs = seeds.rng_seed(presets.RNG_BASE, b)
@@ -63,8 +64,8 @@ def test_tiny_cuda_graph_replay(tiny):
     pipe.run(torch.from_numpy(S0).cuda(), 1)
     torch.cuda.synchronize()
     pipe.capture()
-    rows = loader.host_row_provider(p.graph(), rp, col)
-    feats = loader.host_feat_provider(p)
+    rows = providers.host_row_provider(p.graph(), rp, col)
+    feats = providers.host_feat_provider(p)
     for b in (3, 4, 5):
         n = 100 + 150 * (b - 3)      # fewer seeds than the capacity: device counts drive the graph
         S = seeds.seed_nodes(p.n, n, presets.SEED_BASE, b)
@@ -183,34 +184,20 @@ def test_gather_rows(dim, dtype):
     dsm.destroy()
 
 
-def test_feat_split_layout_off_subprocess():
-    """WG_FEAT_SPLIT=0 (whole rows at a 64 B pitch, read once at create) gathers the same bytes."""
-    import os
-    import subprocess
-    import sys
-    code = r'''
-import sys, numpy as np, torch
-sys.path.insert(0, "tests")
-from gpu_helpers import make_dsm
-import oracle
-from synth import features, presets
-for dim, dtype in ((100, "fp32"), (36, "fp32"), (200, "fp16")):
-    n = 4000
-    rp = np.zeros(n + 1, dtype=np.int64)
-    feat = features.feature_bytes(presets.FEAT_SEED, np.arange(n), dim, dtype)
-    dsm = make_dsm(rp, np.zeros(0, np.int64), feat, dim, dtype)
-    assert dsm.tail_pitch == 0 and dsm.body_bytes == dsm.row_bytes
-    ids = np.random.default_rng(dim).integers(0, n, 6000).astype(np.int64)
-    X = dsm.gather(torch.from_numpy(ids).cuda())
-    torch.cuda.synchronize()
-    assert np.array_equal(X.cpu().numpy(), oracle.gather(feat, np.arange(n), ids)), (dim, dtype)
-    dsm.destroy()
-print("NOSPLIT OK")
-'''
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    r = subprocess.run([sys.executable, "-c", code], cwd=root, env=dict(os.environ, WG_FEAT_SPLIT="0"),
-                       capture_output=True, text=True, timeout=600)
-    assert r.returncode == 0 and "NOSPLIT OK" in r.stdout, r.stdout + r.stderr
+def test_feat_whole_rows_flag():
+    """WG_DSM_WHOLE_ROWS (whole rows at a 64 B pitch instead of the split body + tail layout)
+    gathers the same bytes."""
+    for dim, dtype in ((100, "fp32"), (36, "fp32"), (200, "fp16")):
+        n = 4000
+        rp = np.zeros(n + 1, dtype=np.int64)
+        feat = features.feature_bytes(presets.FEAT_SEED, np.arange(n), dim, dtype)
+        dsm = make_dsm(rp, np.zeros(0, np.int64), feat, dim, dtype, flags=pkg.WG_DSM_WHOLE_ROWS)
+        assert dsm.tail_pitch == 0 and dsm.body_bytes == dsm.row_bytes
+        ids = np.random.default_rng(dim).integers(0, n, 6000).astype(np.int64)
+        X = dsm.gather(torch.from_numpy(ids).cuda())
+        torch.cuda.synchronize()
+        assert np.array_equal(X.cpu().numpy(), oracle.gather(feat, np.arange(n), ids)), (dim, dtype)
+        dsm.destroy()
 
 
 def test_determinism_two_runs(tiny):
@@ -239,8 +226,8 @@ def test_fork_concurrent_streams(tiny):
     pipes = [pkg.MiniBatchPipeline(h, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
              for h in (dsm, child)]
     streams = [torch.cuda.Stream(), torch.cuda.Stream()]
-    rows = loader.host_row_provider(p.graph(), rp, col)
-    feats = loader.host_feat_provider(p)
+    rows = providers.host_row_provider(p.graph(), rp, col)
+    feats = providers.host_feat_provider(p)
     for rnd in range(3):
         Ss, rss = [], []
         for j in range(2):
@@ -264,51 +251,6 @@ def test_fork_concurrent_streams(tiny):
     dsm.destroy()
 
 
-@pytest.mark.parametrize("knob", ["WG_GATHER_TMA", "WG_GATHER_ASYNC", "WG_GATHER_G4"])
-def test_gather_tma_variant_subprocess(knob):
-    """The TMA bulk-copy gather (WG_GATHER_TMA=1) and the cp.async gather (WG_GATHER_ASYNC=1), chosen
-    once per process, are bit-exact too (whole / split rows, pitched outputs, partial ranges)."""
-    import os
-    import subprocess
-    import sys
-    code = r'''
-import sys, numpy as np, torch
-sys.path.insert(0, "tests")
-from gpu_helpers import make_dsm
-import oracle
-from synth import features, presets
-for dim, dtype in ((100, "fp32"), (4, "fp32"), (768, "fp16"), (1024, "fp32"), (3, "fp32")):
-    n = 5000
-    rp = np.zeros(n + 1, dtype=np.int64)
-    feat = features.feature_bytes(presets.FEAT_SEED, np.arange(n), dim, dtype)
-    dsm = make_dsm(rp, np.zeros(0, np.int64), feat, dim, dtype)
-    rng = np.random.default_rng(dim)
-    for ids in (rng.integers(0, n, 7777), np.arange(n)[::-1], np.full(33, 7), np.zeros(0)):
-        ids = np.ascontiguousarray(ids, dtype=np.int64)
-        X = dsm.gather(torch.from_numpy(ids).cuda())
-        torch.cuda.synchronize()
-        assert np.array_equal(X[:len(ids)].cpu().numpy(), oracle.gather(feat, np.arange(n), ids)), (dim, dtype)
-        # pitched output through wg_gather_rows (rows [begin, end) only)
-        if len(ids) > 10:
-            pitch = dsm.out_pitch()
-            out = torch.full((len(ids), pitch), 0xAB, dtype=torch.uint8, device="cuda")
-            be = torch.tensor([5, len(ids) - 3], dtype=torch.int64, device="cuda")
-            dsm.gather_rows(torch.from_numpy(ids).cuda(), len(ids), be[0:1], be[1:2], out)
-            torch.cuda.synchronize()
-            o = out.cpu().numpy()
-            rb = dsm.row_bytes
-            assert np.array_equal(o[5:len(ids) - 3, :rb], oracle.gather(feat, np.arange(n), ids[5:len(ids) - 3]))
-            assert (o[:5] == 0xAB).all() and (o[len(ids) - 3:] == 0xAB).all()
-    assert dsm.device_error() == 0
-    dsm.destroy()
-print("TMA OK")
-'''
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    r = subprocess.run([sys.executable, "-c", code], cwd=root, env=dict(os.environ, **{knob: "1"}),
-                       capture_output=True, text=True, timeout=600)
-    assert r.returncode == 0 and "TMA OK" in r.stdout, r.stdout + r.stderr
-
-
 @pytest.mark.parametrize("M", [33, 64, 100, 257, 1024])
 def test_sample_large_fanout_block_kernel(M):
     """fanout > 32: block per target running Algorithm 1 with a block bitonic sort (NEXT #4)."""
@@ -329,6 +271,27 @@ def test_sample_large_fanout_block_kernel(M):
     dsm.destroy()
 
 
+def test_pipeline_five_hops_fused(tiny):
+    """More hops than the workspace's ring of 4 scan buffers: the fused pipeline joins the relabel side
+    stream before hop 4 reuses hop 0's buffer, so every hop's sub_col / dup stays exact (captured graph)."""
+    p, rp, col = tiny
+    fan = [4, 3, 2, 2, 2]
+    dsm, _ = loader.build_dsm(p, on_device=False, max_seeds=64, extra_keys=pkg.required_keys(p.n, fan, 64))
+    pipe = pkg.MiniBatchPipeline(dsm, fan, 64, with_pos=True, with_dup=True)
+    rows = providers.host_row_provider(p.graph(), rp, col)
+    feats = providers.host_feat_provider(p)
+    for b in range(4):
+        S = seeds.seed_nodes(p.n, 64, presets.SEED_BASE, 700 + b)
+        rs = seeds.rng_seed(presets.RNG_BASE, 700 + b)
+        pipe.run(torch.from_numpy(S).cuda(), rs)
+        torch.cuda.synchronize()
+        _check_batch(pipe, oracle.minibatch(rows, feats, S, fan, rs), fan)
+        if b == 0:
+            pipe.capture()
+    assert dsm.device_error() == 0
+    dsm.destroy()
+
+
 def test_pipeline_large_fanout(tiny):
     p, rp, col = tiny
     dsm, _ = loader.build_dsm(p, on_device=False, max_seeds=64, extra_keys=64 * 60 * 41 + 64 * 60)
@@ -338,21 +301,9 @@ def test_pipeline_large_fanout(tiny):
     rs = seeds.rng_seed(presets.RNG_BASE, 3)
     pipe.run(torch.from_numpy(S).cuda(), rs)
     torch.cuda.synchronize()
-    ref = oracle.minibatch(loader.host_row_provider(p.graph(), rp, col), loader.host_feat_provider(p), S, fan, rs)
+    ref = oracle.minibatch(providers.host_row_provider(p.graph(), rp, col), providers.host_feat_provider(p), S, fan, rs)
     _check_batch(pipe, ref, fan)
     assert dsm.device_error() == 0
-    dsm.destroy()
-
-
-def test_dsm_chase_latency_runs():
-    """wg_dsm_chase (Table I analogue): a positive, plausible per-access latency; span checks."""
-    n = 1 << 16
-    rp = np.zeros(n + 1, dtype=np.int64)
-    dsm = pkg.DSM(n, 0, 16, "fp32", 16)
-    ns = dsm.chase(0, n * 64, 20000)
-    assert 20 < ns < 5000
-    with pytest.raises(pkg.WgError):
-        dsm.chase(0, n * 64 * 2, 10)
     dsm.destroy()
 
 
@@ -389,6 +340,24 @@ def test_spmm_mean_forward_backward_vs_oracle(tiny):
     out = layers.SpMMMean.apply(Xg, row_ptr, sub_col, dup)
     (out * dY).sum().backward()
     assert np.allclose(Xg.grad.cpu().numpy(), dXo, rtol=1e-5, atol=1e-5)
+    # the pipeline's untrimmed buffers with the device row count (the previous hop's num_unique)
+    b = pipe.hops[1]
+    Xg2 = X.clone().requires_grad_(True)
+    out2 = layers.SpMMMean.apply(Xg2, b["row_ptr"], b["sub_col"], b["dup"], pipe.hops[0]["num_unique"])
+    assert np.allclose(out2[:nT].detach().cpu().numpy(), Yo, rtol=0, atol=1e-5)
+    assert not out2[nT:].any()
+    dYp = torch.zeros_like(out2)
+    dYp[:nT] = dY
+    (out2 * dYp).sum().backward()
+    assert np.allclose(Xg2.grad.cpu().numpy(), dXo, rtol=1e-5, atol=1e-5)
+    # an out-of-range sub-graph id (the -1 of an invalid id) is skipped, never dereferenced
+    bad = sub_col.clone()
+    bad[0] = -1
+    bad[1] = U + 5
+    Yb = layers.spmm_mean_forward(row_ptr, bad, X)
+    dXb = layers.spmm_mean_backward(row_ptr, bad, dup, dY, U)
+    torch.cuda.synchronize()
+    assert torch.isfinite(Yb).all() and torch.isfinite(dXb).all()
     dsm.destroy()
 
 
@@ -400,10 +369,10 @@ def test_distributed_memory_gather_w1():
     feat = features.feature_bytes(presets.FEAT_SEED, np.arange(n), dim, "fp32")
     dsm = make_dsm(rp, np.zeros(0, np.int64), feat, dim, "fp32")
     ids = torch.from_numpy(np.random.default_rng(3).integers(0, n, 20000)).cuda()
-    a = dsm.gather(ids)
     b = DistributedGather(dsm).gather(ids)
     torch.cuda.synchronize()
-    assert torch.equal(a[:20000], b[:20000])
+    exp = oracle.gather(feat, np.arange(n), ids.cpu().numpy())   # the closed-form rows, not the P2P path
+    assert np.array_equal(b[:20000].cpu().numpy(), exp)
     assert dsm.device_error() == 0
     dsm.destroy()
 
@@ -420,7 +389,7 @@ def test_pipeline_degenerate_batches(tiny):
     feat = features.feature_bytes(presets.FEAT_SEED, np.arange(n), 8, "fp32")
     dsm = make_dsm(g_rp, g_col, feat, 8, "fp32", max_keys=4096)
     pipe = pkg.MiniBatchPipeline(dsm, [3, 2], 16, with_pos=True, with_dup=True)
-    rowsf = loader.host_row_provider(None, g_rp, g_col)
+    rowsf = providers.host_row_provider(None, g_rp, g_col)
 
     def feats(ids):
         u = np.unique(np.asarray(ids, dtype=np.int64))
@@ -437,38 +406,27 @@ def test_pipeline_degenerate_batches(tiny):
     dsm.destroy()
 
 
-def test_epoch_exhaustion_and_reset(tiny):
-    """The hash-table epoch space: near its end an op latches WG_DEVERR_EPOCH;
-    wg_dsm_reset_workspace restores correct operation (test hook WG_EPOCH_START)."""
-    import os
-    import subprocess
-    import sys
-    code = r'''
-import sys, numpy as np, torch
-sys.path.insert(0, "tests")
-import oracle
-from gpu_helpers import make_dsm, gpu_unique
-T = np.array([4, 9], np.int64); nb = np.array([1, 4, 1, 7], np.int64)
-rp = np.zeros(11, np.int64)
-dsm = make_dsm(rp, np.zeros(0, np.int64), max_keys=64)
-U, sc, dup = gpu_unique(dsm, T, nb)          # uses epoch EPOCH_MAX-2 -> bumps to EPOCH_MAX-1
-assert list(U) == [4, 9, 1, 7] and dsm.device_error() == 0
-gpu_unique(dsm, T, nb)                       # epoch + 1 would reach EPOCH_MAX: latched
-assert dsm.device_error() & 0x10
-dsm.reset_workspace(); torch.cuda.synchronize()
-for _ in range(3):
-    U, sc, dup = gpu_unique(dsm, T, nb)
-    Uo, sco, dupo = oracle.append_unique(T, nb)
-    assert np.array_equal(U, Uo) and np.array_equal(sc, sco) and np.array_equal(dup, dupo)
-assert dsm.device_error() == 0
-dsm.destroy()
-print("EPOCH OK")
-'''
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    r = subprocess.run([sys.executable, "-c", code], cwd=root,
-                       env=dict(os.environ, WG_EPOCH_START=str((1 << 23) - 3), WG_HASH_COMPACT="0"),
-                       capture_output=True, text=True, timeout=600)
-    assert r.returncode == 0 and "EPOCH OK" in r.stdout, r.stdout + r.stderr
+def test_epoch_exhaustion_and_reset():
+    """The wide table's epoch space: near its end an op latches WG_DEVERR_EPOCH;
+    wg_dsm_reset_workspace restores correct operation (test hook wg_dsm_debug_set_epoch)."""
+    T = np.array([4, 9], np.int64)
+    nb = np.array([1, 4, 1, 7], np.int64)
+    dsm = make_dsm(np.zeros(11, np.int64), np.zeros(0, np.int64), max_keys=64, flags=pkg.WG_DSM_WIDE_HASH)
+    dsm.debug_set_epoch((1 << 23) - 3)
+    U, sc, dup = gpu_unique(dsm, T, nb)          # uses epoch EPOCH_MAX-2 -> bumps to EPOCH_MAX-1
+    assert list(U) == [4, 9, 1, 7] and dsm.device_error() == 0
+    gpu_unique(dsm, T, nb)                       # epoch + 1 would reach EPOCH_MAX: latched
+    assert dsm.device_error() & 0x10
+    dsm.reset_workspace()
+    torch.cuda.synchronize()
+    for _ in range(3):
+        U, sc, dup = gpu_unique(dsm, T, nb)
+        Uo, sco, dupo = oracle.append_unique(T, nb)
+        assert np.array_equal(U, Uo) and np.array_equal(sc, sco) and np.array_equal(dup, dupo)
+    assert dsm.device_error() == 0
+    with pytest.raises(pkg.WgError):
+        dsm.debug_set_epoch(0)
+    dsm.destroy()
 
 
 def test_compact_table_epoch_cycles(tiny):
@@ -476,54 +434,33 @@ def test_compact_table_epoch_cycles(tiny):
     (by the fused hop's sampler, or before a standalone insert): 140 tiny batches (280 fused hops,
     more than a whole cycle, starting just before a restart) and standalone append-unique calls
     across a restart, all bit-exact against the oracle."""
-    import os
-    import subprocess
-    import sys
-    code = r'''
-import sys, numpy as np, torch
-sys.path.insert(0, "tests")
-import oracle
-import paper_conf_sc_yanglql22_b200 as pkg
-from paper_conf_sc_yanglql22_b200 import loader
-from gpu_helpers import make_dsm, gpu_unique
-from synth import graph, presets, seeds
-p = presets.get("tiny")
-rp, col = graph.csr(p.graph())
-rows = loader.host_row_provider(p.graph(), rp, col)
-feats = loader.host_feat_provider(p)
-dsm, _ = loader.build_dsm(p, on_device=False)
-pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
-pipe.run(torch.from_numpy(seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 0)).cuda(), 5)
-pipe.capture()
-for b in range(140):
-    S = seeds.seed_nodes(p.n, p.seeds_per_batch - (b % 5) * 11, presets.SEED_BASE, 1000 + b)
-    rs = seeds.rng_seed(presets.RNG_BASE, 1000 + b)
-    pipe.run(torch.from_numpy(S).cuda(), rs)
-    torch.cuda.synchronize()
-    ref = oracle.minibatch(rows, feats, S, p.fanouts, rs)
-    for h in range(len(p.fanouts)):
-        got, exp = pipe.result(h), ref["hops"][h]
-        for k in ("row_ptr", "nbrs", "pos", "unique", "sub_col", "dup"):
-            assert np.array_equal(got[k], exp[k]), (b, h, k)
-    assert np.array_equal(pipe.features(), ref["X"]), b
-assert dsm.device_error() == 0
-dsm.destroy()
-rng = np.random.default_rng(3)
-d2 = make_dsm(np.zeros(2001, np.int64), np.zeros(0, np.int64), max_keys=4096)
-for i in range(300):
-    T = rng.choice(2000, 40, replace=False).astype(np.int64)
-    nb = rng.integers(0, 2000, 600).astype(np.int64)
-    U, sc, dup = gpu_unique(d2, T, nb)
-    Uo, sco, dupo = oracle.append_unique(T, nb)
-    assert np.array_equal(U, Uo) and np.array_equal(sc, sco) and np.array_equal(dup, dupo), i
-assert d2.device_error() == 0
-d2.destroy()
-print("CYCLE OK")
-'''
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    r = subprocess.run([sys.executable, "-c", code], cwd=root, env=dict(os.environ, WG_EPOCH_START="250"),
-                       capture_output=True, text=True, timeout=900)
-    assert r.returncode == 0 and "CYCLE OK" in r.stdout, r.stdout + r.stderr
+    p, rp, col = tiny
+    rows = providers.host_row_provider(p.graph(), rp, col)
+    feats = providers.host_feat_provider(p)
+    dsm, _ = loader.build_dsm(p, on_device=False)
+    dsm.debug_set_epoch(250)
+    pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
+    pipe.run(torch.from_numpy(seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 0)).cuda(), 5)
+    pipe.capture()
+    for b in range(140):
+        S = seeds.seed_nodes(p.n, p.seeds_per_batch - (b % 5) * 11, presets.SEED_BASE, 1000 + b)
+        rs = seeds.rng_seed(presets.RNG_BASE, 1000 + b)
+        pipe.run(torch.from_numpy(S).cuda(), rs)
+        torch.cuda.synchronize()
+        _check_batch(pipe, oracle.minibatch(rows, feats, S, p.fanouts, rs), p.fanouts)
+    assert dsm.device_error() == 0
+    dsm.destroy()
+    rng = np.random.default_rng(3)
+    d2 = make_dsm(np.zeros(2001, np.int64), np.zeros(0, np.int64), max_keys=4096)
+    d2.debug_set_epoch(250)
+    for i in range(300):
+        T = rng.choice(2000, 40, replace=False).astype(np.int64)
+        nb = rng.integers(0, 2000, 600).astype(np.int64)
+        U, sc, dup = gpu_unique(d2, T, nb)
+        Uo, sco, dupo = oracle.append_unique(T, nb)
+        assert np.array_equal(U, Uo) and np.array_equal(sc, sco) and np.array_equal(dup, dupo), i
+    assert d2.device_error() == 0
+    d2.destroy()
 
 
 def test_gather_occupancy_setting(tiny):
@@ -533,7 +470,7 @@ def test_gather_occupancy_setting(tiny):
     dsm, _ = loader.build_dsm(p, on_device=False)
     S = seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 5)
     rs = seeds.rng_seed(presets.RNG_BASE, 5)
-    ref = oracle.minibatch(loader.host_row_provider(p.graph(), rp, col), loader.host_feat_provider(p), S,
+    ref = oracle.minibatch(providers.host_row_provider(p.graph(), rp, col), providers.host_feat_provider(p), S,
                            p.fanouts, rs)
     for occ in (1, 2, 3, 0):
         pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, gather_occupancy=occ)
@@ -550,55 +487,34 @@ def test_gather_occupancy_setting(tiny):
     dsm.destroy()
 
 
-@pytest.mark.parametrize("env", [{"WG_HASH_COMPACT": "0"}, {"WG_HASH_COMPACT": "0", "WG_HASH_CAS128": "0"},
-                                 {"WG_PAD32": "0"}, {"WG_HASH_PER_CALL": "0"}])
-def test_table_and_slot_formats_subprocess(env):
-    """The non-default hash-table / padded-slot formats (16 B wide slots with 128-bit or 64-bit CAS
-    claims, int64 padded sampler slots, whole-table calls) stay bit-exact: 12 tiny batches through
-    the fused pipeline and hub-heavy standalone append-unique calls."""
-    import os
-    import subprocess
-    import sys
-    code = r'''
-import sys, numpy as np, torch
-sys.path.insert(0, "tests")
-import oracle
-import paper_conf_sc_yanglql22_b200 as pkg
-from paper_conf_sc_yanglql22_b200 import loader
-from gpu_helpers import make_dsm, gpu_unique
-from synth import graph, presets, seeds
-p = presets.get("tiny")
-rp, col = graph.csr(p.graph())
-rows = loader.host_row_provider(p.graph(), rp, col)
-feats = loader.host_feat_provider(p)
-dsm, _ = loader.build_dsm(p, on_device=False)
-pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
-for b in range(12):
-    S = seeds.seed_nodes(p.n, p.seeds_per_batch - b * 7, presets.SEED_BASE, 300 + b)
-    rs = seeds.rng_seed(presets.RNG_BASE, 300 + b)
-    pipe.run(torch.from_numpy(S).cuda(), rs)
-    torch.cuda.synchronize()
-    ref = oracle.minibatch(rows, feats, S, p.fanouts, rs)
-    for h in range(len(p.fanouts)):
-        got, exp = pipe.result(h), ref["hops"][h]
-        for k in ("row_ptr", "nbrs", "pos", "unique", "sub_col", "dup"):
-            assert np.array_equal(got[k], exp[k]), (b, h, k)
-    assert np.array_equal(pipe.features(), ref["X"]), b
-assert dsm.device_error() == 0
-dsm.destroy()
-rng = np.random.default_rng(11)
-d2 = make_dsm(np.zeros(5001, np.int64), np.zeros(0, np.int64), max_keys=1 << 16)
-for i in range(20):
-    T = rng.choice(5000, 300, replace=False).astype(np.int64)
-    nb = np.minimum((rng.pareto(1.2, 20000) * 3).astype(np.int64), 4999)   # hub-heavy
-    U, sc, dup = gpu_unique(d2, T, nb)
-    Uo, sco, dupo = oracle.append_unique(T, nb)
-    assert np.array_equal(U, Uo) and np.array_equal(sc, sco) and np.array_equal(dup, dupo), i
-assert d2.device_error() == 0
-d2.destroy()
-print("FORMAT OK")
-'''
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    r = subprocess.run([sys.executable, "-c", code], cwd=root, env=dict(os.environ, **env),
-                       capture_output=True, text=True, timeout=900)
-    assert r.returncode == 0 and "FORMAT OK" in r.stdout, r.stdout + r.stderr
+@pytest.mark.parametrize("flags", ["WG_DSM_WIDE_HASH", "WG_DSM_PAD64", "WG_DSM_WIDE_HASH|WG_DSM_PAD64"])
+def test_table_and_slot_formats(tiny, flags):
+    """The non-default hash-table / padded-slot formats (16 B wide slots claimed with one 128-bit CAS,
+    int64 padded sampler slots) stay bit-exact: 12 tiny batches through the fused pipeline and
+    hub-heavy standalone append-unique calls."""
+    fl = 0
+    for f in flags.split("|"):
+        fl |= getattr(pkg, f)
+    p, rp, col = tiny
+    rows = providers.host_row_provider(p.graph(), rp, col)
+    feats = providers.host_feat_provider(p)
+    dsm, _ = loader.build_dsm(p, on_device=False, flags=fl)
+    pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
+    for b in range(12):
+        S = seeds.seed_nodes(p.n, p.seeds_per_batch - b * 7, presets.SEED_BASE, 300 + b)
+        rs = seeds.rng_seed(presets.RNG_BASE, 300 + b)
+        pipe.run(torch.from_numpy(S).cuda(), rs)
+        torch.cuda.synchronize()
+        _check_batch(pipe, oracle.minibatch(rows, feats, S, p.fanouts, rs), p.fanouts)
+    assert dsm.device_error() == 0
+    dsm.destroy()
+    rng = np.random.default_rng(11)
+    d2 = make_dsm(np.zeros(5001, np.int64), np.zeros(0, np.int64), max_keys=1 << 16, flags=fl)
+    for i in range(20):
+        T = rng.choice(5000, 300, replace=False).astype(np.int64)
+        nb = np.minimum((rng.pareto(1.2, 20000) * 3).astype(np.int64), 4999)   # hub-heavy
+        U, sc, dup = gpu_unique(d2, T, nb)
+        Uo, sco, dupo = oracle.append_unique(T, nb)
+        assert np.array_equal(U, Uo) and np.array_equal(sc, sco) and np.array_equal(dup, dupo), i
+    assert d2.device_error() == 0
+    d2.destroy()
