@@ -64,6 +64,8 @@ def parse():
     ap.add_argument("--no-parity", dest="parity", action="store_false",
                     help="skip the per-rank oracle check of two batches after the timed passes")
     ap.add_argument("--chase-accesses", type=int, default=100_000)
+    ap.add_argument("--x-pitch", type=int, default=None,
+                    help="diagnostics: output row pitch of X (default: DSM.out_pitch(), the row rounded up to 32 B)")
     return ap.parse_args()
 
 
@@ -485,7 +487,7 @@ class Workload:
         # the W of the feature table (NVLink share (W-1)/W of the gathered rows)
         self.w_feat = 1 if placement == "replicas" else d.world
         self.handles = [self.dsm] + [self.dsm.fork() for _ in range(P - 1)]
-        self.pipes = [pkg.MiniBatchPipeline(h, p.fanouts, S) for h in self.handles]
+        self.pipes = [pkg.MiniBatchPipeline(h, p.fanouts, S, x_pitch=args.x_pitch) for h in self.handles]
         self.streams = [torch.cuda.Stream(device=d.dev) for _ in range(P)]
         self.n_single = n_single
         self.batches = [k * d.world + d.rank for k in range(n_single + n_conc)]

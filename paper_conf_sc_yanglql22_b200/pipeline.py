@@ -40,7 +40,7 @@ PARAMS_RING = 64  # pinned staging slots for the per-batch scalars (batches enqu
 
 class MiniBatchPipeline:
     def __init__(self, dsm: DSM, fanouts, max_seeds, with_pos=False, with_dup=False, fused=True,
-                 incremental_gather=True, gather_priority=0, side_priority=0, gather_occupancy=None):
+                 incremental_gather=True, gather_priority=0, side_priority=0, gather_occupancy=None, x_pitch=None):
         self.dsm, self.fanouts, self.max_seeds = dsm, list(fanouts), max_seeds
         # None: use the handle's setting; an int: applied to this pipeline's gathers at enqueue
         self.gather_occupancy = gather_occupancy
@@ -76,9 +76,11 @@ class MiniBatchPipeline:
                 num_edges=self.counts_dev[h, 0:1], unique=torch.zeros(max(T + E, 1), **i64),
                 num_unique=self.counts_dev[h, 1:2], sub_col=torch.zeros(max(E, 1), **i32),
                 dup=torch.zeros(max(T + E, 1), **i32) if with_dup else None))
-        # X is pitched to a 32 B multiple so every row moves as whole 32 B vectors; X_rows is the
-        # [U, row_bytes] view of the feature bytes (self.X[:, :row_bytes])
-        self.X = torch.zeros((max(self.U_cap[-1], 1), dsm.out_pitch()), dtype=torch.uint8, device=dev) \
+        # X is pitched to a 32 B multiple (DSM.out_pitch) so every row moves as whole 32 B vectors; X_rows is
+        # the [U, row_bytes] view of the feature bytes (self.X[:, :row_bytes]).  x_pitch: another output
+        # pitch (a multiple of 16 >= row_bytes, e.g. 400 = dense 400 B rows, 16 B vectors; A/B only)
+        pitch = dsm.out_pitch() if x_pitch is None else x_pitch
+        self.X = torch.zeros((max(self.U_cap[-1], 1), pitch), dtype=torch.uint8, device=dev) \
             if dsm.row_bytes else None
         self.X_rows = self.X[:, :dsm.row_bytes] if self.X is not None else None
         self.graph = None

@@ -3,7 +3,7 @@
 a markdown table of the key counters per kernel and latest_gather_ncu.json (the
 gather kernel's DRAM traffic per launch, read by bench.py's roofline.traffic).
 
-    python profiles/summarize_ncu.py gpurun_out/prof_step.ncu-rep profiles/r01 [rows_gathered]
+    python profiles/summarize_ncu.py gpurun_out/prof_step.ncu-rep profiles/r02 [rows_gathered] [workload]
 """
 
 import csv
@@ -23,20 +23,32 @@ KEYS = [
     ("launch__grid_size", "grid"),
     ("launch__registers_per_thread", "regs"),
     ("launch__occupancy_limit_registers", "occ_limit_regs"),
+    ("lts__t_requests_op_atom_dot_cas.sum", "l2_cas_requests"),
+    ("lts__t_sectors_op_atom.sum", "l2_atom_sectors"),
 ]
+
+
+def sectors_per_request(r, idx):
+    """global-load sectors per request (4 = a fully used 128 B line per warp request of 32 x 4 B)."""
+    s, q = "l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum", "l1tex__t_requests_pipe_lsu_mem_global_op_ld.sum"
+    try:
+        return f"{float(r[idx[s]].replace(',', '')) / float(r[idx[q]].replace(',', '')):.2f}"
+    except (KeyError, ValueError, ZeroDivisionError):
+        return ""
 
 
 def main():
     rep, outdir = sys.argv[1], sys.argv[2]
     rows_gathered = float(sys.argv[3]) if len(sys.argv) > 3 else None
+    workload = sys.argv[4] if len(sys.argv) > 4 else "products"
     raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(io.StringIO(raw)))
     hdr, units, data = rows[0], rows[1], rows[2:]
     idx = {k: j for j, k in enumerate(hdr)}
     stall = [k for k in hdr if k.startswith("smsp__average_warps_issue_stalled_") and k.endswith("_per_issue_active.ratio")]
     os.makedirs(outdir, exist_ok=True)
-    md = ["| # | kernel | " + " | ".join(n for _, n in KEYS) + " | top stalls (cycles/issue) |",
-          "|---|---|" + "---|" * len(KEYS) + "---|"]
+    md = ["| # | kernel | " + " | ".join(n for _, n in KEYS) + " | ld_sectors_per_request | top stalls (cycles/issue) |",
+          "|---|---|" + "---|" * len(KEYS) + "---|---|"]
     gather = None
     for n, r in enumerate(data):
         name = r[idx["Kernel Name"]]
@@ -45,9 +57,9 @@ def main():
             vals.append(r[idx[k]] if k in idx else "")
         st = sorted(((float(r[idx[k]] or 0), k[len("smsp__average_warps_issue_stalled_"):-len("_per_issue_active.ratio")])
                      for k in stall), reverse=True)[:3]
-        md.append(f"| {n} | `{name[:48]}` | " + " | ".join(vals) + " | " +
+        md.append(f"| {n} | `{name[:48]}` | " + " | ".join(vals) + f" | {sectors_per_request(r, idx)} | " +
                   ", ".join(f"{s}={v:.1f}" for v, s in st) + " |")
-        if "gather_kernel" in name:
+        if "gather_kernel" in name or "gather_dense_kernel" in name:
             rd = float(r[idx["dram__bytes_read.sum"]])
             wr = float(r[idx["dram__bytes_write.sum"]])
             unit = units[idx["dram__bytes_read.sum"]]
@@ -63,8 +75,16 @@ def main():
     if gather:
         with open(os.path.join(outdir, "gather_ncu.json"), "w") as f:
             json.dump(gather, f, indent=1)
-        with open(os.path.join(os.path.dirname(outdir.rstrip("/")), "latest_gather_ncu.json"), "w") as f:
-            json.dump(gather, f, indent=1)
+        latest = os.path.join(os.path.dirname(outdir.rstrip("/")), "latest_gather_ncu.json")
+        try:
+            with open(latest) as f:
+                allw = json.load(f)
+            allw = allw if "kernel" not in allw else {}
+        except (OSError, ValueError):
+            allw = {}
+        allw[workload] = gather
+        with open(latest, "w") as f:
+            json.dump(allw, f, indent=1)
     print("\n".join(md))
 
 
