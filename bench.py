@@ -334,26 +334,33 @@ def measure_ceilings(dsm, reps=3):
     return out
 
 
+def hop_kernels(m):
+    """Kernel stages of one wg_sample_hop (the stage events the library records): the single-pass hop
+    kernel for fanout <= 32 (preceded by the compact table's cycle-restart check), else four kernels."""
+    return ("table_clear", "sample_insert_scan", "relabel") if m <= 32 else ("sample", "insert", "flag", "relabel")
+
+
 def stage_breakdown(pipe, seeds_dev, rngs, flush, ceil=None, nb=20):
-    """SURVEY 8(d) per-kernel device times of one batch (outside every timed region): each hop's
-    sampler, insert, flag scan and relabel (wg_dsm_set_stage_events: an event after every kernel, eager
-    launches, everything on one stream), then the whole gather; L2 flushed before each batch; medians.
-    With the measured ceilings, every prep kernel gets a fraction of its own bound: sampler = (T + E)
-    random accesses (row_ptr pairs + col entries) / t vs the random 8 B load rate over the col shard;
-    insert = (T + E) keys / t vs the L2 probe-CAS rate; flag and relabel = E random reads (hash word,
-    scan entry) / t vs the random 8 B load rate over an L2-sized span."""
+    """SURVEY 8(d) per-kernel device times of one batch (outside every timed region): each hop's kernels
+    (wg_dsm_set_stage_events: an event after every kernel, eager launches, everything on one stream),
+    then the whole gather; L2 flushed before each batch; medians.  With the measured ceilings, every
+    prep kernel gets a fraction of its own bound.  Per hop with T targets and E sampled edges the
+    single-pass hop kernel must at least issue T + E random loads (row_ptr pairs, col entries), T + E
+    L2 probe/CAS operations (the keys) and E random L2 reads (first positions): its bound is the SLOWEST
+    of the three at the measured rates (random 8 B loads over the col shard, probe-CAS, random 8 B
+    loads over an L2-sized span), frac = that time / the kernel's time; the relabel's E random reads
+    against the L2-span load rate."""
     import torch
     st = torch.cuda.current_stream()
     H = len(pipe.fanouts)
-    kinds = ("sample", "insert", "flag", "relabel")
-    acc = {f"hop{h}_{k}": [] for h in range(H) for k in kinds}
+    acc = {f"hop{h}_{k}": [] for h in range(H) for k in hop_kernels(pipe.fanouts[h])}
     acc["gather"] = []
     cnt = []
     for b in range(nb + 2):
         pipe.set_inputs(seeds_dev[b % len(seeds_dev)], rngs[b % len(rngs)])
         if flush is not None:
             flush.fill_(b & 0xFF)
-        evs = [[torch.cuda.Event(enable_timing=True) for _ in range(5)] for _ in range(H)]
+        evs = [[torch.cuda.Event(enable_timing=True) for _ in range(len(hop_kernels(m)) + 1)] for m in pipe.fanouts]
         for row in evs:               # create the events (torch creates them lazily at the first record)
             for e in row:
                 e.record(st)
@@ -371,34 +378,43 @@ def stage_breakdown(pipe, seeds_dev, rngs, flush, ceil=None, nb=20):
         g1.record(st)
         torch.cuda.synchronize()
         if b >= 2:
-            for h in range(H):
-                for k, kind in enumerate(kinds):
+            for h, m in enumerate(pipe.fanouts):
+                for k, kind in enumerate(hop_kernels(m)):
                     acc[f"hop{h}_{kind}"].append(evs[h][k].elapsed_time(evs[h][k + 1]))
             acc["gather"].append(g0.elapsed_time(g1))
             cnt.append(pipe.counts_dev.cpu().numpy().copy())
     out = {n: statistics.median(v) for n, v in acc.items()}
-    for h in range(H):
-        out[f"hop{h}"] = sum(out[f"hop{h}_{k}"] for k in kinds)
+    for h, m in enumerate(pipe.fanouts):
+        out[f"hop{h}"] = sum(out[f"hop{h}_{k}"] for k in hop_kernels(m))
     c = np.mean(cnt, axis=0)
     fr = {}
     if ceil:
         T = float(pipe.max_seeds)
-        for h in range(H):
+        for h, m in enumerate(pipe.fanouts):
             E, U = float(c[h, 0]), float(c[h, 1])
-            t = {k: out[f"hop{h}_{k}"] / 1e3 for k in kinds}
-            fr[f"hop{h}"] = {
-                "sample": (T + E) / t["sample"] / ceil["random_8B_loads_per_s_col_shard"],
-                "insert": (T + E) / t["insert"] / ceil["l2_cas_probe_per_s_17MB"],
-                "flag": E / t["flag"] / ceil["random_8B_loads_per_s_16MB"],
-                "relabel": E / t["relabel"] / ceil["random_8B_loads_per_s_16MB"],
-                "targets": T, "edges": E, "unique": U}
+            t = {k: out[f"hop{h}_{k}"] / 1e3 for k in hop_kernels(m)}
+            phases = {"random_loads": (T + E) / ceil["random_8B_loads_per_s_col_shard"],
+                      "l2_probe_cas": (T + E) / ceil["l2_cas_probe_per_s_17MB"],
+                      "l2_reads": E / ceil["random_8B_loads_per_s_16MB"]}
+            d = {"targets": T, "edges": E, "unique": U}
+            if m <= 32:
+                bind = max(phases, key=phases.get)
+                d["sample_insert_scan"] = phases[bind] / t["sample_insert_scan"]
+                d["sample_insert_scan_bound"] = bind
+            else:
+                d["sample"] = phases["random_loads"] / t["sample"]
+                d["insert"] = phases["l2_probe_cas"] / t["insert"]
+                d["flag"] = phases["l2_reads"] / t["flag"]
+            d["relabel"] = E / t["relabel"] / ceil["random_8B_loads_per_s_16MB"]
+            fr[f"hop{h}"] = d
             T = U
+        kinds = ("sample_insert_scan", "sample", "insert", "flag", "relabel")
         worst = min(((h, k, v) for h, d in fr.items() for k, v in d.items() if k in kinds), key=lambda x: x[2])
         fr["furthest_below"] = {"hop": worst[0], "kernel": worst[1], "frac": worst[2]}
     out["frac"] = fr
     out["note"] = ("median ms per kernel of one batch (eager launches, an event after every kernel, L2 flushed per "
-                   "batch; hop h = wg_sample_hop: sample + insert + flag-scan + relabel); frac = each kernel's "
-                   "operation rate over its measured ceiling (ceilings)")
+                   "batch; hop h = wg_sample_hop); frac = each kernel's operation rate over its measured ceiling "
+                   "(ceilings)")
     return out
 
 

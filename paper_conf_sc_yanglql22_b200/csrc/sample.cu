@@ -24,6 +24,7 @@
 // or the flag pass of Append Unique for the fused hop (unique.cu), which scans the
 // valid slots and the first occurrences together.
 #include "hash.cuh"
+#include "sample_warp.cuh"
 #include "scan.cuh"
 
 namespace wg {
@@ -35,12 +36,8 @@ constexpr int SAMPLE_THREADS = WG_SAMPLE_THREADS;
 #ifndef SAMPLE_MINB
 #define SAMPLE_MINB 6  // resident sampler blocks per SM the register allocation must allow
 #endif
-constexpr int SAMPLE_UNR_MAX = 4;
 // SAMPLE_UNR = rounds per warp, all in flight at once (1, 2 or 4; chosen per launch: small hops use
-// fewer rounds per warp and therefore more blocks / SMs)
-// Lane groups are G = max(M, SAMPLE_UNR) lanes (not a power of two), so a warp holds
-// floor(32 / G) targets per round: e.g. 6 targets for M = 5, 3 for M = 10.
-__host__ __device__ inline int sample_group(int M) { return M > SAMPLE_UNR_MAX ? M : SAMPLE_UNR_MAX; }
+// fewer rounds per warp and therefore more blocks / SMs); sample_group / the per-warp body: sample_warp.cuh
 
 struct SampleArgs {
   ShardView s;
@@ -73,7 +70,7 @@ __global__ void __launch_bounds__(SAMPLE_THREADS, SAMPLE_MINB) sample_kernel(con
   pdl_enter();
   if (CLR) clear_table_if_cycle_restarts(a.hclear, a.hwords, a.ctrl);
   __shared__ unsigned sm_chain[SAMPLE_THREADS / 32][32];
-  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int tid = threadIdx.x, warp = tid >> 5;
   int64_t nT = a.cap;
   if (a.d_n) {
     nT = *a.d_n;
@@ -83,97 +80,18 @@ __global__ void __launch_bounds__(SAMPLE_THREADS, SAMPLE_MINB) sample_kernel(con
     }
   }
   const int M = a.M;
-  const int G = sample_group(M);
-  const int TPW = 32 / G;      // targets per warp per round
-  const int g = lane / G;      // target slot within the warp (g == TPW: leftover lanes, idle)
-  const int i = lane - g * G;  // draw index
+  const int TPW = 32 / sample_group(M);
   const int64_t warp_base = ((int64_t)blockIdx.x * (SAMPLE_THREADS / 32) + warp) * (TPW * SAMPLE_UNR);
-  if (warp_base >= nT) return;  // warp-uniform
-
-  // ---- row_ptr pairs: lane u of each group fetches round u's target (all in flight)
-  int64_t my_v = -1, my_start = 0;
-  unsigned my_deg = 0;
-  if (i < SAMPLE_UNR && g < TPW) {
-    const int64_t k = warp_base + (int64_t)i * TPW + g;
-    if (k < nT) {
-      my_v = a.targets[k];
-      if (my_v < 0 || my_v >= a.s.n) {
-        latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_ID_RANGE);
-        my_v = -1;
-      } else {
-        int o;
-        int64_t l;
-        csr_owner_local(a.s, my_v, o, l);
-        const int64_t* rp = a.s.row_ptr[o] + l;
-        my_start = rp[0];
-        const int64_t d = rp[1] - my_start;
-        if (d >= (int64_t(1) << 32) || d < 0)
-          latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DEGREE);
-        else
-          my_deg = (unsigned)d;
-      }
-    }
-  }
   const unsigned long long seed = a.d_seed ? *a.d_seed : a.seed;
   const uint2 key = make_uint2((unsigned)(seed & 0xffffffffu), (unsigned)(seed >> 32));
-
-  const int64_t* src[SAMPLE_UNR];
-  int64_t dst[SAMPLE_UNR];
-  unsigned pos[SAMPLE_UNR];
-  bool ok[SAMPLE_UNR];
-#pragma unroll
-  for (int u = 0; u < SAMPLE_UNR; ++u) {
-    const int64_t k = warp_base + (int64_t)u * TPW + g;
-    const int from = g * G + u;  // the lane that loaded this round's row_ptr pair
-    const int64_t tv = __shfl_sync(FULL_MASK, my_v, from);
-    const int64_t tstart = __shfl_sync(FULL_MASK, my_start, from);
-    const unsigned N = __shfl_sync(FULL_MASK, my_deg, from);
-    const bool active = g < TPW && k < nT && tv >= 0;
-    const bool full = N <= (unsigned)M;
-    const bool draw = active && !full && i < M;
-    unsigned r = 0;
-    if (draw) {
-      const uint4 x = philox4x32_10(make_uint4((unsigned)(i >> 2), (unsigned)a.hop,
-                                               (unsigned)((uint64_t)tv & 0xffffffffu), (unsigned)((uint64_t)tv >> 32)),
-                                    key);
-      const unsigned xi = (i & 3) == 0 ? x.x : (i & 3) == 1 ? x.y : (i & 3) == 2 ? x.z : x.w;
-      r = __umulhi(xi, N - (unsigned)i);  // floor(x * (N-i) / 2^32), in [0, N-1-i]
-    }
-    const unsigned long long mkey =
-        draw ? (((unsigned long long)g << 32) | r) : (0xffffffff00000000ull | (unsigned)lane);
-    const unsigned same = __match_any_sync(FULL_MASK, mkey);
-    const unsigned below = same & ((1u << lane) - 1u);
-    const int prev = below ? 31 - __clz(below) : -1;  // previous draw with value r (Alg.1 p[q[i]-1])
-    const bool is_last = (same >> lane) == 1u;        // no later draw with value r (Alg.1 line 4)
-    sm_chain[warp][lane] = (unsigned)i;               // Alg.1 line 1: chain[i] = i
-    __syncwarp();
-    if (draw && is_last && r >= N - (unsigned)M)      // Alg.1 lines 4-5
-      sm_chain[warp][g * G + (int)(N - 1u - r)] = (unsigned)i;
-    __syncwarp();
-    unsigned c = sm_chain[warp][lane];
-    for (int s = 1; s < M; s <<= 1) c = __shfl_sync(FULL_MASK, c, g * G + (int)c);  // line 12
-    const unsigned last = N - c - 1u;                                                 // line 14
-    const unsigned lastp = __shfl_sync(FULL_MASK, last, prev >= 0 ? prev : lane);
-    __syncwarp();
-    pos[u] = full ? (unsigned)i : (prev < 0 ? r : lastp);  // lines 16-22
-    ok[u] = active && (full ? (unsigned)i < N : i < M);
-    int o = 0;
-    int64_t l;
-    if (ok[u]) csr_owner_local(a.s, tv, o, l);
-    src[u] = a.s.col[o] + tstart + pos[u];
-    dst[u] = k * M + i;
-    if (i == 0 && g < TPW && k < nT) a.cnt[k] = active ? (int32_t)min(N, (unsigned)M) : 0;
-  }
-  int64_t nb[SAMPLE_UNR];
-#pragma unroll
-  for (int u = 0; u < SAMPLE_UNR; ++u) nb[u] = ok[u] ? *src[u] : -1;
-#pragma unroll
-  for (int u = 0; u < SAMPLE_UNR; ++u) {
-    if (ok[u]) {
-      st_pad(a.nbrs_pad, a.pad32, dst[u], nb[u]);
-      if (a.pos_pad) a.pos_pad[dst[u]] = (int32_t)pos[u];
-    }
-  }
+  // padded slots k*M + i of the workspace (the scan pass that follows compacts them)
+  sample_warp<SAMPLE_UNR>(
+      a.s, a.targets, nT, M, a.hop, key, warp_base, sm_chain[warp], &a.ctrl[CTRL_ERR],
+      [&](int64_t k, int c) { a.cnt[k] = c; },
+      [&](int64_t k, int i, int64_t nb, unsigned pos) {
+        st_pad(a.nbrs_pad, a.pad32, k * M + i, nb);
+        if (a.pos_pad) a.pos_pad[k * M + i] = (int32_t)pos;
+      });
 }
 
 // ---------------------------------------------------------------- fanout > 32

@@ -302,6 +302,42 @@ __global__ void __launch_bounds__(256) hash_clear_kernel(unsigned long long* w, 
   for (int64_t i = (int64_t)blockIdx.x * 256 + threadIdx.x; i < words; i += (int64_t)gridDim.x * 256) w[i] = 0ull;
 }
 
+cudaError_t launch_hash_clear(wg_dsm* h, cudaStream_t st) {
+  return launch_pdl(hash_clear_kernel, (unsigned)h->sm_count * 4, 256, 0, st,
+                    reinterpret_cast<unsigned long long*>(h->ws.hslots), (int64_t)h->ws.hcap, (const unsigned*)h->ws.ctrl);
+}
+
+// The relabel of a hop whose scan pass left, per dense edge p, the first key-list position of its key in
+// sub_col[p] and, per first occurrence at padded neighbour slot j, its new-node index in excl[j]
+// (hop.cu): on `side` (forked from st with an event) when given.
+cudaError_t launch_relabel(wg_dsm* h, const int64_t* d_nT, int64_t capT, const int64_t* d_nE, int64_t capE,
+                           int32_t* sub_col, int32_t* dup, const int32_t* excl, cudaStream_t st, cudaStream_t side) {
+  if (capE <= 0) return cudaSuccess;
+  UniqueArgs r{};
+  r.capT = capT;
+  r.d_nT = d_nT;
+  r.capE = capE;
+  r.d_nE = d_nE;
+  r.sub_col = sub_col;
+  r.dup = dup;
+  r.excl = const_cast<int32_t*>(excl);
+  r.ctrl = h->ws.ctrl;
+  const int64_t max_blocks = (int64_t)h->sm_count * PREP_BPS;
+  int64_t rb = (capE + UQ_THREADS - 1) / UQ_THREADS;
+  rb = rb > max_blocks ? max_blocks : rb;
+  cudaStream_t rs = st;
+  if (side && side != st) {
+    cudaError_t e = cudaEventRecord(h->fork_event, st);
+    if (e != cudaSuccess) return e;
+    e = cudaStreamWaitEvent(side, h->fork_event, 0);
+    if (e != cudaSuccess) return e;
+    rs = side;
+  }
+  unique_relabel_kernel<<<(unsigned)rb, UQ_THREADS, 0, rs>>>(r);
+  stage_mark(h, rs);
+  return cudaGetLastError();
+}
+
 template <bool C>
 static cudaError_t launch_insert_flag(wg_dsm* h, bool padded, int items, int64_t ib, unsigned fb, const UniqueArgs& a,
                                       cudaStream_t st) {
@@ -334,10 +370,7 @@ static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, c
   // about as many lines as it has keys instead of random lines all over the table sized for the
   // largest hop.  Slots outside the prefix, or left by earlier calls, carry older epochs and read as
   // empty.
-  int64_t hc = (int64_t)(HASH_FACTOR * (double)(a.capT + a.capE)) + 8;
-  hc = std::max<int64_t>(hc, HASH_MIN_SLOTS);
-  hc = std::min<int64_t>((hc + 7) / 8 * 8, h->ws.hcap);
-  a.ht = HashTable{h->ws.hslots, (unsigned long long)hc, h->ws.compact};
+  a.ht = HashTable{h->ws.hslots, (unsigned long long)table_prefix(h, a.capT + a.capE), h->ws.compact};
   a.status = h->ws.status_unique;
   a.ctrl = h->ws.ctrl;
   a.n = h->n;
@@ -352,8 +385,7 @@ static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, c
   const unsigned fb = (unsigned)(a.capE > 0 ? (a.capE + tile - 1) / tile : 1);
   cudaError_t e;
   if (!padded && h->ws.compact) {
-    e = launch_pdl(hash_clear_kernel, (unsigned)h->sm_count * 4, 256, 0, st,
-                   reinterpret_cast<unsigned long long*>(h->ws.hslots), (int64_t)h->ws.hcap, (const unsigned*)h->ws.ctrl);
+    e = launch_hash_clear(h, st);
     if (e != cudaSuccess) return e;
   }
   if (h->ws.compact)
@@ -409,6 +441,11 @@ cudaError_t launch_hop(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t*
                        const uint64_t* d_seed, int hop, int64_t* out_row_ptr, int64_t* out_nbrs, int32_t* out_pos,
                        int64_t* d_num_edges, int64_t* U, int64_t* d_nU, int32_t* sub_col, int32_t* dup,
                        cudaStream_t st, cudaStream_t side) {
+#ifndef WG_HOP_UNFUSED  // A/B build: the four-kernel hop below for every fanout
+  if (fanout <= 32)     // one single-pass kernel (hop.cu); larger fanouts use the block sampler
+    return launch_hop_fused(h, T, capT, d_nT, fanout, seed, d_seed, hop, out_row_ptr, out_nbrs, out_pos, d_num_edges,
+                            U, d_nU, sub_col, dup, st, side);
+#endif
   h->stage_i = 0;
   cudaError_t e = launch_sample_padded(h, T, capT, d_nT, fanout, seed, d_seed, hop, out_pos != nullptr, st);
   if (e != cudaSuccess) return e;

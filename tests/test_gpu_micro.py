@@ -71,23 +71,25 @@ def test_micro_ceilings_plausible():
     assert lib().wg_micro_atomics(P(table), table.numel(), 3, 8, 8, P(sink), None, st) != 0
 
 
-def test_stage_events_split_a_hop():
-    """wg_dsm_set_stage_events: the events recorded after the sampler, insert, flag scan and relabel of a
-    hop are ordered, and together they cover the hop."""
+@pytest.mark.parametrize("fanout,stages", [(10, 3), (40, 4)])
+def test_stage_events_split_a_hop(fanout, stages):
+    """wg_dsm_set_stage_events: the events recorded after the kernels of a hop (table clear, single-pass
+    hop kernel, relabel for fanout <= 32; sampler, insert, flag scan, relabel above) are ordered and
+    together cover the hop."""
     p = presets.get("tiny")
-    dsm, _ = loader.build_dsm(p, on_device=False)
+    dsm, _ = loader.build_dsm(p, on_device=False, extra_keys=p.seeds_per_batch * (1 + fanout))
     S = torch.from_numpy(seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 1)).cuda()
-    evs = [torch.cuda.Event(enable_timing=True) for _ in range(5)]
+    evs = [torch.cuda.Event(enable_timing=True) for _ in range(stages + 1)]
     for e in evs:
         e.record()
     evs[0].record()
     dsm.set_stage_events(evs[1:])
-    o = dsm.sample_hop(S, p.fanouts[0], 5, 0)
+    o = dsm.sample_hop(S, fanout, 5, 0)
     dsm.set_stage_events([])
     end = torch.cuda.Event(enable_timing=True)
     end.record()
     torch.cuda.synchronize()
-    parts = [evs[k].elapsed_time(evs[k + 1]) for k in range(4)]
+    parts = [evs[k].elapsed_time(evs[k + 1]) for k in range(stages)]
     assert all(x >= 0 for x in parts), parts
     assert sum(parts) <= evs[0].elapsed_time(end) + 1e-3
     assert int(o["num_unique"].item()) > len(S)
