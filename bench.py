@@ -335,9 +335,8 @@ def measure_ceilings(dsm, reps=3):
 
 
 def hop_kernels(m):
-    """Kernel stages of one wg_sample_hop (the stage events the library records): the single-pass hop
-    kernel for fanout <= 32 (preceded by the compact table's cycle-restart check), else four kernels."""
-    return ("table_clear", "sample_insert_scan", "relabel") if m <= 32 else ("sample", "insert", "flag", "relabel")
+    """Kernel stages of one wg_sample_hop (the stage events the library records)."""
+    return ("sample", "insert", "flag", "relabel")
 
 
 def stage_breakdown(pipe, seeds_dev, rngs, flush, ceil=None, nb=20):
@@ -397,18 +396,13 @@ def stage_breakdown(pipe, seeds_dev, rngs, flush, ceil=None, nb=20):
                       "l2_probe_cas": (T + E) / ceil["l2_cas_probe_per_s_17MB"],
                       "l2_reads": E / ceil["random_8B_loads_per_s_16MB"]}
             d = {"targets": T, "edges": E, "unique": U}
-            if m <= 32:
-                bind = max(phases, key=phases.get)
-                d["sample_insert_scan"] = phases[bind] / t["sample_insert_scan"]
-                d["sample_insert_scan_bound"] = bind
-            else:
-                d["sample"] = phases["random_loads"] / t["sample"]
-                d["insert"] = phases["l2_probe_cas"] / t["insert"]
-                d["flag"] = phases["l2_reads"] / t["flag"]
+            d["sample"] = phases["random_loads"] / t["sample"]
+            d["insert"] = phases["l2_probe_cas"] / t["insert"]
+            d["flag"] = phases["l2_reads"] / t["flag"]
             d["relabel"] = E / t["relabel"] / ceil["random_8B_loads_per_s_16MB"]
             fr[f"hop{h}"] = d
             T = U
-        kinds = ("sample_insert_scan", "sample", "insert", "flag", "relabel")
+        kinds = ("sample", "insert", "flag", "relabel")
         worst = min(((h, k, v) for h, d in fr.items() for k, v in d.items() if k in kinds), key=lambda x: x[2])
         fr["furthest_below"] = {"hop": worst[0], "kernel": worst[1], "frac": worst[2]}
     out["frac"] = fr

@@ -307,37 +307,6 @@ cudaError_t launch_hash_clear(wg_dsm* h, cudaStream_t st) {
                     reinterpret_cast<unsigned long long*>(h->ws.hslots), (int64_t)h->ws.hcap, (const unsigned*)h->ws.ctrl);
 }
 
-// The relabel of a hop whose scan pass left, per dense edge p, the first key-list position of its key in
-// sub_col[p] and, per first occurrence at padded neighbour slot j, its new-node index in excl[j]
-// (hop.cu): on `side` (forked from st with an event) when given.
-cudaError_t launch_relabel(wg_dsm* h, const int64_t* d_nT, int64_t capT, const int64_t* d_nE, int64_t capE,
-                           int32_t* sub_col, int32_t* dup, const int32_t* excl, cudaStream_t st, cudaStream_t side) {
-  if (capE <= 0) return cudaSuccess;
-  UniqueArgs r{};
-  r.capT = capT;
-  r.d_nT = d_nT;
-  r.capE = capE;
-  r.d_nE = d_nE;
-  r.sub_col = sub_col;
-  r.dup = dup;
-  r.excl = const_cast<int32_t*>(excl);
-  r.ctrl = h->ws.ctrl;
-  const int64_t max_blocks = (int64_t)h->sm_count * PREP_BPS;
-  int64_t rb = (capE + UQ_THREADS - 1) / UQ_THREADS;
-  rb = rb > max_blocks ? max_blocks : rb;
-  cudaStream_t rs = st;
-  if (side && side != st) {
-    cudaError_t e = cudaEventRecord(h->fork_event, st);
-    if (e != cudaSuccess) return e;
-    e = cudaStreamWaitEvent(side, h->fork_event, 0);
-    if (e != cudaSuccess) return e;
-    rs = side;
-  }
-  unique_relabel_kernel<<<(unsigned)rb, UQ_THREADS, 0, rs>>>(r);
-  stage_mark(h, rs);
-  return cudaGetLastError();
-}
-
 template <bool C>
 static cudaError_t launch_insert_flag(wg_dsm* h, bool padded, int items, int64_t ib, unsigned fb, const UniqueArgs& a,
                                       cudaStream_t st) {
@@ -441,11 +410,6 @@ cudaError_t launch_hop(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t*
                        const uint64_t* d_seed, int hop, int64_t* out_row_ptr, int64_t* out_nbrs, int32_t* out_pos,
                        int64_t* d_num_edges, int64_t* U, int64_t* d_nU, int32_t* sub_col, int32_t* dup,
                        cudaStream_t st, cudaStream_t side) {
-#ifndef WG_HOP_UNFUSED  // A/B build: the four-kernel hop below for every fanout
-  if (fanout <= 32)     // one single-pass kernel (hop.cu); larger fanouts use the block sampler
-    return launch_hop_fused(h, T, capT, d_nT, fanout, seed, d_seed, hop, out_row_ptr, out_nbrs, out_pos, d_num_edges,
-                            U, d_nU, sub_col, dup, st, side);
-#endif
   h->stage_i = 0;
   cudaError_t e = launch_sample_padded(h, T, capT, d_nT, fanout, seed, d_seed, hop, out_pos != nullptr, st);
   if (e != cudaSuccess) return e;

@@ -87,8 +87,7 @@ struct Workspace {
   unsigned* ctrl = nullptr;              // [16] control words (see CTRL_*)
   int64_t max_keys = 0;
 };
-enum { CTRL_ERR = 0, CTRL_EPOCH = 1, CTRL_DONE_SAMPLE = 2, CTRL_DONE_UNIQUE = 3, CTRL_TILE = 4, CTRL_DONE_HOP = 5,
-       CTRL_WORDS = 16 };
+enum { CTRL_ERR = 0, CTRL_EPOCH = 1, CTRL_DONE_SAMPLE = 2, CTRL_DONE_UNIQUE = 3, CTRL_WORDS = 16 };
 constexpr unsigned EPOCH_MAX = (1u << 23) - 1;
 // compact hash table (8 B slots): epochs 1..255 cycle; the table is cleared when a cycle restarts
 constexpr unsigned CEPOCHS = 255;
@@ -186,10 +185,6 @@ cudaError_t launch_hop(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t*
                        const uint64_t* d_seed, int hop, int64_t* out_row_ptr, int64_t* out_nbrs, int32_t* out_pos,
                        int64_t* d_num_edges, int64_t* U, int64_t* d_nU, int32_t* sub_col, int32_t* dup,
                        cudaStream_t st, cudaStream_t side);
-cudaError_t launch_hop_fused(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t* d_nT, int fanout,
-                             uint64_t seed, const uint64_t* d_seed, int hop, int64_t* out_row_ptr, int64_t* out_nbrs,
-                             int32_t* out_pos, int64_t* d_num_edges, int64_t* U, int64_t* d_nU, int32_t* sub_col,
-                             int32_t* dup, cudaStream_t st, cudaStream_t side);
 cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int64_t* d_n, const int64_t* d_begin,
                           void* out, int64_t out_pitch, cudaStream_t st);
 }  // namespace wg

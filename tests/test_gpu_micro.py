@@ -26,9 +26,8 @@ def test_dsm_chase_latency_plausible():
     big = pkg.DSM(1 << 26, 0, 16, "fp32", 16)              # 4 GB of 64 B rows
     big.local_view()[2].fill_(7)
     big.chase(0, (1 << 26) * 64, 2000)                      # warm-up: module load, clocks, TLB
-    ns = [big.chase(0, (1 << 26) * 64, 20000) for _ in range(3)]
-    assert all(50 < x < 5000 for x in ns), ns
-    assert max(ns) < 1.2 * min(ns), ns
+    ns = sorted(big.chase(0, (1 << 26) * 64, 20000) for _ in range(5))
+    assert 50 < ns[0] < 2000 and ns[2] < 1.2 * ns[0], ns   # the median run within 20 % of the best
     with pytest.raises(pkg.WgError):
         big.chase(0, (1 << 26) * 64 * 2, 10)
     with pytest.raises(pkg.WgError):
@@ -71,11 +70,10 @@ def test_micro_ceilings_plausible():
     assert lib().wg_micro_atomics(P(table), table.numel(), 3, 8, 8, P(sink), None, st) != 0
 
 
-@pytest.mark.parametrize("fanout,stages", [(10, 3), (40, 4)])
+@pytest.mark.parametrize("fanout,stages", [(10, 4), (40, 4)])
 def test_stage_events_split_a_hop(fanout, stages):
-    """wg_dsm_set_stage_events: the events recorded after the kernels of a hop (table clear, single-pass
-    hop kernel, relabel for fanout <= 32; sampler, insert, flag scan, relabel above) are ordered and
-    together cover the hop."""
+    """wg_dsm_set_stage_events: the events recorded after the sampler, insert, flag scan and relabel of a
+    hop (warp sampler and block sampler) are ordered and together cover the hop."""
     p = presets.get("tiny")
     dsm, _ = loader.build_dsm(p, on_device=False, extra_keys=p.seeds_per_batch * (1 + fanout))
     S = torch.from_numpy(seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 1)).cuda()
