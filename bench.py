@@ -64,6 +64,7 @@ def parse():
     ap.add_argument("--no-parity", dest="parity", action="store_false",
                     help="skip the per-rank oracle check of two batches after the timed passes")
     ap.add_argument("--chase-accesses", type=int, default=100_000)
+    ap.add_argument("--latency-spans", default="1,8,16,32,64,128", help="--latency: spans in GiB (comma list)")
     ap.add_argument("--x-pitch", type=int, default=None,
                     help="diagnostics: output row pitch of X (default: DSM.out_pitch(), the row rounded up to 32 B)")
     return ap.parse_args()
@@ -1007,8 +1008,8 @@ def bench_latency(args):
     d = Dist()
     free, _ = torch.cuda.mem_get_info()
     gib = 1 << 30
-    spans = [s * gib for s in (1, 8, 16, 32, 64, 128)]
-    spans = [sp for sp in spans if d.all_true(sp < 0.85 * free)]
+    spans = [int(float(s) * gib) // 512 * 512 for s in args.latency_spans.split(",")]
+    spans = [sp for sp in spans if d.all_true(sp < 0.85 * free / max(1, d.world if d.shared_gpu else 1))]
     rows_per_rank = max(spans) // 512
     dsm = pkg.DSM(rows_per_rank * d.world, 0, 128, "fp32", 1, rank=d.rank, world_size=d.world, device=d.local,
                   allgather=d.ag)   # 512 B rows, filled with generator bits
@@ -1019,7 +1020,7 @@ def bench_latency(args):
     peer_ok = d.world > 1 and not d.shared_gpu
     if d.rank == 0:
         for sp in spans:
-            row = {"span_gb": sp / gib}
+            row = {"span_gb": round(sp / gib, 4)}
             for name, r in (("local_ns", 0), ("peer_ns", 1)):
                 if r >= d.world:
                     row[name] = None

@@ -135,3 +135,42 @@ def test_bench_torchrun_two_ranks(placement):
     assert d["config"]["parallelism"].startswith({"dsm": "dsm-w2", "csr-replicated": "csr-replicated-w2",
                                                   "replicas": "replicas-x2"}[placement])
     assert d["parity"]["ok"] is True and d["parity"]["ranks"] == 2 and d["parity"]["batches"] == 2
+
+
+def _torchrun_line(args, port):
+    import json
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node", "2", "--master-addr",
+           "127.0.0.1", "--master-port", str(port), os.path.join(ROOT, "bench.py")] + args
+    r = subprocess.run(cmd, cwd=ROOT, capture_output=True, text=True, timeout=600)
+    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-3000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1, r.stdout
+    return json.loads(lines[0])
+
+
+def test_sweep_two_ranks_byte_checked():
+    """config-4 sweep under torchrun: the table row-sharded over 2 ranks, each gathering its own ids at once,
+    every cell byte-checked against the generator on both ranks."""
+    d = _torchrun_line(["--sweep", "--sweep-rows", "200000", "--sweep-ids", "20000", "--sweep-cells", "fp32:100,fp16:64",
+                        "--steps", "2"], 29700 + os.getpid() % 300)
+    assert d["n_gpus"] == 2 and len(d["cells"]) == 2
+    for c in d["cells"]:
+        assert c["bytes_ok"] is True and c["ms"] > 0 and c["busbw_gbs_per_gpu"] == c["algo_gbs_per_gpu"] / 2
+
+
+def test_compare_gather_two_ranks():
+    """NEXT #1 under torchrun (2 ranks sharing the GPU: gloo all-to-alls through the host): both gathers
+    byte-checked, and the line says it is not the paper's experiment."""
+    d = _torchrun_line(["--compare-gather", "--config", "tiny", "--sweep-ids", "20000", "--steps", "2"],
+                       29720 + os.getpid() % 300)
+    assert d["n_gpus"] == 2 and d["is_paper_experiment"] is False and d["note"]
+    for r in d["results"].values():
+        assert r["bytes_ok"] is True
+
+
+def test_latency_two_ranks_peer_column():
+    """Table I analogue under torchrun: rank 0 chases its own shard and rank 1's (labelled as local HBM when
+    the ranks share a GPU)."""
+    d = _torchrun_line(["--latency", "--latency-spans", "0.0625", "--chase-accesses", "2000"], 29740 + os.getpid() % 300)
+    row = d["spans"][0]
+    assert row["local_ns"] > 0 and row["peer_ns"] > 0 and "peer_note" in row
