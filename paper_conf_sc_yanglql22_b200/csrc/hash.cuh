@@ -6,7 +6,7 @@
 // position.  A key from an older epoch reads as an empty slot and an older
 // value always loses an atomicMin against the current epoch, so the table is never
 // cleared between calls.  Linear probing, fmix64 hash mapped onto [0, size) by a multiply-high,
-// load factor <= 1 / WG_HASH_FACTOR at the capacity bound.
+// load factor <= 1 / HASH_FACTOR (2) at the capacity bound.
 #pragma once
 
 #include "device_util.cuh"
