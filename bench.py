@@ -65,6 +65,8 @@ def parse():
                     help="skip the per-rank oracle check of two batches after the timed passes")
     ap.add_argument("--chase-accesses", type=int, default=100_000)
     ap.add_argument("--latency-spans", default="1,8,16,32,64,128", help="--latency: spans in GiB (comma list)")
+    ap.add_argument("--col64", action="store_true",
+                    help="store col_idx as int64 (default: uint32, WG_DSM_COL32, whenever the node ids fit)")
     ap.add_argument("--x-pitch", type=int, default=None,
                     help="diagnostics: output row pitch of X (default: DSM.out_pitch(), the row rounded up to 32 B)")
     return ap.parse_args()
@@ -488,12 +490,14 @@ class Workload:
         self.p, self.d, self.P, self.placement = p, d, P, placement
         S = p.seeds_per_batch
         t0 = time.perf_counter()
+        col32 = False if args.col64 else None   # None: the loader's default (uint32 when the ids fit)
         if placement == "replicas":   # every rank its own whole copy (a W=1 DSM); batches still b = r mod W
-            self.dsm, self.info = loader.build_dsm(p, rank=0, world=1, device=d.local, allgather=None)
+            self.dsm, self.info = loader.build_dsm(p, rank=0, world=1, device=d.local, allgather=None, col32=col32)
         else:
             flags = pkg.WG_DSM_CSR_REPLICATED if placement == "csr-replicated" else 0
             self.dsm, self.info = loader.build_dsm(p, rank=d.rank, world=d.world, device=d.local, allgather=d.ag,
-                                                   flags=flags)
+                                                   flags=flags, col32=col32)
+        self.info["col_idx_bytes"] = 4 if self.dsm.flags & pkg.WG_DSM_COL32 else 8
         self.setup_s = time.perf_counter() - t0
         # the W of the feature table (NVLink share (W-1)/W of the gathered rows)
         self.w_feat = 1 if placement == "replicas" else d.world
@@ -1115,7 +1119,7 @@ def bench_compare_gather(args):
     d = Dist()
     p = presets.get(args.config)
     dsm, _ = loader.build_dsm(p, rank=d.rank, world=d.world, device=d.local, allgather=d.ag)
-    dg = DistributedGather(dsm)
+    dg = DistributedGather(dsm)  # (the CSR is not read here)
     ids_np = seeds.gather_ids(p.n, args.sweep_ids, presets.SEED_BASE, d.rank)
     ids = torch.from_numpy(ids_np).to(d.dev)
     out = torch.empty((ids.numel(), dsm.row_bytes), dtype=torch.uint8, device=d.dev)

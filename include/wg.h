@@ -77,6 +77,9 @@ typedef enum { WG_F32 = 0, WG_F16 = 1, WG_BF16 = 2 } wg_dtype;
                                        CSR (row_ptr int64[num_nodes+1], col_idx int64[local_num_edges =
                                        all E]) and samples locally; only the feature table is row-sharded
                                        (o(v) = v mod W) and read over NVLink.  Results are identical. */
+#define WG_DSM_COL32          0x10u /* col_idx entries stored as uint32 (needs num_nodes <= 2^32): half the
+                                       bytes of every sampled line; wg_dsm_local_view's d_col_idx then points
+                                       to uint32 entries (ids in every op stay int64) */
 
 /* Allgather of host bytes across the W ranks of the DSM ("an
  * AllGather pattern communication is performed so that each process can get all
@@ -107,7 +110,8 @@ typedef struct {
 
 /* Create the DSM (section III-B).  COLLECTIVE over the W ranks.
  * Each rank allocates its shard slab on its device -- row_ptr int64[n_local+1] (int64[num_nodes+1]
- * with WG_DSM_CSR_REPLICATED), col_idx int64[local_num_edges], features [n_local][row stride] (+ a tail region for the
+ * with WG_DSM_CSR_REPLICATED), col_idx int64[local_num_edges] (uint32 with WG_DSM_COL32), features
+ * [n_local][row stride] (+ a tail region for the
  * split row layout, see wg_dsm_feat_layout) -- exports a CUDA IPC handle, allgathers the
  * handles (L100), opens every peer's handle (L100-106; same-process peers are used
  * directly) and keeps the W base pointers as the "memory pointer table" (L106),

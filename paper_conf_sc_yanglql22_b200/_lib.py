@@ -29,6 +29,7 @@ WG_DSM_WHOLE_ROWS = 0x1
 WG_DSM_WIDE_HASH = 0x2
 WG_DSM_PAD64 = 0x4
 WG_DSM_CSR_REPLICATED = 0x8
+WG_DSM_COL32 = 0x10
 
 
 class WgError(RuntimeError):

@@ -180,8 +180,11 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
     return fail(WG_ERR_INVALID_ARG, "sizes out of range (num_nodes < 2^40, max_batch_keys < 2^31)");
   if (d->feat_dtype < WG_F32 || d->feat_dtype > WG_BF16) return fail(WG_ERR_INVALID_ARG, "feat_dtype");
   if (d->world_size > 1 && !d->allgather) return fail(WG_ERR_INVALID_ARG, "allgather callback required for W > 1");
-  if ((d->flags & ~(WG_DSM_WHOLE_ROWS | WG_DSM_WIDE_HASH | WG_DSM_PAD64 | WG_DSM_CSR_REPLICATED)) || d->reserved)
+  if ((d->flags & ~(WG_DSM_WHOLE_ROWS | WG_DSM_WIDE_HASH | WG_DSM_PAD64 | WG_DSM_CSR_REPLICATED | WG_DSM_COL32)) ||
+      d->reserved)
     return fail(WG_ERR_INVALID_ARG, "unknown flags");
+  if ((d->flags & WG_DSM_COL32) && d->num_nodes > (int64_t(1) << 32))
+    return fail(WG_ERR_INVALID_ARG, "WG_DSM_COL32 needs num_nodes <= 2^32");
 
   WG_CUDA_TRY(cudaSetDevice(d->device));
   int major = 0, minor = 0, sms = 0;
@@ -210,7 +213,8 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
   const bool csr_rep = (h->flags & WG_DSM_CSR_REPLICATED) != 0;
   const int64_t csr_rows = csr_rep ? h->n : h->n_local;
   const int64_t off_col = round_up((csr_rows + 1) * 8, 256);
-  const int64_t off_feat = round_up(off_col + h->e_local * 8, 256);
+  const int64_t col_bytes = (h->flags & WG_DSM_COL32) ? 4 : 8;
+  const int64_t off_feat = round_up(off_col + h->e_local * col_bytes, 256);
   const int64_t off_tail = round_up(off_feat + h->n_local * h->feat_stride, 256);
   h->slab_bytes = (size_t)round_up(off_tail + h->n_local * h->tail_pitch, 256);
   if (cudaMalloc(&h->slab, h->slab_bytes) != cudaSuccess) {
@@ -317,7 +321,7 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
     }
     uint8_t* b = static_cast<uint8_t*>(h->peer_base[r]);
     h->view.row_ptr[r] = reinterpret_cast<const int64_t*>(b);
-    h->view.col[r] = reinterpret_cast<const int64_t*>(b + all[r].off_col);
+    h->view.col[r] = b + all[r].off_col;
     h->view.feat[r] = b + all[r].off_feat;
     h->view.tail[r] = h->tail_pitch ? b + all[r].off_tail : nullptr;
   }
@@ -330,6 +334,7 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
   for (int k = 0; k <= 3; ++k)
     if ((1 << k) == h->world) h->view.log2w = k;
   h->view.csr_rank = csr_rep ? h->rank : -1;
+  h->view.col32 = (h->flags & WG_DSM_COL32) ? 1 : 0;
   // Zero this rank's row_ptr so an unfilled shard reads as degree 0.
   if (cudaMemset(h->slab, 0, (csr_rows + 1) * 8) != cudaSuccess) {
     cudaGetLastError();
@@ -348,7 +353,7 @@ wg_status wg_dsm_local_view(wg_dsm_t h, int64_t** row_ptr, int64_t** col, void**
                             int64_t* stride) {
   if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
   if (row_ptr) *row_ptr = const_cast<int64_t*>(h->view.row_ptr[h->rank]);
-  if (col) *col = const_cast<int64_t*>(h->view.col[h->rank]);
+  if (col) *col = const_cast<int64_t*>(static_cast<const int64_t*>(h->view.col[h->rank]));
   if (feat) *feat = const_cast<uint8_t*>(h->view.feat[h->rank]);
   if (n_local_rows) *n_local_rows = h->n_local;
   if (stride) *stride = h->feat_stride;

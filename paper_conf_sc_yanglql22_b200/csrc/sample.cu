@@ -65,7 +65,7 @@ __device__ __noinline__ void clear_table_if_cycle_restarts(unsigned long long* w
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < words; i += stride) w[i] = 0ull;
 }
 
-template <int SAMPLE_UNR, bool CLR>
+template <int SAMPLE_UNR, bool CLR, bool COL32>
 __global__ void __launch_bounds__(SAMPLE_THREADS, SAMPLE_MINB) sample_kernel(const SampleArgs a) {
   pdl_enter();
   if (CLR) clear_table_if_cycle_restarts(a.hclear, a.hwords, a.ctrl);
@@ -85,7 +85,7 @@ __global__ void __launch_bounds__(SAMPLE_THREADS, SAMPLE_MINB) sample_kernel(con
   const unsigned long long seed = a.d_seed ? *a.d_seed : a.seed;
   const uint2 key = make_uint2((unsigned)(seed & 0xffffffffu), (unsigned)(seed >> 32));
   // padded slots k*M + i of the workspace (the scan pass that follows compacts them)
-  sample_warp<SAMPLE_UNR>(
+  sample_warp<SAMPLE_UNR, COL32>(
       a.s, a.targets, nT, M, a.hop, key, warp_base, sm_chain[warp], &a.ctrl[CTRL_ERR],
       [&](int64_t k, int c) { a.cnt[k] = c; },
       [&](int64_t k, int i, int64_t nb, unsigned pos) {
@@ -100,7 +100,7 @@ __global__ void __launch_bounds__(SAMPLE_THREADS, SAMPLE_MINB) sample_kernel(con
 // (L118): Algorithm 1 exactly as listed (L122-158), with parallel_sort = a block bitonic
 // sort of the packed 64-bit keys (r << 32 | i) (L118-120) in shared memory, chain / q /
 // last in shared memory and path doubling as ceil(log2 M) synchronous rounds.
-template <int BT, bool CLR>
+template <int BT, bool CLR, bool COL32>
 __global__ void __launch_bounds__(BT) sample_block_kernel(const SampleArgs a) {
   pdl_enter();
   if (CLR) clear_table_if_cycle_restarts(a.hclear, a.hwords, a.ctrl);
@@ -147,10 +147,10 @@ __global__ void __launch_bounds__(BT) sample_block_kernel(const SampleArgs a) {
   int o;
   int64_t l;
   csr_owner_local(a.s, v, o, l);
-  const int64_t* col = a.s.col[o] + s_start;
+  const int64_t cbase = s_start;
   if (N <= (unsigned)M) {  // L118: all of N neighbours, CSR order (A5)
     for (unsigned j = i; j < N; j += BT) {
-      st_pad(a.nbrs_pad, a.pad32, k * M + j, col[j]);
+      st_pad(a.nbrs_pad, a.pad32, k * M + j, ld_col<COL32>(a.s, o, cbase + j));
       if (a.pos_pad) a.pos_pad[k * M + j] = (int32_t)j;
     }
     return;
@@ -212,7 +212,7 @@ __global__ void __launch_bounds__(BT) sample_block_kernel(const SampleArgs a) {
       res = s_r[i];
     else
       res = s_last[(unsigned)(s_key[qi - 1] & 0xffffffffu)];
-    st_pad(a.nbrs_pad, a.pad32, k * M + i, col[res]);
+    st_pad(a.nbrs_pad, a.pad32, k * M + i, ld_col<COL32>(a.s, o, cbase + res));
     if (a.pos_pad) a.pos_pad[k * M + i] = (int32_t)res;
   }
 }
@@ -282,13 +282,20 @@ __global__ void __launch_bounds__(COMPACT_THREADS) sample_compact_kernel(const C
   }
 }
 
-template <bool CLR>
+template <bool CLR, bool COL32>
 static cudaError_t launch_block_sampler(int fanout, unsigned blocks, const SampleArgs& a, cudaStream_t st) {
-  if (fanout <= 64) return launch_pdl(sample_block_kernel<64, CLR>, blocks, 64, 0, st, a);
-  if (fanout <= 128) return launch_pdl(sample_block_kernel<128, CLR>, blocks, 128, 0, st, a);
-  if (fanout <= 256) return launch_pdl(sample_block_kernel<256, CLR>, blocks, 256, 0, st, a);
-  if (fanout <= 512) return launch_pdl(sample_block_kernel<512, CLR>, blocks, 512, 0, st, a);
-  return launch_pdl(sample_block_kernel<1024, CLR>, blocks, 1024, 0, st, a);
+  if (fanout <= 64) return launch_pdl(sample_block_kernel<64, CLR, COL32>, blocks, 64, 0, st, a);
+  if (fanout <= 128) return launch_pdl(sample_block_kernel<128, CLR, COL32>, blocks, 128, 0, st, a);
+  if (fanout <= 256) return launch_pdl(sample_block_kernel<256, CLR, COL32>, blocks, 256, 0, st, a);
+  if (fanout <= 512) return launch_pdl(sample_block_kernel<512, CLR, COL32>, blocks, 512, 0, st, a);
+  return launch_pdl(sample_block_kernel<1024, CLR, COL32>, blocks, 1024, 0, st, a);
+}
+
+template <bool CLR, bool COL32>
+static cudaError_t launch_warp_sampler(int unr, unsigned blocks, const SampleArgs& a, cudaStream_t st) {
+  if (unr == 4) return launch_pdl(sample_kernel<4, CLR, COL32>, blocks, SAMPLE_THREADS, 0, st, a);
+  if (unr == 2) return launch_pdl(sample_kernel<2, CLR, COL32>, blocks, SAMPLE_THREADS, 0, st, a);
+  return launch_pdl(sample_kernel<1, CLR, COL32>, blocks, SAMPLE_THREADS, 0, st, a);
 }
 
 cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap, const int64_t* d_n, int fanout,
@@ -311,8 +318,10 @@ cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap,
   a.hwords = h->ws.hcap;
   if (fanout > 32) {  // block per target (Algorithm 1 with a block sort)
     const unsigned blocks = (unsigned)(cap > 0 ? cap : 1);
-    if (a.hclear) return launch_block_sampler<true>(fanout, blocks, a, st);
-    return launch_block_sampler<false>(fanout, blocks, a, st);
+    if (a.s.col32) return a.hclear ? launch_block_sampler<true, true>(fanout, blocks, a, st)
+                                   : launch_block_sampler<false, true>(fanout, blocks, a, st);
+    return a.hclear ? launch_block_sampler<true, false>(fanout, blocks, a, st)
+                    : launch_block_sampler<false, false>(fanout, blocks, a, st);
   }
   const int G = sample_group(fanout);
   const int tpw = 32 / G;
@@ -320,14 +329,9 @@ cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap,
   while (unr > 1 && cap < (int64_t)(SAMPLE_THREADS / 32) * tpw * unr * 2 * h->sm_count) unr >>= 1;
   const int64_t tile = (int64_t)(SAMPLE_THREADS / 32) * tpw * unr;
   const unsigned blocks = (unsigned)(cap > 0 ? (cap + tile - 1) / tile : 1);
-  if (a.hclear) {
-    if (unr == 4) return launch_pdl(sample_kernel<4, true>, blocks, SAMPLE_THREADS, 0, st, a);
-    if (unr == 2) return launch_pdl(sample_kernel<2, true>, blocks, SAMPLE_THREADS, 0, st, a);
-    return launch_pdl(sample_kernel<1, true>, blocks, SAMPLE_THREADS, 0, st, a);
-  }
-  if (unr == 4) return launch_pdl(sample_kernel<4, false>, blocks, SAMPLE_THREADS, 0, st, a);
-  if (unr == 2) return launch_pdl(sample_kernel<2, false>, blocks, SAMPLE_THREADS, 0, st, a);
-  return launch_pdl(sample_kernel<1, false>, blocks, SAMPLE_THREADS, 0, st, a);
+  if (a.s.col32) return a.hclear ? launch_warp_sampler<true, true>(unr, blocks, a, st)
+                                 : launch_warp_sampler<false, true>(unr, blocks, a, st);
+  return a.hclear ? launch_warp_sampler<true, false>(unr, blocks, a, st) : launch_warp_sampler<false, false>(unr, blocks, a, st);
 }
 
 cudaError_t launch_sample(wg_dsm* h, const int64_t* targets, int64_t cap, const int64_t* d_n, int fanout,

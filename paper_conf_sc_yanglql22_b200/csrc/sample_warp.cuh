@@ -25,7 +25,7 @@ __host__ __device__ inline int sample_group(int M) { return M > SAMPLE_UNR_MAX ?
 // emit_cnt(k, c) is called once per target k < nT (c = min(M, deg), 0 for an invalid id); emit(k, i, nb,
 // pos) for every sampled slot i < c (draw order, A5).  chain: this warp's 32 words of shared memory.
 // All 32 lanes must call it (warp-collective); warps past nT return at once.
-template <int UNR, typename EmitCnt, typename Emit>
+template <int UNR, bool COL32, typename EmitCnt, typename Emit>
 __device__ __forceinline__ void sample_warp(const ShardView& s, const int64_t* targets, int64_t nT, int M, int hop,
                                             uint2 key, int64_t warp_base, unsigned* chain, unsigned* ctrl_err,
                                             EmitCnt emit_cnt, Emit emit) {
@@ -61,7 +61,8 @@ __device__ __forceinline__ void sample_warp(const ShardView& s, const int64_t* t
     }
   }
 
-  const int64_t* src[UNR];
+  int64_t src[UNR];  // col_idx entry of the draw
+  int osrc[UNR];     // its owner rank
   int64_t kk[UNR];
   unsigned pos[UNR];
   bool ok[UNR];
@@ -104,13 +105,14 @@ __device__ __forceinline__ void sample_warp(const ShardView& s, const int64_t* t
     int o = 0;
     int64_t l;
     if (ok[u]) csr_owner_local(s, tv, o, l);
-    src[u] = s.col[o] + tstart + pos[u];
+    osrc[u] = o;
+    src[u] = tstart + pos[u];
     kk[u] = k;
     if (i == 0 && g < TPW && k < nT) emit_cnt(k, active ? (int)min(N, (unsigned)M) : 0);
   }
   int64_t nb[UNR];
 #pragma unroll
-  for (int u = 0; u < UNR; ++u) nb[u] = ok[u] ? *src[u] : -1;
+  for (int u = 0; u < UNR; ++u) nb[u] = ok[u] ? ld_col<COL32>(s, osrc[u], src[u]) : -1;
 #pragma unroll
   for (int u = 0; u < UNR; ++u)
     if (ok[u]) emit(kk[u], i, nb[u], pos[u]);

@@ -26,7 +26,7 @@ wg_status fail(wg_status s, const std::string& msg);
 // BY VALUE as a kernel parameter (constant bank; no global load per access).
 struct ShardView {
   const int64_t* row_ptr[WG_MAX_WORLD];
-  const int64_t* col[WG_MAX_WORLD];
+  const void* col[WG_MAX_WORLD];      // col_idx entries: int64, or uint32 with WG_DSM_COL32
   const uint8_t* feat[WG_MAX_WORLD];  // feature rows (their first body_bytes bytes), pitch feat_stride
   const uint8_t* tail[WG_MAX_WORLD];  // split layout: bytes [body_bytes, row_bytes) of every row, pitch tail_pitch
   int64_t n;            // num_nodes
@@ -36,7 +36,15 @@ struct ShardView {
   int32_t world;
   int32_t log2w;        // log2(world) if world is a power of two, else -1
   int32_t csr_rank;     // WG_DSM_CSR_REPLICATED: this rank, whose slab holds the whole CSR; -1: CSR row-sharded
+  int32_t col32;        // WG_DSM_COL32: col_idx entries are uint32
 };
+
+// Neighbour id at entry e of rank o's col_idx shard (8 B, or 4 B with WG_DSM_COL32).
+template <bool COL32>
+__device__ __forceinline__ int64_t ld_col(const ShardView& s, int o, int64_t e) {
+  if (COL32) return (int64_t)static_cast<const uint32_t*>(s.col[o])[e];
+  return static_cast<const int64_t*>(s.col[o])[e];
+}
 
 // Owner rank and local row of node v in the feature table (hash partition o(v) = v mod W,
 // l(v) = v div W; A11).

@@ -141,7 +141,8 @@ class DSM:
         _, e_local = self.shard_info(self.rank)
         csr_rows = self.num_nodes if self.csr_replicated else n_local
         row_ptr = device_view(rp.value, (csr_rows + 1,), torch.int64, self.device)
-        colv = device_view(col.value, (e_local,), torch.int64, self.device)
+        col_dtype = torch.int32 if self.flags & _lib.WG_DSM_COL32 else torch.int64  # uint32 entries (< 2^31 here)
+        colv = device_view(col.value, (e_local,), col_dtype, self.device)
         featv = device_view(feat.value, (n_local, stride.value), torch.uint8, self.device) if self.row_bytes else None
         return row_ptr, colv, featv
 

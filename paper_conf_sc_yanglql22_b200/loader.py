@@ -19,10 +19,15 @@ from .pipeline import required_keys
 
 
 def build_dsm(preset, rank=0, world=1, device=None, allgather=None, max_seeds=None, on_device=None,
-              feat_dim=None, feat_dtype=None, extra_keys=0, flags=0):
+              feat_dim=None, feat_dtype=None, extra_keys=0, flags=0, col32=None):
     """Create and fill a DSM for ``preset`` (a synth.presets.Preset).  Returns (dsm, info).
-    ``flags``: wg_dsm_desc.flags (e.g. WG_DSM_CSR_REPLICATED: every rank holds the whole CSR)."""
-    from ._lib import WG_DSM_CSR_REPLICATED
+    ``flags``: wg_dsm_desc.flags (e.g. WG_DSM_CSR_REPLICATED: every rank holds the whole CSR).
+    ``col32``: store col_idx as uint32 (WG_DSM_COL32); default: whenever the node ids fit (n < 2^31)."""
+    from ._lib import WG_DSM_COL32, WG_DSM_CSR_REPLICATED
+    if col32 is None:
+        col32 = preset.n < (1 << 31)
+    if col32:
+        flags |= WG_DSM_COL32
     csr_rep = bool(flags & WG_DSM_CSR_REPLICATED)
     c_rank, c_world = (0, 1) if csr_rep else (rank, world)   # which CSR rows this rank's slab holds
     device = torch.device("cuda", torch.cuda.current_device() if device is None else device)

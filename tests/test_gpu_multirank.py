@@ -21,14 +21,15 @@ pytestmark = pytest.mark.gpu
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 
 
-def _create_all(p, W, flags=0):
+def _create_all(p, W, flags=0, col32=None):
     ag = pkg.ThreadAllgather(W)
     out = [None] * W
     errs = []
 
     def run(r):
         try:
-            out[r] = loader.build_dsm(p, rank=r, world=W, allgather=ag.for_rank(r), on_device=False, flags=flags)[0]
+            out[r] = loader.build_dsm(p, rank=r, world=W, allgather=ag.for_rank(r), on_device=False, flags=flags,
+                                      col32=col32)[0]
         except Exception as e:  # pragma: no cover
             errs.append(e)
     ths = [threading.Thread(target=run, args=(r,)) for r in range(W)]
@@ -45,19 +46,20 @@ def _destroy_all(dsms):
 
 
 @pytest.mark.parametrize("W,placement", [(2, "dsm"), (3, "dsm"), (4, "dsm"), (8, "dsm"), (2, "csr-replicated"),
-                                         (4, "csr-replicated"), (8, "csr-replicated")])
+                                         (4, "csr-replicated"), (8, "csr-replicated"), (4, "dsm-col64"),
+                                         (4, "csr-replicated-col64")])
 def test_virtual_ranks_w_invariance(W, placement):
     """Every rank's batches are byte-identical to the oracle for the paper's placement (CSR and features
     row-sharded) and for the hybrid one (whole CSR on every rank, features sharded)."""
     p = presets.get("tiny")
     rp, col = graph.csr(p.graph())
-    flags = pkg.WG_DSM_CSR_REPLICATED if placement == "csr-replicated" else 0
-    dsms = _create_all(p, W, flags)
+    flags = pkg.WG_DSM_CSR_REPLICATED if placement.startswith("csr-replicated") else 0
+    dsms = _create_all(p, W, flags, col32=not placement.endswith("col64"))
     rows = providers.host_row_provider(p.graph(), rp, col)
     feats = providers.host_feat_provider(p)
     for r, dsm in enumerate(dsms):
         assert dsm.shard_info(r)[0] == len(graph.shard_rows(p.n, r, W))
-        if flags:
+        if flags & pkg.WG_DSM_CSR_REPLICATED:
             lrp, lcol, _ = dsm.local_view()
             assert lrp.numel() == p.n + 1 and lcol.numel() == len(col)   # the whole CSR on every rank
         pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)

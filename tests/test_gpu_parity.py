@@ -330,9 +330,11 @@ def test_pipeline_five_hops_fused(tiny):
     dsm.destroy()
 
 
-def test_pipeline_large_fanout(tiny):
+@pytest.mark.parametrize("col32", [False, True])
+def test_pipeline_large_fanout(tiny, col32):
+    """Fan-outs above 32 (the block sampler), int64 and uint32 (WG_DSM_COL32) col_idx."""
     p, rp, col = tiny
-    dsm, _ = loader.build_dsm(p, on_device=False, max_seeds=64, extra_keys=64 * 60 * 41 + 64 * 60)
+    dsm, _ = loader.build_dsm(p, on_device=False, max_seeds=64, extra_keys=64 * 60 * 41 + 64 * 60, col32=col32)
     fan = [60, 40]
     pipe = pkg.MiniBatchPipeline(dsm, fan, 64, with_pos=True, with_dup=True)
     S = seeds.seed_nodes(p.n, 64, presets.SEED_BASE, 3)
@@ -525,18 +527,19 @@ def test_gather_occupancy_setting(tiny):
     dsm.destroy()
 
 
-@pytest.mark.parametrize("flags", ["WG_DSM_WIDE_HASH", "WG_DSM_PAD64", "WG_DSM_WIDE_HASH|WG_DSM_PAD64"])
+@pytest.mark.parametrize("flags", ["WG_DSM_WIDE_HASH", "WG_DSM_PAD64", "WG_DSM_WIDE_HASH|WG_DSM_PAD64", "COL64",
+                                   "COL64|WG_DSM_PAD64"])
 def test_table_and_slot_formats(tiny, flags):
-    """The non-default hash-table / padded-slot formats (16 B wide slots claimed with one 128-bit CAS,
-    int64 padded sampler slots) stay bit-exact: 12 tiny batches through the fused pipeline and
-    hub-heavy standalone append-unique calls."""
+    """The non-default hash-table / padded-slot / column formats (16 B wide slots claimed with one 128-bit
+    CAS, int64 padded sampler slots, int64 col_idx instead of the loader's default uint32) stay bit-exact: 12 tiny batches through the fused
+    pipeline and hub-heavy standalone append-unique calls."""
     fl = 0
     for f in flags.split("|"):
-        fl |= getattr(pkg, f)
+        fl |= getattr(pkg, f) if f != "COL64" else 0
     p, rp, col = tiny
     rows = providers.host_row_provider(p.graph(), rp, col)
     feats = providers.host_feat_provider(p)
-    dsm, _ = loader.build_dsm(p, on_device=False, flags=fl)
+    dsm, _ = loader.build_dsm(p, on_device=False, flags=fl, col32="COL64" not in flags)
     pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
     for b in range(12):
         S = seeds.seed_nodes(p.n, p.seeds_per_batch - b * 7, presets.SEED_BASE, 300 + b)
