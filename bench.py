@@ -321,8 +321,9 @@ def measure_ceilings(dsm, reps=3):
         return n.value / best
 
     out = {}
-    for name, buf, span, width in (("random_8B_loads_per_s_col_shard", col, col.numel() * 8, 8),
-                                   ("random_32B_loads_per_s_col_shard", col, col.numel() * 8, 32),
+    col_bytes = col.numel() * col.element_size()   # 4 B entries with WG_DSM_COL32
+    for name, buf, span, width in (("random_8B_loads_per_s_col_shard", col, col_bytes, 8),
+                                   ("random_32B_loads_per_s_col_shard", col, col_bytes, 32),
                                    ("random_8B_loads_per_s_16MB", small, small.numel(), 8)):
         out[name] = timed(lambda: check(lib().wg_micro_random_read(ctypes.c_void_p(buf.data_ptr()), span, width, 16, 8,
                                                                     ctypes.c_void_p(sink.data_ptr()), ctypes.byref(n),
@@ -331,7 +332,7 @@ def measure_ceilings(dsm, reps=3):
         out[name] = timed(lambda: check(lib().wg_micro_atomics(ctypes.c_void_p(table.data_ptr()), table.numel(), op, 16, 8,
                                                                 ctypes.c_void_p(sink.data_ptr()), ctypes.byref(n),
                                                                 ctypes.c_void_p(st.cuda_stream))))
-    out["col_shard_bytes"] = col.numel() * 8
+    out["col_shard_bytes"] = col_bytes
     out["note"] = ("wg_micro_random_read / wg_micro_atomics: 148 SMs x 8 blocks x 256 threads, 8 independent "
                    "operations in flight per thread, best of 3")
     return out
@@ -343,15 +344,13 @@ def hop_kernels(m):
 
 
 def stage_breakdown(pipe, seeds_dev, rngs, flush, ceil=None, nb=20):
-    """SURVEY 8(d) per-kernel device times of one batch (outside every timed region): each hop's kernels
-    (wg_dsm_set_stage_events: an event after every kernel, eager launches, everything on one stream),
-    then the whole gather; L2 flushed before each batch; medians.  With the measured ceilings, every
-    prep kernel gets a fraction of its own bound.  Per hop with T targets and E sampled edges the
-    single-pass hop kernel must at least issue T + E random loads (row_ptr pairs, col entries), T + E
-    L2 probe/CAS operations (the keys) and E random L2 reads (first positions): its bound is the SLOWEST
-    of the three at the measured rates (random 8 B loads over the col shard, probe-CAS, random 8 B
-    loads over an L2-sized span), frac = that time / the kernel's time; the relabel's E random reads
-    against the L2-span load rate."""
+    """SURVEY 8(d) per-kernel device times of one batch (outside every timed region): each hop's sampler,
+    insert, flag scan and relabel (wg_dsm_set_stage_events: an event after every kernel, eager launches,
+    everything on one stream), then the whole gather; L2 flushed before each batch; medians.  With the
+    measured ceilings every prep kernel gets a fraction of its own bound: per hop with T targets and E
+    sampled edges, the sampler's T + E random loads (row_ptr pairs, col entries) against the random 8 B
+    load rate over the col shard, the insert's T + E keys against the L2 probe-CAS rate, the flag scan's
+    and the relabel's E random reads against the random 8 B load rate over an L2-sized span."""
     import torch
     st = torch.cuda.current_stream()
     H = len(pipe.fanouts)

@@ -91,3 +91,28 @@ def test_create_without_gpu_fails_cleanly():
     st = L.wg_dsm_create(ctypes.byref(d), ctypes.byref(h))
     assert st != 0 and not h.value
     assert L.wg_sample_neighbors(None, None, 0, None, 5, 0, None, 0, None, None, None, None, None) == 1
+
+
+def test_bench_reference_arm_cpu():
+    """bench.py --impl reference (the oracle arm; no GPU, no product library): one JSON line with the
+    contract's keys, a cpu_baseline describing the run, zero-copy e2e."""
+    import json
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--config", "tiny",
+                        "--steps", "2", "--warmup", "0"], cwd=ROOT, capture_output=True, text=True, timeout=300)
+    assert r.returncode == 0, r.stderr[-2000:]
+    lines = [ln for ln in r.stdout.splitlines() if ln.startswith("{")]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    assert d["impl"] == "reference" and d["value"] > 0 and d["unit"] == "seeds/s" and d["higher_is_better"] is True
+    cb = d["cpu_baseline"]
+    assert cb["kind"] == "oracle" and cb["cores"] == 1 and cb["value"] == d["value"] and cb["cores_available_before_pinning"] >= 1
+    assert d["e2e"] == {"value": d["value"], "unit": "seeds/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}
+    assert d["config"]["workload"] == "tiny"
+
+
+def test_bench_reference_arm_nonzero_rank_exits_quietly():
+    """Under torchrun the reference arm runs on rank 0 only; other ranks exit 0 without output."""
+    r = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--impl", "reference", "--config", "tiny",
+                        "--steps", "1", "--warmup", "0"], cwd=ROOT, capture_output=True, text=True, timeout=300,
+                       env=dict(os.environ, RANK="1", WORLD_SIZE="2"))
+    assert r.returncode == 0 and not r.stdout.strip()
