@@ -124,6 +124,9 @@ wg_status wg_dsm_create(const wg_dsm_desc* desc, wg_dsm_t* out);
 
 /* Device pointers of THIS rank's shard, for filling it (any stream; the caller
  * synchronises and barriers before other ranks read).  Any output may be NULL.
+ * d_row_ptr: int64[n_local_rows + 1] local offsets (int64[num_nodes + 1] with
+ * WG_DSM_CSR_REPLICATED); d_col_idx: the local CSR entries as int64, or as uint32 with
+ * WG_DSM_COL32 (reinterpret the pointer); n_local_rows = feature rows of this rank.
  * feat_row_stride_bytes is the row pitch of the feature shard, which holds the first
  * body_bytes bytes of every row (wg_dsm_feat_layout; the whole row unless the layout is split). */
 wg_status wg_dsm_local_view(wg_dsm_t h, int64_t** d_row_ptr, int64_t** d_col_idx, void** d_feat,
