@@ -42,7 +42,10 @@ constexpr int UQ_THREADS = WG_UQ_THREADS;
 // neighbour positions per thread of the flag scan: 1..8, chosen per launch so that small hops
 // spread over many SMs (latency-bound) and large hops keep several loads in flight per thread
 constexpr int CNT_BITS = 31;                    // packed scan value: (valid << 31) | first
-constexpr int PREP_BPS = 8;                     // insert / relabel blocks per SM (full occupancy)
+#ifndef WG_PREP_BPS
+#define WG_PREP_BPS 8
+#endif
+constexpr int PREP_BPS = WG_PREP_BPS;           // insert / relabel blocks per SM (full occupancy; A/B via WG_NVCC_DEFS)
 constexpr int FLAG_ITEMS_MAX = 8;               // most positions per thread of the flag scan
 constexpr int32_t SLOT_EMPTY = -1;              // slot_of: padded slot without a sample
 constexpr int32_t SLOT_BADID = -2;              // slot_of: sample whose id is out of range
