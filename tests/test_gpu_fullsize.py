@@ -186,3 +186,52 @@ def test_products_throughput_configuration_bit_exact(products):
         seen += 1
     assert seen == nb and ld.device_error() == 0
     ld.close()
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("placement", ["dsm", "csr-replicated"])
+def test_products_w4_virtual_ranks_bit_exact(placement):
+    """configs[1] at full size sharded over W=4 in-process virtual ranks on the one GPU, for the paper's
+    placement (CSR and 400 B split feature rows row-sharded: most row_ptr / col_idx / feature reads go to
+    other ranks' shards through the pointer table) and the CSR-replicated one (whole uint32 CSR per rank,
+    features sharded): one batch on ranks 0 and 3, every array compared with the oracle."""
+    import threading
+    p = presets.get("products")
+    W = 4
+    flags = pkg.WG_DSM_CSR_REPLICATED if placement == "csr-replicated" else 0
+    ag = pkg.ThreadAllgather(W)
+    dsms, errs = [None] * W, []
+
+    def create(r):
+        try:
+            dsms[r] = loader.build_dsm(p, rank=r, world=W, allgather=ag.for_rank(r), flags=flags)[0]
+        except Exception as e:  # pragma: no cover
+            errs.append(e)
+    ths = [threading.Thread(target=create, args=(r,)) for r in range(W)]
+    [t.start() for t in ths]
+    [t.join() for t in ths]
+    assert not errs, errs
+    try:
+        rows = providers.host_row_provider(p.graph())
+        feats = providers.host_feat_provider(p)
+        for r in (0, 3):
+            if flags:
+                assert dsms[r].local_view()[0].numel() == p.n + 1
+            pipe = pkg.MiniBatchPipeline(dsms[r], p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
+            b = next(iter(seeds.rank_batches(2 * W, r, W)))
+            S = seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, b)
+            rs = seeds.rng_seed(presets.RNG_BASE, b)
+            pipe.run(torch.from_numpy(S).cuda(), rs)
+            torch.cuda.synchronize()
+            ref = oracle.minibatch(rows, feats, S, p.fanouts, rs)
+            for h in range(len(p.fanouts)):
+                got, exp = pipe.result(h), ref["hops"][h]
+                for k in ("row_ptr", "nbrs", "pos", "unique", "sub_col", "dup"):
+                    assert np.array_equal(got[k], exp[k]), (placement, r, h, k)
+            assert np.array_equal(pipe.features(), ref["X"]), (placement, r)
+            assert dsms[r].device_error() == 0
+            del pipe
+    finally:
+        ths = [threading.Thread(target=d.destroy) for d in dsms if d is not None]
+        [t.start() for t in ths]
+        [t.join() for t in ths]
