@@ -80,9 +80,6 @@ typedef enum { WG_F32 = 0, WG_F16 = 1, WG_BF16 = 2 } wg_dtype;
 #define WG_DSM_COL32          0x10u /* col_idx entries stored as uint32 (needs num_nodes <= 2^32): half the
                                        bytes of every sampled line; wg_dsm_local_view's d_col_idx then points
                                        to uint32 entries (ids in every op stay int64) */
-#define WG_DSM_NO_CLUSTER_HOP 0x20u /* wg_sample_hop never uses the one-kernel cluster form for small hops
-                                       (n_targets * (1 + fanout) <= 32768, fanout <= 32, num_nodes < 2^32):
-                                       always the four-kernel general path (results are identical) */
 
 /* Allgather of host bytes across the W ranks of the DSM ("an
  * AllGather pattern communication is performed so that each process can get all

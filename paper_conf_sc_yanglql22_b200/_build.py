@@ -10,7 +10,7 @@ ROOT = os.path.dirname(PKG)
 CSRC = os.path.join(PKG, "csrc")
 INCLUDE = os.path.join(ROOT, "include")
 LIB = os.path.join(PKG, "libwg.so")
-SOURCES = ["dsm.cu", "sample.cu", "unique.cu", "gather.cu", "micro.cu", "spmm.cu", "exchange.cu", "hop_small.cu"]
+SOURCES = ["dsm.cu", "sample.cu", "unique.cu", "gather.cu", "micro.cu", "spmm.cu", "exchange.cu"]
 HEADERS = ["wg_internal.cuh", "device_util.cuh", "hash.cuh", "scan.cuh", "sample_warp.cuh"]
 
 NVCC = os.environ.get("NVCC", "/usr/local/cuda/bin/nvcc")

@@ -30,7 +30,6 @@ WG_DSM_WIDE_HASH = 0x2
 WG_DSM_PAD64 = 0x4
 WG_DSM_CSR_REPLICATED = 0x8
 WG_DSM_COL32 = 0x10
-WG_DSM_NO_CLUSTER_HOP = 0x20
 
 
 class WgError(RuntimeError):

@@ -180,8 +180,7 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
     return fail(WG_ERR_INVALID_ARG, "sizes out of range (num_nodes < 2^40, max_batch_keys < 2^31)");
   if (d->feat_dtype < WG_F32 || d->feat_dtype > WG_BF16) return fail(WG_ERR_INVALID_ARG, "feat_dtype");
   if (d->world_size > 1 && !d->allgather) return fail(WG_ERR_INVALID_ARG, "allgather callback required for W > 1");
-  if ((d->flags & ~(WG_DSM_WHOLE_ROWS | WG_DSM_WIDE_HASH | WG_DSM_PAD64 | WG_DSM_CSR_REPLICATED | WG_DSM_COL32 |
-                     WG_DSM_NO_CLUSTER_HOP)) ||
+  if ((d->flags & ~(WG_DSM_WHOLE_ROWS | WG_DSM_WIDE_HASH | WG_DSM_PAD64 | WG_DSM_CSR_REPLICATED | WG_DSM_COL32)) ||
       d->reserved)
     return fail(WG_ERR_INVALID_ARG, "unknown flags");
   if ((d->flags & WG_DSM_COL32) && d->num_nodes > (int64_t(1) << 32))

@@ -101,8 +101,6 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueA
   load_counts<PADDED>(a, nT, nE);
   const unsigned epoch = a.ctrl[CTRL_EPOCH];
   const int64_t total = nT + nE;
-  HashTable ht = a.ht;
-  if (WG_HASH_ACTUAL) ht.size = live_table_size(a.ht.size, total);
   const int lane = threadIdx.x & 31;
   const int64_t warps = (int64_t)gridDim.x * (UQ_THREADS / 32);
   for (int64_t base = ((int64_t)blockIdx.x * (UQ_THREADS / 32) + (threadIdx.x >> 5)) * 32; base < total;
@@ -144,16 +142,16 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueA
     if (valid && leader == lane) {
       if (COMPACT) {
         unsigned long long old;
-        slot = chash_insert(ht, key, q, compact_epoch(epoch), is_target, &old);
+        slot = chash_insert(a.ht, key, q, compact_epoch(epoch), is_target, &old);
         // a target meeting an earlier TARGET record of its key: duplicate target (A8)
         if (is_target && slot >= 0 && old != 0 && (int64_t)(old & CPOS_MASK) < nT)
           latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DUP_TARGET);
       } else if (is_target) {
         bool dup = false;
-        slot = hash_insert_target(ht, key, q, nT, epoch, &dup);
+        slot = hash_insert_target(a.ht, key, q, nT, epoch, &dup);
         if (dup) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DUP_TARGET);
       } else {
-        slot = hash_insert_min(ht, key, q, epoch);
+        slot = hash_insert_min(a.ht, key, q, epoch);
       }
       if (slot < 0) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_CAPACITY);
     }
@@ -416,16 +414,6 @@ cudaError_t launch_hop(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t*
                        int64_t* d_num_edges, int64_t* U, int64_t* d_nU, int32_t* sub_col, int32_t* dup,
                        cudaStream_t st, cudaStream_t side) {
   h->stage_i = 0;
-  if (small_hop_eligible(h, capT, fanout)) {  // one cluster kernel (hop_small.cu)
-    bool launched = false;
-    cudaError_t e = launch_small_hop(h, T, capT, d_nT, fanout, seed, d_seed, hop, out_row_ptr, out_nbrs, out_pos,
-                                     d_num_edges, U, d_nU, sub_col, dup, st, &launched);
-    if (e != cudaSuccess) return e;
-    if (launched) {
-      for (int i = 0; i < 4; ++i) stage_mark(h, st);  // sample | insert | flag | relabel: all in the one kernel
-      return cudaSuccess;
-    }
-  }
   cudaError_t e = launch_sample_padded(h, T, capT, d_nT, fanout, seed, d_seed, hop, out_pos != nullptr, st);
   if (e != cudaSuccess) return e;
   stage_mark(h, st);

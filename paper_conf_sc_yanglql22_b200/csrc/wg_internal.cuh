@@ -109,9 +109,6 @@ constexpr int EXCL_RING = 4;
 #ifndef WG_HASH_MIN_LOG2
 #define WG_HASH_MIN_LOG2 20
 #endif
-#ifndef WG_HASH_ACTUAL
-#define WG_HASH_ACTUAL 0
-#endif
 constexpr double HASH_FACTOR = WG_HASH_FACTOR_PCT / 100.0;
 constexpr int64_t HASH_MIN_SLOTS = int64_t(1) << WG_HASH_MIN_LOG2;
 constexpr int64_t HASH_MAX_SLOTS = (int64_t(1) << 31) - 8;  // slot indices are stored as int32 (slot_of)
@@ -175,15 +172,6 @@ inline int64_t table_prefix(const wg_dsm* h, int64_t key_bound) {
   return hc < h->ws.hcap ? hc : h->ws.hcap;
 }
 
-// The prefix a call really uses, from its DEVICE key count (WG_HASH_ACTUAL): HASH_FACTOR x keys slots
-// (a multiple of 16 = one 128 B line), at least HASH_MIN_SLOTS, at most the host bound `bound`.
-__device__ __forceinline__ unsigned long long live_table_size(unsigned long long bound, int64_t keys) {
-  long long hc = (long long)(HASH_FACTOR * (double)keys) + 16;
-  hc = hc < HASH_MIN_SLOTS ? HASH_MIN_SLOTS : hc;
-  hc = (hc + 15) / 16 * 16;
-  return (unsigned long long)hc < bound ? (unsigned long long)hc : bound;
-}
-
 // Record the next stage event (if any are set) on st, after the kernel just enqueued there.
 inline void stage_mark(wg_dsm* h, cudaStream_t st) {
   if (h->stage_i < h->stage_n) cudaEventRecord(h->stage_ev[h->stage_i++], st);
@@ -211,11 +199,6 @@ cudaError_t launch_hop(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t*
                        const uint64_t* d_seed, int hop, int64_t* out_row_ptr, int64_t* out_nbrs, int32_t* out_pos,
                        int64_t* d_num_edges, int64_t* U, int64_t* d_nU, int32_t* sub_col, int32_t* dup,
                        cudaStream_t st, cudaStream_t side);
-bool small_hop_eligible(const wg_dsm* h, int64_t capT, int fanout);
-cudaError_t launch_small_hop(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t* d_nT, int fanout, uint64_t seed,
-                             const uint64_t* d_seed, int hop, int64_t* out_row_ptr, int64_t* out_nbrs,
-                             int32_t* out_pos, int64_t* d_num_edges, int64_t* U, int64_t* d_nU, int32_t* sub_col,
-                             int32_t* dup, cudaStream_t st, bool* launched);
 cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int64_t* d_n, const int64_t* d_begin,
                           void* out, int64_t out_pitch, cudaStream_t st);
 }  // namespace wg

@@ -1,7 +1,6 @@
 """Seeded randomized parity campaign (tolerance 0 against the oracle): random graphs (power-law degrees with
 planted hubs, empty rows, self-loop-free sorted rows), random fan-out lists (1-4 hops, 1..40 per hop: both
-samplers), random seed counts (0, 1, ragged), every layout / placement flag (small hops take the one-kernel cluster
-form unless WG_DSM_NO_CLUSTER_HOP), W in {1, 2, 3} virtual ranks,
+samplers), random seed counts (0, 1, ragged), every layout / placement flag, W in {1, 2, 3} virtual ranks,
 eager runs and CUDA-graph replays, with and without positions / duplicate counts."""
 
 import threading
@@ -20,8 +19,7 @@ from gpu_helpers import csr_from_rows
 pytestmark = pytest.mark.gpu
 
 FLAG_SETS = [0, pkg.WG_DSM_COL32, pkg.WG_DSM_WIDE_HASH, pkg.WG_DSM_PAD64 | pkg.WG_DSM_COL32,
-             pkg.WG_DSM_WHOLE_ROWS, pkg.WG_DSM_CSR_REPLICATED | pkg.WG_DSM_COL32, pkg.WG_DSM_CSR_REPLICATED,
-             pkg.WG_DSM_NO_CLUSTER_HOP | pkg.WG_DSM_COL32, pkg.WG_DSM_NO_CLUSTER_HOP]
+             pkg.WG_DSM_WHOLE_ROWS, pkg.WG_DSM_CSR_REPLICATED | pkg.WG_DSM_COL32, pkg.WG_DSM_CSR_REPLICATED]
 
 
 def _random_graph(rng, n):
@@ -126,7 +124,7 @@ def test_random_standalone_ops_bit_exact(case):
     M = int(rng.choice([1, 4, 5, 10, 16, 31, 32, 33, 64, 129]))
     nT = int(rng.integers(0, min(n, 300) + 1))
     T = rng.choice(n, nT, replace=False).astype(np.int64)
-    flags = [0, pkg.WG_DSM_COL32, pkg.WG_DSM_WIDE_HASH, pkg.WG_DSM_PAD64, pkg.WG_DSM_NO_CLUSTER_HOP][case % 5]
+    flags = [0, pkg.WG_DSM_COL32, pkg.WG_DSM_WIDE_HASH, pkg.WG_DSM_PAD64][case % 4]
     dsms, feat = _make(rp, col, n, 12, "fp32", flags, 1, max(nT * (M + 1), 1))
     dsm = dsms[0]
     try:
