@@ -508,6 +508,8 @@ class Workload:
         self.seeds_dev = [torch.from_numpy(seeds.seed_nodes(p.n, S, presets.SEED_BASE, b)).to(d.dev)
                           for b in self.batches]
         self.rngs = [seeds.rng_seed(presets.RNG_BASE, b) for b in self.batches]
+        # each batch's inputs resident in HBM as the pipeline's packed input layout: one D2D copy per batch
+        self.packed_dev = [pipemod.pack_inputs(s_, r_, d.dev) for s_, r_ in zip(self.seeds_dev, self.rngs)]
         self.flush = None if args.no_flush else torch.empty(512 << 20, dtype=torch.uint8, device=d.dev)
         occ_b = args.gather_occupancy
         if occ_b is None:
@@ -551,7 +553,7 @@ class Workload:
         pl, g = self.pipes[j], self.graphs[j]
         with torch.cuda.stream(st):
             if k is not None:
-                pl.set_inputs(self.seeds_dev[k], self.rngs[k])
+                pl.set_inputs_packed(self.packed_dev[k])
             if g is not None:
                 g[kind].replay()
             elif kind == "prep":

@@ -57,13 +57,15 @@ class MiniBatchPipeline:
             raise ValueError("DSM workspace too small for this pipeline (max_batch_keys)")
         i64 = dict(dtype=torch.int64, device=dev)
         i32 = dict(dtype=torch.int32, device=dev)
-        self.seeds = torch.zeros(max(self.max_seeds, 1), **i64)
-        # per-batch scalars in one device buffer [n_seeds, rng_seed (uint64 bit pattern)], written by ONE
-        # H2D copy from a pinned staging buffer; per-hop counts in one [H, 2] buffer (one D2H copy)
-        self.params = torch.zeros(2, **i64)
-        self.n_seeds, self.rng_seed = self.params[0:1], self.params[1:2]
+        # the batch's inputs in ONE device buffer [n_seeds, rng_seed (uint64 bit pattern), seed ids...], so a
+        # batch is written by one copy (set_inputs from host ids / set_inputs_packed); per-hop counts in one
+        # [H, 2] buffer (one D2H copy)
+        self.inbuf = torch.zeros(2 + max(self.max_seeds, 1), **i64)
+        self.params = self.inbuf[0:2]
+        self.n_seeds, self.rng_seed = self.inbuf[0:1], self.inbuf[1:2]
+        self.seeds = self.inbuf[2:]
         # a ring of pinned staging buffers, so the host can enqueue many batches ahead without waiting
-        self._params_host = torch.zeros((PARAMS_RING, 2), dtype=torch.int64, pin_memory=True)
+        self._params_host = torch.zeros((PARAMS_RING, self.inbuf.numel()), dtype=torch.int64, pin_memory=True)
         self._params_ev = [None] * PARAMS_RING
         self._params_next = 0
         self.counts_dev = torch.zeros((len(self.fanouts), 2), **i64)
@@ -142,8 +144,9 @@ class MiniBatchPipeline:
         self.dsm.gather_rows(last["unique"], self.U_cap[-1], None, last["num_unique"], self.X, stream=stream)
 
     def set_inputs(self, seeds: torch.Tensor, rng_seed: int, stream=None):
-        """Copy this batch's seed nodes (device or pinned host int64) and (n_seeds, rng_seed) into the
-        pipeline's device buffers: two stream-ordered copies, no kernel."""
+        """Write this batch's seed nodes (host or device int64) and (n_seeds, rng_seed) into the pipeline's
+        input buffer, stream-ordered, no kernel: host ids are packed with the scalars into a pinned staging
+        slot and moved by ONE H2D copy; device ids take a D2D copy plus a 16 B H2D of the scalars."""
         n = seeds.numel()
         if n > self.max_seeds:
             raise ValueError("too many seeds")
@@ -158,9 +161,21 @@ class MiniBatchPipeline:
         stage[0] = n
         stage[1] = to_i64(rng_seed)
         with torch.cuda.stream(s):
-            self.seeds[:n].copy_(seeds, non_blocking=True)
-            self.params.copy_(stage, non_blocking=True)
+            if seeds.is_cuda:
+                self.seeds[:n].copy_(seeds, non_blocking=True)
+                self.params.copy_(stage[:2], non_blocking=True)
+            else:
+                stage[2:2 + n].copy_(seeds)
+                self.inbuf[:2 + n].copy_(stage[:2 + n], non_blocking=True)
             self._params_ev[k].record(s)
+
+    def set_inputs_packed(self, packed: torch.Tensor, stream=None):
+        """One D2D copy of a device int64 buffer already laid out as the input buffer: [n_seeds, rng_seed,
+        seed ids...] (pack_inputs); n_seeds must equal packed.numel() - 2."""
+        if packed.numel() - 2 > self.max_seeds or packed.numel() < 2:
+            raise ValueError("packed inputs do not fit this pipeline")
+        with torch.cuda.stream(stream or torch.cuda.current_stream()):
+            self.inbuf[:packed.numel()].copy_(packed, non_blocking=True)
 
     def run(self, seeds, rng_seed, stream=None):
         self.set_inputs(seeds, rng_seed, stream)
@@ -203,6 +218,14 @@ class MiniBatchPipeline:
     def features(self):
         u = int(self.hops[-1]["num_unique"].item())
         return self.X_rows[:u].contiguous().cpu().numpy()
+
+
+def pack_inputs(seeds, rng_seed: int, device=None) -> torch.Tensor:
+    """[n_seeds, rng_seed, seed ids...] as one int64 tensor (for MiniBatchPipeline.set_inputs_packed)."""
+    s = torch.as_tensor(seeds, dtype=torch.int64).reshape(-1).cpu()
+    head = torch.tensor([s.numel(), to_i64(rng_seed)], dtype=torch.int64)
+    out = torch.cat([head, s])
+    return out.to(device) if device is not None else out
 
 
 def to_i64(x: int) -> int:

@@ -55,6 +55,40 @@ def test_tiny_pipeline_many_batches(tiny, fused, incr):
     dsm.destroy()
 
 
+@pytest.mark.parametrize("how", ["device", "host", "pinned", "packed"])
+def test_pipeline_input_paths(tiny, how):
+    """The batch inputs reach the captured graph through every set_inputs path -- device ids (D2D + 16 B
+    H2D), host / pinned ids (packed into the pinned staging ring, one H2D), a packed device buffer
+    (one D2D) -- with ragged seed counts, and every batch stays bit-exact."""
+    p, rp, col = tiny
+    dsm, _ = loader.build_dsm(p, on_device=False)
+    pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
+    rows = providers.host_row_provider(p.graph(), rp, col)
+    feats = providers.host_feat_provider(p)
+    for b, cnt in enumerate([p.seeds_per_batch, 7, p.seeds_per_batch - 3, 1]):
+        S = seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 40 + b)[:cnt]
+        rs = seeds.rng_seed(presets.RNG_BASE, 40 + b)
+        t = torch.from_numpy(S)
+        if how == "device":
+            pipe.set_inputs(t.cuda(), rs)
+        elif how == "host":
+            pipe.set_inputs(t, rs)
+        elif how == "pinned":
+            pipe.set_inputs(t.pin_memory(), rs)
+        else:
+            pipe.set_inputs_packed(pkg.pipeline.pack_inputs(S, rs, "cuda"))
+        if pipe.graph is not None:
+            pipe.graph.replay()
+        else:
+            pipe.enqueue()
+        torch.cuda.synchronize()
+        _check_batch(pipe, oracle.minibatch(rows, feats, S, p.fanouts, rs), p.fanouts)
+        if b == 0:
+            pipe.capture()
+    assert dsm.device_error() == 0
+    dsm.destroy()
+
+
 def test_tiny_cuda_graph_replay(tiny):
     """The captured batch graph replays with new seeds / rng_seed and stays bit-exact."""
     p, rp, col = tiny
