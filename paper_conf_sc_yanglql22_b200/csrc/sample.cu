@@ -261,8 +261,10 @@ __global__ void __launch_bounds__(COMPACT_THREADS) sample_compact_kernel(const C
     const int c = k < nT ? a.cnt[k] : 0;
     int agg;
     const int ex = block_exclusive_sum<COMPACT_THREADS>(c, sm_wtot, &agg);
-    const unsigned long long pre = block_lookback<COMPACT_THREADS>(a.status, (long)blockIdx.x,
-                                                                   (unsigned long long)agg, lb);
+    const unsigned long long pre =
+        gridDim.x <= WG_LB_DIRECT_MAX
+            ? block_prefix_direct<COMPACT_THREADS>(a.status, (long)blockIdx.x, (unsigned long long)agg, lb)
+            : block_lookback<COMPACT_THREADS>(a.status, (long)blockIdx.x, (unsigned long long)agg, lb);
     const int64_t off = (int64_t)pre + ex;
     if (k < nT) {
       a.out_row_ptr[k] = off;

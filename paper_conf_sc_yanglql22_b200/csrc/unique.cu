@@ -227,7 +227,9 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArg
     unsigned long long ex =
         block_exclusive_sum<UQ_THREADS>(lane == 0 ? ((wv << CNT_BITS) | wf) : 0ull, sm_wtot, &agg);
     ex = __shfl_sync(FULL_MASK, ex, 0);  // this warp's offset inside the tile
-    const unsigned long long pre = block_lookback<UQ_THREADS>(a.status, (long)blockIdx.x, agg, lb);
+    const unsigned long long pre = gridDim.x <= WG_LB_DIRECT_MAX
+                                       ? block_prefix_direct<UQ_THREADS>(a.status, (long)blockIdx.x, agg, lb)
+                                       : block_lookback<UQ_THREADS>(a.status, (long)blockIdx.x, agg, lb);
     const unsigned long long base = pre + ex;
     int64_t ev = (int64_t)(base >> CNT_BITS);                 // dense position of this warp's next valid slot
     int64_t ef = (int64_t)(base & ((1ull << CNT_BITS) - 1));  // next new-node index
