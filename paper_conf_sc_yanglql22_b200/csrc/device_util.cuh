@@ -5,6 +5,10 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#if defined(WG_KTIMING) && WG_KTIMING
+#include <cstdio>
+#endif
+
 namespace wg {
 
 constexpr unsigned FULL_MASK = 0xffffffffu;
@@ -145,5 +149,57 @@ struct FastDiv {
     return (unsigned)(((unsigned long long)t + n) >> shift);
   }
 };
+
+// ---------------------------------------------------------------- diagnostics (WG_KTIMING=1 builds only)
+// Per-block globaltimer marks of the hot kernels; the last block of a large launch prints when its blocks
+// started and ended (10-bin histograms over the launch's span).  profiles/probes/ktiming.py.
+#ifndef WG_KTIMING
+#define WG_KTIMING 0
+#endif
+#if WG_KTIMING
+static __device__ unsigned long long g_kt[4][16384][2];
+static __device__ unsigned g_kt_done[4];
+static __device__ __forceinline__ unsigned long long kt_now() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %globaltimer;" : "=l"(t));
+  return t;
+}
+static __device__ __forceinline__ void kt_begin(int k) {
+  if (threadIdx.x == 0 && blockIdx.x < 16384) g_kt[k][blockIdx.x][0] = kt_now();
+}
+static __device__ __noinline__ void kt_end(int k, const char* name, int64_t work) {
+  __syncthreads();
+  if (threadIdx.x != 0 || blockIdx.x >= 16384) return;
+  g_kt[k][blockIdx.x][1] = kt_now();
+  __threadfence();
+  if (atomicAdd(&g_kt_done[k], 1u) != gridDim.x - 1) return;
+  g_kt_done[k] = 0;
+  const unsigned nb = gridDim.x < 16384 ? gridDim.x : 16384;
+  if (nb < 256) return;
+  unsigned long long t0 = ~0ull, t1 = 0;
+  for (unsigned b = 0; b < nb; ++b) {
+    t0 = min(t0, g_kt[k][b][0]);
+    t1 = max(t1, g_kt[k][b][1]);
+  }
+  const unsigned long long span = t1 - t0 + 1;
+  unsigned hs[10] = {0}, he[10] = {0};
+  unsigned long long dsum = 0, dmax = 0;
+  for (unsigned b = 0; b < nb; ++b) {
+    hs[min(9ull, (g_kt[k][b][0] - t0) * 10 / span)]++;
+    he[min(9ull, (g_kt[k][b][1] - t0) * 10 / span)]++;
+    const unsigned long long d = g_kt[k][b][1] - g_kt[k][b][0];
+    dsum += d;
+    dmax = max(dmax, d);
+  }
+  printf("KT %s blocks %u work %lld span %llu ns | block mean %llu max %llu | start %u %u %u %u %u %u %u %u %u %u | end %u %u %u %u %u %u %u %u %u %u\n",
+         name, nb, (long long)work, span, dsum / nb, dmax, hs[0], hs[1], hs[2], hs[3], hs[4], hs[5], hs[6], hs[7], hs[8],
+         hs[9], he[0], he[1], he[2], he[3], he[4], he[5], he[6], he[7], he[8], he[9]);
+}
+#define KT_BEGIN(k) kt_begin(k)
+#define KT_END(k, name, work) kt_end(k, name, work)
+#else
+#define KT_BEGIN(k)
+#define KT_END(k, name, work)
+#endif
 
 }  // namespace wg

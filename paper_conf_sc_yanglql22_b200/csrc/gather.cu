@@ -139,6 +139,7 @@ __device__ __forceinline__ void st_out<u32x8>(u32x8* p, const u32x8& r) {
 template <typename V, int GATHER_UNROLL, int MINB = GATHER_MINB>
 __global__ void __launch_bounds__(GATHER_THREADS, MINB) gather_kernel(const GatherArgs a) {
   pdl_enter();
+  KT_BEGIN(3);
   int64_t n = a.cap;
   if (a.d_n) {
     n = *a.d_n;
@@ -182,6 +183,7 @@ __global__ void __launch_bounds__(GATHER_THREADS, MINB) gather_kernel(const Gath
     for (int j = 0; j < GATHER_UNROLL; ++j)
       if (dst[j] < total) st_out<V>(&out[dst[j]], val[j]);
   }
+  KT_END(3, "gather", n);
 }
 
 cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int64_t* d_n, const int64_t* d_begin,

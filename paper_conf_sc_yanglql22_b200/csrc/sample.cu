@@ -68,6 +68,7 @@ __device__ __noinline__ void clear_table_if_cycle_restarts(unsigned long long* w
 template <int SAMPLE_UNR, bool CLR, bool COL32>
 __global__ void __launch_bounds__(SAMPLE_THREADS, SAMPLE_MINB) sample_kernel(const SampleArgs a) {
   pdl_enter();
+  KT_BEGIN(0);
   if (CLR) clear_table_if_cycle_restarts(a.hclear, a.hwords, a.ctrl);
   __shared__ unsigned sm_chain[SAMPLE_THREADS / 32][32];
   const int tid = threadIdx.x, warp = tid >> 5;
@@ -92,6 +93,7 @@ __global__ void __launch_bounds__(SAMPLE_THREADS, SAMPLE_MINB) sample_kernel(con
         st_pad(a.nbrs_pad, a.pad32, k * M + i, nb);
         if (a.pos_pad) a.pos_pad[k * M + i] = (int32_t)pos;
       });
+  KT_END(0, "sample", nT);
 }
 
 // ---------------------------------------------------------------- fanout > 32

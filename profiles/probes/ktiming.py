@@ -1,6 +1,6 @@
 """Run a few products batches (one batch at a time, L2 flushed) through the shipped graph of a
-WG_FLAG_TIMING=1 build: the flag scan of hop 2 prints when its tiles started, published their aggregate
-and finished, as 8-bin histograms over the kernel's span."""
+WG_KTIMING=1 build (profiles/mk_ab.sh kt "-DWG_KTIMING=1"): every large launch of the sampler, insert,
+flag scan and gather prints when its blocks started and ended (10-bin histograms over its span)."""
 import os, sys
 sys.path.insert(0, os.getcwd())
 import torch
