@@ -181,6 +181,31 @@ def test_append_unique_random_vs_oracle():
     dsm.destroy()
 
 
+@pytest.mark.parametrize("n_nbrs", [2_000_000, 2_200_000, 3_500_000])
+def test_scan_prefix_forms_large(n_nbrs):
+    """The flag scan takes the direct tile-prefix sum for <= WG_LB_DIRECT_MAX (1024) tiles of 2048 positions
+    and the decoupled look-back above: append-unique calls on both sides of the boundary (977, 1075 and 1709
+    tiles), and the standalone sampler's compaction scan (256 targets per tile) with 200k and 400k targets,
+    all against the oracle."""
+    n, (rp, col) = _edge_graph()
+    dsm = make_dsm(rp, col, max_keys=4_000_000)
+    rng = np.random.default_rng(n_nbrs)
+    pool = n  # ids must be node ids; hub-heavy repeats (the scan sees every position)
+    T = rng.choice(pool, size=3000, replace=False).astype(np.int64)
+    nbrs = np.minimum((rng.random(n_nbrs) ** 2 * pool).astype(np.int64), pool - 1)
+    U, sc, dup = gpu_unique(dsm, T, nbrs)
+    Uo, sco, dupo = oracle.append_unique(T, nbrs)
+    assert np.array_equal(U, Uo) and np.array_equal(sc, sco) and np.array_equal(dup, dupo)
+    nT = 200_000 if n_nbrs < 3_000_000 else 400_000
+    Ts = rng.integers(0, n, nT).astype(np.int64)
+    got = gpu_hop(dsm, Ts, 3, 77, 1)
+    exp = oracle_hop(rp, col, Ts, 3, 77, 1)
+    for g, e in zip(got, exp):
+        assert np.array_equal(g, e)
+    assert dsm.device_error() == 0
+    dsm.destroy()
+
+
 @pytest.mark.parametrize("dim,dtype", [(4, "fp32"), (32, "fp32"), (100, "fp32"), (1024, "fp32"), (768, "fp16"),
                                        (3, "fp32"), (1, "fp16"), (7, "bf16"), (36, "fp32"), (56, "fp32"),
                                        (60, "fp32"), (200, "fp16"), (72, "bf16")])
