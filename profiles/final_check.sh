@@ -9,4 +9,5 @@ timeout 600 python bench.py --impl reference --steps 3 --warmup 1 > gpurun_out/b
 timeout 900 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29911 \
     bench.py --gpus 2 --steps 5 --warmup 3 --cpu-sample-s 0 --north-star "" > gpurun_out/bench_w2.log 2>&1; echo w2=$?
 python profiles/bench_summary.py gpurun_out/bench_w2.log
-bash profiles/sanitize.sh
+# compute-sanitizer is closed on the GPU pool now (runs left GPUs needing a reset); logs from round 2 in profiles/r02/
+[ "${WG_RUN_SANITIZER:-0}" = 1 ] && bash profiles/sanitize.sh

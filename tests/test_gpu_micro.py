@@ -119,8 +119,14 @@ print("BATCH OK")
     cs = "/usr/local/cuda/bin/compute-sanitizer"
     if not os.path.exists(cs):
         pytest.skip("compute-sanitizer not installed")
+    # the GPU pool closed compute-sanitizer (runs under it left GPUs needing a reset): opt-in only;
+    # the committed logs are profiles/r02/sanitize_*.log
+    if os.environ.get("WG_RUN_SANITIZER") != "1":
+        pytest.skip("compute-sanitizer runs are opt-in (WG_RUN_SANITIZER=1); logs in profiles/r02/sanitize_*.log")
     for tool, summary in (("racecheck", "RACECHECK SUMMARY: 0 hazards"), ("synccheck", "ERROR SUMMARY: 0 errors")):
         r = subprocess.run([cs, "--tool", tool, "--kernel-name", "kns=2wg", "--error-exitcode", "17", sys.executable,
                             "-c", code], cwd=ROOT, capture_output=True, text=True, timeout=900)
+        if "closed on this pool" in r.stderr:
+            pytest.skip("compute-sanitizer is closed on this GPU pool")
         assert r.returncode == 0 and "BATCH OK" in r.stdout and summary in r.stdout, (tool, r.stdout[-2000:],
                                                                                       r.stderr[-2000:])
