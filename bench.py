@@ -67,6 +67,8 @@ def parse():
     ap.add_argument("--latency-spans", default="1,8,16,32,64,128", help="--latency: spans in GiB (comma list)")
     ap.add_argument("--col64", action="store_true",
                     help="store col_idx as int64 (default: uint32, WG_DSM_COL32, whenever the node ids fit)")
+    ap.add_argument("--hashed", action="store_true",
+                    help="Append Unique in a hash table even when the direct table fits (WG_DSM_HASHED)")
     ap.add_argument("--x-pitch", type=int, default=None,
                     help="diagnostics: output row pitch of X (default: DSM.out_pitch(), the row rounded up to 32 B)")
     return ap.parse_args()
@@ -338,9 +340,10 @@ def measure_ceilings(dsm, reps=3):
     return out
 
 
-def hop_kernels(m):
-    """Kernel stages of one wg_sample_hop (the stage events the library records)."""
-    return ("sample", "insert", "flag", "relabel")
+def hop_kernels(m, direct=False):
+    """Kernel stages of one wg_sample_hop (the stage events the library records); with the direct key
+    table the sampler inserts every key and there is no insert pass."""
+    return ("sample", "flag", "relabel") if direct else ("sample", "insert", "flag", "relabel")
 
 
 def stage_breakdown(pipe, seeds_dev, rngs, flush, ceil=None, nb=20):
@@ -354,14 +357,19 @@ def stage_breakdown(pipe, seeds_dev, rngs, flush, ceil=None, nb=20):
     import torch
     st = torch.cuda.current_stream()
     H = len(pipe.fanouts)
-    acc = {f"hop{h}_{k}": [] for h in range(H) for k in hop_kernels(pipe.fanouts[h])}
+    from paper_conf_sc_yanglql22_b200 import WG_UNIQUE_DIRECT
+    direct = pipe.dsm.unique_format() == WG_UNIQUE_DIRECT
+
+    def hop_kernels_(m):
+        return hop_kernels(m, direct)
+    acc = {f"hop{h}_{k}": [] for h in range(H) for k in hop_kernels_(pipe.fanouts[h])}
     acc["gather"] = []
     cnt = []
     for b in range(nb + 2):
         pipe.set_inputs(seeds_dev[b % len(seeds_dev)], rngs[b % len(rngs)])
         if flush is not None:
             flush.fill_(b & 0xFF)
-        evs = [[torch.cuda.Event(enable_timing=True) for _ in range(len(hop_kernels(m)) + 1)] for m in pipe.fanouts]
+        evs = [[torch.cuda.Event(enable_timing=True) for _ in range(len(hop_kernels_(m)) + 1)] for m in pipe.fanouts]
         for row in evs:               # create the events (torch creates them lazily at the first record)
             for e in row:
                 e.record(st)
@@ -380,26 +388,27 @@ def stage_breakdown(pipe, seeds_dev, rngs, flush, ceil=None, nb=20):
         torch.cuda.synchronize()
         if b >= 2:
             for h, m in enumerate(pipe.fanouts):
-                for k, kind in enumerate(hop_kernels(m)):
+                for k, kind in enumerate(hop_kernels_(m)):
                     acc[f"hop{h}_{kind}"].append(evs[h][k].elapsed_time(evs[h][k + 1]))
             acc["gather"].append(g0.elapsed_time(g1))
             cnt.append(pipe.counts_dev.cpu().numpy().copy())
     out = {n: statistics.median(v) for n, v in acc.items()}
     for h, m in enumerate(pipe.fanouts):
-        out[f"hop{h}"] = sum(out[f"hop{h}_{k}"] for k in hop_kernels(m))
+        out[f"hop{h}"] = sum(out[f"hop{h}_{k}"] for k in hop_kernels_(m))
     c = np.mean(cnt, axis=0)
     fr = {}
     if ceil:
         T = float(pipe.max_seeds)
         for h, m in enumerate(pipe.fanouts):
             E, U = float(c[h, 0]), float(c[h, 1])
-            t = {k: out[f"hop{h}_{k}"] / 1e3 for k in hop_kernels(m)}
+            t = {k: out[f"hop{h}_{k}"] / 1e3 for k in hop_kernels_(m)}
             phases = {"random_loads": (T + E) / ceil["random_8B_loads_per_s_col_shard"],
                       "l2_probe_cas": (T + E) / ceil["l2_cas_probe_per_s_17MB"],
                       "l2_reads": E / ceil["random_8B_loads_per_s_16MB"]}
             d = {"targets": T, "edges": E, "unique": U}
             d["sample"] = phases["random_loads"] / t["sample"]
-            d["insert"] = phases["l2_probe_cas"] / t["insert"]
+            if "insert" in t:
+                d["insert"] = phases["l2_probe_cas"] / t["insert"]
             d["flag"] = phases["l2_reads"] / t["flag"]
             d["relabel"] = E / t["relabel"] / ceil["random_8B_loads_per_s_16MB"]
             fr[f"hop{h}"] = d
@@ -408,6 +417,7 @@ def stage_breakdown(pipe, seeds_dev, rngs, flush, ceil=None, nb=20):
         worst = min(((h, k, v) for h, d in fr.items() for k, v in d.items() if k in kinds), key=lambda x: x[2])
         fr["furthest_below"] = {"hop": worst[0], "kernel": worst[1], "frac": worst[2]}
     out["frac"] = fr
+    out["unique_format"] = "direct" if direct else "hashed"
     out["note"] = ("median ms per kernel of one batch (eager launches, an event after every kernel, L2 flushed per "
                    "batch; hop h = wg_sample_hop); frac = each kernel's operation rate over its measured ceiling "
                    "(ceilings)")
@@ -490,10 +500,12 @@ class Workload:
         S = p.seeds_per_batch
         t0 = time.perf_counter()
         col32 = False if args.col64 else None   # None: the loader's default (uint32 when the ids fit)
+        hashed = pkg.WG_DSM_HASHED if args.hashed else 0
         if placement == "replicas":   # every rank its own whole copy (a W=1 DSM); batches still b = r mod W
-            self.dsm, self.info = loader.build_dsm(p, rank=0, world=1, device=d.local, allgather=None, col32=col32)
+            self.dsm, self.info = loader.build_dsm(p, rank=0, world=1, device=d.local, allgather=None, col32=col32,
+                                                   flags=hashed)
         else:
-            flags = pkg.WG_DSM_CSR_REPLICATED if placement == "csr-replicated" else 0
+            flags = (pkg.WG_DSM_CSR_REPLICATED if placement == "csr-replicated" else 0) | hashed
             self.dsm, self.info = loader.build_dsm(p, rank=d.rank, world=d.world, device=d.local, allgather=d.ag,
                                                    flags=flags, col32=col32)
         self.info["col_idx_bytes"] = 4 if self.dsm.flags & pkg.WG_DSM_COL32 else 8

@@ -30,6 +30,10 @@ WG_DSM_WIDE_HASH = 0x2
 WG_DSM_PAD64 = 0x4
 WG_DSM_CSR_REPLICATED = 0x8
 WG_DSM_COL32 = 0x10
+WG_DSM_HASHED = 0x20
+
+# wg_dsm_unique_format (include/wg.h)
+WG_UNIQUE_WIDE, WG_UNIQUE_COMPACT, WG_UNIQUE_DIRECT = 0, 1, 2
 
 
 class WgError(RuntimeError):
@@ -71,13 +75,15 @@ def lib():
     L.wg_dsm_set_gather_occupancy.argtypes = [P, I32]
     L.wg_dsm_debug_set_epoch.argtypes = [P, ctypes.c_uint32]
     L.wg_dsm_set_stage_events.argtypes = [P, P, I32]
+    L.wg_dsm_unique_format.argtypes = [P, P]
     L.wg_micro_random_read.argtypes = [P, I64, I32, I32, I32, P, P, P]
     L.wg_micro_atomics.argtypes = [P, I64, I32, I32, I32, P, P, P]
     for f in ("wg_dsm_create", "wg_dsm_fork", "wg_dsm_local_view", "wg_dsm_shard_info", "wg_dsm_feat_layout",
               "wg_dsm_destroy", "wg_sample_neighbors", "wg_append_unique", "wg_sample_hop", "wg_gather", "wg_gather_rows",
               "wg_dsm_chase", "wg_spmm_mean_forward", "wg_spmm_mean_backward", "wg_bucket_by_owner", "wg_rows_permute",
               "wg_device_error", "wg_dsm_reset_workspace", "wg_dsm_set_gather_occupancy",
-              "wg_dsm_debug_set_epoch", "wg_micro_random_read", "wg_micro_atomics", "wg_dsm_set_stage_events"):
+              "wg_dsm_debug_set_epoch", "wg_micro_random_read", "wg_micro_atomics", "wg_dsm_set_stage_events",
+              "wg_dsm_unique_format"):
         getattr(L, f).restype = ctypes.c_int
     L.wg_last_error.restype = ctypes.c_char_p
     L.wg_last_error.argtypes = []
@@ -95,4 +101,4 @@ def check(status):
 EXPORTS = ["wg_dsm_create", "wg_dsm_fork", "wg_dsm_local_view", "wg_dsm_shard_info", "wg_dsm_feat_layout", "wg_dsm_destroy", "wg_sample_neighbors",
            "wg_append_unique", "wg_sample_hop", "wg_gather", "wg_gather_rows", "wg_dsm_chase", "wg_spmm_mean_forward",
            "wg_spmm_mean_backward", "wg_bucket_by_owner", "wg_rows_permute", "wg_device_error", "wg_dsm_reset_workspace", "wg_dsm_set_gather_occupancy",
-           "wg_dsm_debug_set_epoch", "wg_micro_random_read", "wg_micro_atomics", "wg_dsm_set_stage_events", "wg_last_error", "wg_version"]
+           "wg_dsm_debug_set_epoch", "wg_micro_random_read", "wg_micro_atomics", "wg_dsm_set_stage_events", "wg_dsm_unique_format", "wg_last_error", "wg_version"]

@@ -88,6 +88,8 @@ static wg_status barrier(wg_dsm* h) {
 static void free_workspace(wg_dsm* h) {
   Workspace& w = h->ws;
   cudaFree(w.hslots);
+  cudaFree(w.dtab[0]);
+  cudaFree(w.dtab[1]);
   cudaFree(w.status_sample);
   cudaFree(w.status_unique);
   for (int k = 0; k < EXCL_RING; ++k) cudaFree(w.excl[k]);
@@ -125,6 +127,22 @@ static wg_status alloc_workspace(wg_dsm* h, int64_t max_keys) {
   }
   // compact 8 B slots (hash.cuh) when node ids and positions fit 28 bits (WG_DSM_WIDE_HASH: 16 B slots)
   w.compact = !(h->flags & WG_DSM_WIDE_HASH) && h->n <= (int64_t(1) << 28) && max_keys < (int64_t(1) << 28) ? 1 : 0;
+  // direct table (a word per node, hash.cuh) for small graphs unless a hashed format is asked for
+  w.direct = !(h->flags & (WG_DSM_WIDE_HASH | WG_DSM_HASHED)) && h->n <= WG_DIRECT_MAX_NODES &&
+                     max_keys < (int64_t(1) << DPOS_BITS)
+                 ? 1
+                 : 0;
+  if (w.direct) {
+    const size_t db = (size_t)((h->n + 3) / 4) * 16;  // whole 16 B units (dtab_clear_ahead)
+    for (int t = 0; t < 2; ++t) {
+      if (cudaMalloc(&w.dtab[t], db) != cudaSuccess) {
+        cudaGetLastError();
+        free_workspace(h);
+        return fail(WG_ERR_OOM, "workspace allocation failed (direct table)");
+      }
+      WG_CUDA_TRY(cudaMemset(w.dtab[t], 0xff, db));  // every word empty
+    }
+  }
   w.pad32 = !(h->flags & WG_DSM_PAD64) && h->n < (int64_t(1) << 32) ? 1 : 0;
   if (w.compact) {
     WG_CUDA_TRY(cudaMemset(w.hslots, 0, cap * sizeof(HashSlot)));  // every word stale (epoch 0)
@@ -180,7 +198,8 @@ wg_status wg_dsm_create(const wg_dsm_desc* d, wg_dsm_t* out) {
     return fail(WG_ERR_INVALID_ARG, "sizes out of range (num_nodes < 2^40, max_batch_keys < 2^31)");
   if (d->feat_dtype < WG_F32 || d->feat_dtype > WG_BF16) return fail(WG_ERR_INVALID_ARG, "feat_dtype");
   if (d->world_size > 1 && !d->allgather) return fail(WG_ERR_INVALID_ARG, "allgather callback required for W > 1");
-  if ((d->flags & ~(WG_DSM_WHOLE_ROWS | WG_DSM_WIDE_HASH | WG_DSM_PAD64 | WG_DSM_CSR_REPLICATED | WG_DSM_COL32)) ||
+  if ((d->flags & ~(WG_DSM_WHOLE_ROWS | WG_DSM_WIDE_HASH | WG_DSM_PAD64 | WG_DSM_CSR_REPLICATED | WG_DSM_COL32 |
+                    WG_DSM_HASHED)) ||
       d->reserved)
     return fail(WG_ERR_INVALID_ARG, "unknown flags");
   if ((d->flags & WG_DSM_COL32) && d->num_nodes > (int64_t(1) << 32))
@@ -536,6 +555,9 @@ wg_status wg_dsm_reset_workspace(wg_dsm_t h, wg_stream_t stream) {
   if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
   cudaSetDevice(h->device);
   cudaStream_t st = (cudaStream_t)stream;
+  if (h->ws.direct) {
+    for (int t = 0; t < 2; ++t) WG_CUDA_TRY(cudaMemsetAsync(h->ws.dtab[t], 0xff, (size_t)((h->n + 3) / 4) * 16, st));
+  }
   if (h->ws.compact) {
     WG_CUDA_TRY(cudaMemsetAsync(h->ws.hslots, 0, h->ws.hcap * sizeof(HashSlot), st));
   } else {
@@ -560,6 +582,16 @@ wg_status wg_dsm_debug_set_epoch(wg_dsm_t h, uint32_t epoch) {
   cudaSetDevice(h->device);
   WG_CUDA_TRY(cudaDeviceSynchronize());
   WG_CUDA_TRY(cudaMemcpy(h->ws.ctrl + CTRL_EPOCH, &epoch, 4, cudaMemcpyHostToDevice));
+  // the direct tables hold words of the old epoch sequence: empty them (the next op's table must be
+  // clean, hash.cuh)
+  if (h->ws.direct)
+    for (int t = 0; t < 2; ++t) WG_CUDA_TRY(cudaMemset(h->ws.dtab[t], 0xff, (size_t)((h->n + 3) / 4) * 16));
+  return WG_OK;
+}
+
+wg_status wg_dsm_unique_format(wg_dsm_t h, int32_t* format) {
+  if (!h || !format) return fail(WG_ERR_INVALID_ARG, "null argument");
+  *format = h->ws.direct ? WG_UNIQUE_DIRECT : h->ws.compact ? WG_UNIQUE_COMPACT : WG_UNIQUE_WIDE;
   return WG_OK;
 }
 

@@ -68,6 +68,38 @@ __device__ __forceinline__ int64_t chash_min_pos(const HashTable& t, long long s
   return (int64_t)(reinterpret_cast<const unsigned long long*>(t.slots)[slot] & CPOS_MASK);
 }
 
+// ---- direct table: one 32-bit word per node v, [31:24] 255 - compact_epoch(e) (1..255), [23:0] the first
+// position of v in the current call.  A newer epoch has a SMALLER tag, so one atomicMin of the whole word
+// both overrides a stale word and keeps the minimum position; 0xFFFFFFFF is empty.  Epoch e uses table
+// e & 1; the op running at epoch e clears table (e+1) & 1 (idle: its last use was epoch e-1, finished)
+// when compact_epoch(e+1) <= 2, i.e. when a 255-epoch cycle restarts there -- the tables are never
+// cleared per call.  No slot, no probe, no claim: a neighbour insert is a fire-and-forget RED.MIN.
+struct DirectTable {
+  unsigned* t[2];
+  int64_t n;  // words per table (num_nodes)
+};
+constexpr unsigned DPOS_MASK = (1u << DPOS_BITS) - 1u;
+__device__ __forceinline__ unsigned dtag(unsigned epoch) { return 255u - compact_epoch(epoch); }
+__device__ __forceinline__ unsigned dword(unsigned tag, int64_t q) { return (tag << DPOS_BITS) | (unsigned)q; }
+__device__ __forceinline__ unsigned* dtab_cur(const DirectTable& d, unsigned epoch) { return d.t[epoch & 1u]; }
+// First position recorded for v in this epoch, or -1 (not inserted in this epoch).
+__device__ __forceinline__ int64_t dtab_min_pos(const unsigned* t, unsigned tag, int64_t v) {
+  const unsigned w = t[v];
+  return (w >> DPOS_BITS) == tag ? (int64_t)(w & DPOS_MASK) : -1;
+}
+// Called by every thread of the FIRST kernel of an append-unique (the fused hop's sampler, or the
+// standalone insert pass): clear the table of epoch e+1 if a cycle restarts there (grid-strided).
+static __device__ __noinline__ void dtab_clear_words(unsigned* t, int64_t n) {
+  uint4* w = reinterpret_cast<uint4*>(t);
+  const int64_t n4 = (n + 3) / 4;  // tables are allocated in whole 16 B units
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += stride)
+    w[i] = make_uint4(~0u, ~0u, ~0u, ~0u);
+}
+__device__ __forceinline__ void dtab_clear_ahead(const DirectTable& d, unsigned epoch) {
+  if (compact_epoch(epoch + 1u) <= 2u) dtab_clear_words(d.t[(epoch + 1u) & 1u], d.n);
+}
+
 __device__ __forceinline__ unsigned long long stored_key(unsigned epoch, int64_t key) {
   return ((unsigned long long)epoch << 40) | (unsigned long long)key;
 }

@@ -55,7 +55,58 @@ struct SampleArgs {
   unsigned long long* hclear;  // fused hop, compact hash table: zeroed here when its epoch cycle restarts
   int pad32;                   // padded neighbour slots hold uint32 ids (num_nodes < 2^32)
   int64_t hwords;
+  // MODE_DIRECT (fused hop with the direct table): the Append Unique insert happens here -- targets
+  // first (U[k] = T[k], their own position k, duplicate-target check), every sampled id a RED.MIN of
+  // its padded position nT + k*M + i (same order as the dense positions); padding slots get PAD_ID
+  DirectTable dt;
+  int64_t* U;
+  int32_t* dup;
 };
+// sampler modes: plain, plain + compact-table clear (fused hop, compact hash), fused hop with the
+// direct table (inserts here; the hop then has no insert pass)
+enum { MODE_PLAIN = 0, MODE_CLEAR = 1, MODE_DIRECT = 2 };
+
+// Padded slot without a sample (direct mode: the flag pass reads no per-target count)
+__device__ __forceinline__ int64_t pad_id(int pad32) { return pad32 ? (int64_t)0xFFFFFFFFu : (int64_t)-1; }
+
+// Target k of a fused direct hop: U[k] = v (targets first, in order, L160), its word takes position k.
+// Issued as soon as the target id is loaded, so that a hub that is also a target already holds a
+// position smaller than every neighbour's when the neighbours' filtered inserts read it; the returned
+// old word is checked at the end (direct_target_check): an earlier TARGET record of v (position < nT)
+// in this epoch is a duplicate target (A8) -- of two equal targets the later atomic sees the other.
+__device__ __forceinline__ unsigned direct_insert_target(const SampleArgs& a, unsigned* t, unsigned tag, int64_t k,
+                                                         int64_t v) {
+  a.U[k] = v;
+  if (a.dup) a.dup[k] = 0;
+  if (v < 0 || v >= a.s.n) return ~0u;  // the sampler latches WG_DEVERR_ID_RANGE
+  return atomicMin(&t[v], dword(tag, k));
+}
+__device__ __forceinline__ void direct_target_check(const SampleArgs& a, unsigned tag, int64_t nT, unsigned old) {
+  if ((old >> DPOS_BITS) == tag && (int64_t)(old & DPOS_MASK) < nT) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DUP_TARGET);
+}
+// Sampled id nb at padded position q: fire-and-forget atomicMin (compiles to RED.E.MIN).  lead = false:
+// a lower lane of the warp round holds the same id at a smaller position (no atomic needed).
+#ifndef WG_DIRECT_FILTER
+#define WG_DIRECT_FILTER 1  // read the word first and skip the RED when it already holds a smaller position
+#endif
+#ifndef WG_DIRECT_DEDUP
+#define WG_DIRECT_DEDUP 0  // warp-round __match_any_sync before the REDs (A/B: no gain)
+#endif
+__device__ __forceinline__ void direct_insert_nbr(const SampleArgs& a, unsigned* t, unsigned tag, int64_t q,
+                                                  int64_t nb, bool lead = true) {
+  if (nb < 0 || nb >= a.s.n) {
+    latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_ID_RANGE);
+    return;
+  }
+  if (!lead) return;
+  const unsigned mine = dword(tag, q);
+  if (WG_DIRECT_FILTER) {
+    unsigned cur;
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(cur) : "l"(&t[nb]));
+    if (cur <= mine) return;
+  }
+  atomicMin(&t[nb], mine);
+}
 
 // The insert pass that follows this sampler (same hop) needs a zeroed compact table when the epoch
 // cycle restarts (hash.cuh); every block clears a grid-strided share before sampling.
@@ -65,11 +116,16 @@ __device__ __noinline__ void clear_table_if_cycle_restarts(unsigned long long* w
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < words; i += stride) w[i] = 0ull;
 }
 
-template <int SAMPLE_UNR, bool CLR, bool COL32>
+template <int SAMPLE_UNR, int MODE, bool COL32>
 __global__ void __launch_bounds__(SAMPLE_THREADS, SAMPLE_MINB) sample_kernel(const SampleArgs a) {
   pdl_enter();
   KT_BEGIN(0);
-  if (CLR) clear_table_if_cycle_restarts(a.hclear, a.hwords, a.ctrl);
+  if (MODE == MODE_CLEAR) clear_table_if_cycle_restarts(a.hclear, a.hwords, a.ctrl);
+  unsigned epoch = 0;
+  if (MODE == MODE_DIRECT) {
+    epoch = a.ctrl[CTRL_EPOCH];
+    dtab_clear_ahead(a.dt, epoch);
+  }
   __shared__ unsigned sm_chain[SAMPLE_THREADS / 32][32];
   const int tid = threadIdx.x, warp = tid >> 5;
   int64_t nT = a.cap;
@@ -86,12 +142,26 @@ __global__ void __launch_bounds__(SAMPLE_THREADS, SAMPLE_MINB) sample_kernel(con
   const unsigned long long seed = a.d_seed ? *a.d_seed : a.seed;
   const uint2 key = make_uint2((unsigned)(seed & 0xffffffffu), (unsigned)(seed >> 32));
   // padded slots k*M + i of the workspace (the scan pass that follows compacts them)
-  sample_warp<SAMPLE_UNR, COL32>(
+  unsigned* const dt = MODE == MODE_DIRECT ? dtab_cur(a.dt, epoch) : nullptr;
+  const unsigned tag = MODE == MODE_DIRECT ? dtag(epoch) : 0u;
+  sample_warp<SAMPLE_UNR, COL32, MODE == MODE_DIRECT && WG_DIRECT_DEDUP>(
       a.s, a.targets, nT, M, a.hop, key, warp_base, sm_chain[warp], &a.ctrl[CTRL_ERR],
-      [&](int64_t k, int c) { a.cnt[k] = c; },
-      [&](int64_t k, int i, int64_t nb, unsigned pos) {
+      [&](int64_t k, int64_t v) -> unsigned {
+        return MODE == MODE_DIRECT ? direct_insert_target(a, dt, tag, k, v) : 0u;
+      },
+      [&](int64_t k, unsigned old) {
+        if (MODE == MODE_DIRECT) direct_target_check(a, tag, nT, old);
+      },
+      [&](int64_t k, int c) {
+        if (MODE != MODE_DIRECT) a.cnt[k] = c;
+      },
+      [&](int64_t k, int i, int64_t nb, unsigned pos, bool lead) {
         st_pad(a.nbrs_pad, a.pad32, k * M + i, nb);
         if (a.pos_pad) a.pos_pad[k * M + i] = (int32_t)pos;
+        if (MODE == MODE_DIRECT) direct_insert_nbr(a, dt, tag, nT + k * M + i, nb, lead);
+      },
+      [&](int64_t k, int i) {
+        if (MODE == MODE_DIRECT) st_pad(a.nbrs_pad, a.pad32, k * M + i, pad_id(a.pad32));
       });
   KT_END(0, "sample", nT);
 }
@@ -102,10 +172,17 @@ __global__ void __launch_bounds__(SAMPLE_THREADS, SAMPLE_MINB) sample_kernel(con
 // (L118): Algorithm 1 exactly as listed (L122-158), with parallel_sort = a block bitonic
 // sort of the packed 64-bit keys (r << 32 | i) (L118-120) in shared memory, chain / q /
 // last in shared memory and path doubling as ceil(log2 M) synchronous rounds.
-template <int BT, bool CLR, bool COL32>
+template <int BT, int MODE, bool COL32>
 __global__ void __launch_bounds__(BT) sample_block_kernel(const SampleArgs a) {
   pdl_enter();
-  if (CLR) clear_table_if_cycle_restarts(a.hclear, a.hwords, a.ctrl);
+  if (MODE == MODE_CLEAR) clear_table_if_cycle_restarts(a.hclear, a.hwords, a.ctrl);
+  unsigned epoch = 0;
+  if (MODE == MODE_DIRECT) {
+    epoch = a.ctrl[CTRL_EPOCH];
+    dtab_clear_ahead(a.dt, epoch);
+  }
+  unsigned* const dt = MODE == MODE_DIRECT ? dtab_cur(a.dt, epoch) : nullptr;
+  const unsigned tag = MODE == MODE_DIRECT ? dtag(epoch) : 0u;
   __shared__ unsigned long long s_key[BT];
   __shared__ unsigned s_r[BT], s_chain[BT], s_q[BT], s_last[BT];
   __shared__ int64_t s_v, s_start;
@@ -122,6 +199,7 @@ __global__ void __launch_bounds__(BT) sample_block_kernel(const SampleArgs a) {
   if (i == 0) {
     int64_t v = a.targets[k], start = 0;
     unsigned n = 0;
+    if (MODE == MODE_DIRECT) direct_target_check(a, tag, nT, direct_insert_target(a, dt, tag, k, v));
     if (v < 0 || v >= a.s.n) {
       latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_ID_RANGE);
       v = -1;
@@ -140,20 +218,25 @@ __global__ void __launch_bounds__(BT) sample_block_kernel(const SampleArgs a) {
     s_v = v;
     s_start = start;
     s_n = n;
-    a.cnt[k] = v >= 0 ? (int32_t)min(n, (unsigned)M) : 0;
+    if (MODE != MODE_DIRECT) a.cnt[k] = v >= 0 ? (int32_t)min(n, (unsigned)M) : 0;
   }
   __syncthreads();
   const int64_t v = s_v;
-  if (v < 0) return;
   const unsigned N = s_n;
+  // direct mode: slots past min(M, N) (all M for an invalid target) are padding
+  if (MODE == MODE_DIRECT && i < M && (v < 0 || (unsigned)i >= N))
+    st_pad(a.nbrs_pad, a.pad32, k * M + i, pad_id(a.pad32));
+  if (v < 0) return;
   int o;
   int64_t l;
   csr_owner_local(a.s, v, o, l);
   const int64_t cbase = s_start;
   if (N <= (unsigned)M) {  // L118: all of N neighbours, CSR order (A5)
     for (unsigned j = i; j < N; j += BT) {
-      st_pad(a.nbrs_pad, a.pad32, k * M + j, ld_col<COL32>(a.s, o, cbase + j));
+      const int64_t nb = ld_col<COL32>(a.s, o, cbase + j);
+      st_pad(a.nbrs_pad, a.pad32, k * M + j, nb);
       if (a.pos_pad) a.pos_pad[k * M + j] = (int32_t)j;
+      if (MODE == MODE_DIRECT) direct_insert_nbr(a, dt, tag, nT + k * M + j, nb);
     }
     return;
   }
@@ -214,8 +297,10 @@ __global__ void __launch_bounds__(BT) sample_block_kernel(const SampleArgs a) {
       res = s_r[i];
     else
       res = s_last[(unsigned)(s_key[qi - 1] & 0xffffffffu)];
-    st_pad(a.nbrs_pad, a.pad32, k * M + i, ld_col<COL32>(a.s, o, cbase + res));
+    const int64_t nb = ld_col<COL32>(a.s, o, cbase + res);
+    st_pad(a.nbrs_pad, a.pad32, k * M + i, nb);
     if (a.pos_pad) a.pos_pad[k * M + i] = (int32_t)res;
+    if (MODE == MODE_DIRECT) direct_insert_nbr(a, dt, tag, nT + k * M + i, nb);
   }
 }
 
@@ -286,24 +371,33 @@ __global__ void __launch_bounds__(COMPACT_THREADS) sample_compact_kernel(const C
   }
 }
 
-template <bool CLR, bool COL32>
+template <int MODE, bool COL32>
 static cudaError_t launch_block_sampler(int fanout, unsigned blocks, const SampleArgs& a, cudaStream_t st) {
-  if (fanout <= 64) return launch_pdl(sample_block_kernel<64, CLR, COL32>, blocks, 64, 0, st, a);
-  if (fanout <= 128) return launch_pdl(sample_block_kernel<128, CLR, COL32>, blocks, 128, 0, st, a);
-  if (fanout <= 256) return launch_pdl(sample_block_kernel<256, CLR, COL32>, blocks, 256, 0, st, a);
-  if (fanout <= 512) return launch_pdl(sample_block_kernel<512, CLR, COL32>, blocks, 512, 0, st, a);
-  return launch_pdl(sample_block_kernel<1024, CLR, COL32>, blocks, 1024, 0, st, a);
+  if (fanout <= 64) return launch_pdl(sample_block_kernel<64, MODE, COL32>, blocks, 64, 0, st, a);
+  if (fanout <= 128) return launch_pdl(sample_block_kernel<128, MODE, COL32>, blocks, 128, 0, st, a);
+  if (fanout <= 256) return launch_pdl(sample_block_kernel<256, MODE, COL32>, blocks, 256, 0, st, a);
+  if (fanout <= 512) return launch_pdl(sample_block_kernel<512, MODE, COL32>, blocks, 512, 0, st, a);
+  return launch_pdl(sample_block_kernel<1024, MODE, COL32>, blocks, 1024, 0, st, a);
 }
 
-template <bool CLR, bool COL32>
+template <int MODE, bool COL32>
 static cudaError_t launch_warp_sampler(int unr, unsigned blocks, const SampleArgs& a, cudaStream_t st) {
-  if (unr == 4) return launch_pdl(sample_kernel<4, CLR, COL32>, blocks, SAMPLE_THREADS, 0, st, a);
-  if (unr == 2) return launch_pdl(sample_kernel<2, CLR, COL32>, blocks, SAMPLE_THREADS, 0, st, a);
-  return launch_pdl(sample_kernel<1, CLR, COL32>, blocks, SAMPLE_THREADS, 0, st, a);
+  if (unr == 4) return launch_pdl(sample_kernel<4, MODE, COL32>, blocks, SAMPLE_THREADS, 0, st, a);
+  if (unr == 2) return launch_pdl(sample_kernel<2, MODE, COL32>, blocks, SAMPLE_THREADS, 0, st, a);
+  return launch_pdl(sample_kernel<1, MODE, COL32>, blocks, SAMPLE_THREADS, 0, st, a);
+}
+
+template <int MODE>
+static cudaError_t launch_sampler_mode(bool block, bool col32, int fanout, int unr, unsigned blocks,
+                                       const SampleArgs& a, cudaStream_t st) {
+  if (block) return col32 ? launch_block_sampler<MODE, true>(fanout, blocks, a, st)
+                          : launch_block_sampler<MODE, false>(fanout, blocks, a, st);
+  return col32 ? launch_warp_sampler<MODE, true>(unr, blocks, a, st) : launch_warp_sampler<MODE, false>(unr, blocks, a, st);
 }
 
 cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap, const int64_t* d_n, int fanout,
-                                 uint64_t seed, const uint64_t* d_seed, int hop, bool want_pos, cudaStream_t st) {
+                                 uint64_t seed, const uint64_t* d_seed, int hop, bool want_pos, cudaStream_t st,
+                                 int64_t* U, int32_t* dup) {
   SampleArgs a;
   a.s = h->view;
   a.targets = targets;
@@ -320,28 +414,33 @@ cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap,
   a.ctrl = h->ws.ctrl;
   a.hclear = h->ws.compact ? reinterpret_cast<unsigned long long*>(h->ws.hslots) : nullptr;
   a.hwords = h->ws.hcap;
-  if (fanout > 32) {  // block per target (Algorithm 1 with a block sort)
-    const unsigned blocks = (unsigned)(cap > 0 ? cap : 1);
-    if (a.s.col32) return a.hclear ? launch_block_sampler<true, true>(fanout, blocks, a, st)
-                                   : launch_block_sampler<false, true>(fanout, blocks, a, st);
-    return a.hclear ? launch_block_sampler<true, false>(fanout, blocks, a, st)
-                    : launch_block_sampler<false, false>(fanout, blocks, a, st);
+  a.dt = DirectTable{{h->ws.dtab[0], h->ws.dtab[1]}, h->n};
+  a.U = U;
+  a.dup = dup;
+  // U != NULL: the fused hop (wg_sample_hop); with the direct table its inserts happen here
+  const int mode = (U && h->ws.direct) ? MODE_DIRECT : (a.hclear ? MODE_CLEAR : MODE_PLAIN);
+  const bool block = fanout > 32;  // block per target (Algorithm 1 with a block sort)
+  int unr = 1;
+  unsigned blocks = (unsigned)(cap > 0 ? cap : 1);
+  if (!block) {
+    const int G = sample_group(fanout);
+    const int tpw = 32 / G;
+    unr = SAMPLE_UNR_MAX;  // largest of 4/2/1 that still gives >= 2 blocks per SM
+    while (unr > 1 && cap < (int64_t)(SAMPLE_THREADS / 32) * tpw * unr * 2 * h->sm_count) unr >>= 1;
+    const int64_t tile = (int64_t)(SAMPLE_THREADS / 32) * tpw * unr;
+    blocks = (unsigned)(cap > 0 ? (cap + tile - 1) / tile : 1);
   }
-  const int G = sample_group(fanout);
-  const int tpw = 32 / G;
-  int unr = SAMPLE_UNR_MAX;  // largest of 4/2/1 that still gives >= 2 blocks per SM
-  while (unr > 1 && cap < (int64_t)(SAMPLE_THREADS / 32) * tpw * unr * 2 * h->sm_count) unr >>= 1;
-  const int64_t tile = (int64_t)(SAMPLE_THREADS / 32) * tpw * unr;
-  const unsigned blocks = (unsigned)(cap > 0 ? (cap + tile - 1) / tile : 1);
-  if (a.s.col32) return a.hclear ? launch_warp_sampler<true, true>(unr, blocks, a, st)
-                                 : launch_warp_sampler<false, true>(unr, blocks, a, st);
-  return a.hclear ? launch_warp_sampler<true, false>(unr, blocks, a, st) : launch_warp_sampler<false, false>(unr, blocks, a, st);
+  const bool c32 = a.s.col32 != 0;
+  if (mode == MODE_DIRECT) return launch_sampler_mode<MODE_DIRECT>(block, c32, fanout, unr, blocks, a, st);
+  if (mode == MODE_CLEAR) return launch_sampler_mode<MODE_CLEAR>(block, c32, fanout, unr, blocks, a, st);
+  return launch_sampler_mode<MODE_PLAIN>(block, c32, fanout, unr, blocks, a, st);
 }
 
 cudaError_t launch_sample(wg_dsm* h, const int64_t* targets, int64_t cap, const int64_t* d_n, int fanout,
                           uint64_t seed, const uint64_t* d_seed, int hop, int64_t* out_row_ptr,
                           int64_t* out_nbrs, int32_t* out_pos, int64_t* d_num_edges, cudaStream_t st) {
-  cudaError_t e = launch_sample_padded(h, targets, cap, d_n, fanout, seed, d_seed, hop, out_pos != nullptr, st);
+  cudaError_t e =
+      launch_sample_padded(h, targets, cap, d_n, fanout, seed, d_seed, hop, out_pos != nullptr, st, nullptr, nullptr);
   if (e != cudaSuccess) return e;
   CompactArgs c{cap, d_n, fanout, h->ws.nbrs_pad, h->ws.pos_pad, h->ws.cnt, out_row_ptr, out_nbrs, out_pos,
                 d_num_edges, h->ws.status_sample, h->ws.ctrl, h->ws.pad32};

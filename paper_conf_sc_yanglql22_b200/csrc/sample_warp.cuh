@@ -22,13 +22,20 @@ constexpr int SAMPLE_UNR_MAX = 4;
 __host__ __device__ inline int sample_group(int M) { return M > SAMPLE_UNR_MAX ? M : SAMPLE_UNR_MAX; }
 
 // One warp samples the targets k = warp_base + u * TPW + g (u < UNR, g < TPW, k < nT) of targets[].
-// emit_cnt(k, c) is called once per target k < nT (c = min(M, deg), 0 for an invalid id); emit(k, i, nb,
-// pos) for every sampled slot i < c (draw order, A5).  chain: this warp's 32 words of shared memory.
+// on_target(k, v) is called once per target k < nT with its id as loaded (before the range check),
+// right after the load; it returns a token handed to on_target_end(k, token) after every other callback
+// of the warp (the direct table issues the target's atomic early and checks its result late); emit_cnt(k, c) once per target k < nT (c = min(M, deg), 0
+// for an invalid id); emit(k, i, nb, pos, lead) for every sampled slot i < c (draw order, A5), lead =
+// no lower lane of this warp round sampled the same id (DEDUP; always true without); emit_pad(k, i)
+// for the slots c <= i < M.
+// chain: this warp's 32 words of shared memory.
 // All 32 lanes must call it (warp-collective); warps past nT return at once.
-template <int UNR, bool COL32, typename EmitCnt, typename Emit>
+template <int UNR, bool COL32, bool DEDUP, typename OnTarget, typename OnTargetEnd, typename EmitCnt, typename Emit,
+          typename EmitPad>
 __device__ __forceinline__ void sample_warp(const ShardView& s, const int64_t* targets, int64_t nT, int M, int hop,
                                             uint2 key, int64_t warp_base, unsigned* chain, unsigned* ctrl_err,
-                                            EmitCnt emit_cnt, Emit emit) {
+                                            OnTarget on_target, OnTargetEnd on_target_end, EmitCnt emit_cnt, Emit emit,
+                                            EmitPad emit_pad) {
   if (warp_base >= nT) return;  // warp-uniform
   const int lane = threadIdx.x & 31;
   const int G = sample_group(M);
@@ -38,11 +45,12 @@ __device__ __forceinline__ void sample_warp(const ShardView& s, const int64_t* t
 
   // ---- row_ptr pairs: lane u of each group fetches round u's target (all in flight)
   int64_t my_v = -1, my_start = 0;
-  unsigned my_deg = 0;
+  unsigned my_deg = 0, my_tok = 0;
   if (i < UNR && g < TPW) {
     const int64_t k = warp_base + (int64_t)i * TPW + g;
     if (k < nT) {
       my_v = targets[k];
+      my_tok = on_target(k, my_v);
       if (my_v < 0 || my_v >= s.n) {
         latch_error(ctrl_err, WG_DEVERR_ID_RANGE);
         my_v = -1;
@@ -65,7 +73,7 @@ __device__ __forceinline__ void sample_warp(const ShardView& s, const int64_t* t
   int osrc[UNR];     // its owner rank
   int64_t kk[UNR];
   unsigned pos[UNR];
-  bool ok[UNR];
+  bool ok[UNR], pad[UNR];
 #pragma unroll
   for (int u = 0; u < UNR; ++u) {
     const int64_t k = warp_base + (int64_t)u * TPW + g;
@@ -102,6 +110,7 @@ __device__ __forceinline__ void sample_warp(const ShardView& s, const int64_t* t
     __syncwarp();
     pos[u] = full ? (unsigned)i : (prev < 0 ? r : lastp);  // lines 16-22
     ok[u] = active && (full ? (unsigned)i < N : i < M);
+    pad[u] = g < TPW && k < nT && i < M && !ok[u];
     int o = 0;
     int64_t l;
     if (ok[u]) csr_owner_local(s, tv, o, l);
@@ -114,8 +123,20 @@ __device__ __forceinline__ void sample_warp(const ShardView& s, const int64_t* t
 #pragma unroll
   for (int u = 0; u < UNR; ++u) nb[u] = ok[u] ? ld_col<COL32>(s, osrc[u], src[u]) : -1;
 #pragma unroll
-  for (int u = 0; u < UNR; ++u)
-    if (ok[u]) emit(kk[u], i, nb[u], pos[u]);
+  for (int u = 0; u < UNR; ++u) {
+    bool lead = true;
+    if (DEDUP) {  // lanes are in position order within a round: the lowest lane holds the first position
+      const unsigned same =
+          __match_any_sync(FULL_MASK, ok[u] ? (unsigned long long)nb[u] : (0x8000000000000000ull | (unsigned)lane));
+      lead = (same & ((1u << lane) - 1u)) == 0u;
+    }
+    if (ok[u]) emit(kk[u], i, nb[u], pos[u], lead);
+    else if (pad[u]) emit_pad(kk[u], i);
+  }
+  if (i < UNR && g < TPW) {
+    const int64_t k = warp_base + (int64_t)i * TPW + g;
+    if (k < nT) on_target_end(k, my_tok);
+  }
 }
 
 }  // namespace wg

@@ -72,6 +72,7 @@ struct UniqueArgs {
   int32_t* excl;
   int32_t* slot_of;
   HashTable ht;
+  DirectTable dt;          // FMT_DIRECT
   int pad32;               // PADDED: nbrs holds uint32 ids
   unsigned long long* status;
   unsigned* ctrl;
@@ -88,18 +89,25 @@ __device__ __forceinline__ int64_t clamp_count(const int64_t* d, int64_t cap, un
   return v;
 }
 
+// key-table formats (hash.cuh): 16 B hashed slots, 8 B hashed slots, a direct word per node
+enum { FMT_WIDE = 0, FMT_COMPACT = 1, FMT_DIRECT = 2 };
+
 template <bool PADDED>
 __device__ __forceinline__ void load_counts(const UniqueArgs& a, int64_t& nT, int64_t& nE) {
   nT = clamp_count(a.d_nT, a.capT, a.ctrl);
   nE = PADDED ? nT * a.M : clamp_count(a.d_nE, a.capE, a.ctrl);
 }
 
-template <bool PADDED, bool COMPACT>
+template <bool PADDED, int FMT>
 __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueArgs a) {
   pdl_enter();
   int64_t nT, nE;
   load_counts<PADDED>(a, nT, nE);
   const unsigned epoch = a.ctrl[CTRL_EPOCH];
+  constexpr bool COMPACT = FMT == FMT_COMPACT;
+  if (FMT == FMT_DIRECT) dtab_clear_ahead(a.dt, epoch);  // table e+1 is idle (standalone first kernel)
+  unsigned* const dt = FMT == FMT_DIRECT ? dtab_cur(a.dt, epoch) : nullptr;
+  const unsigned tag = FMT == FMT_DIRECT ? dtag(epoch) : 0u;
   const int64_t total = nT + nE;
   const int lane = threadIdx.x & 31;
   const int64_t warps = (int64_t)gridDim.x * (UQ_THREADS / 32);
@@ -116,13 +124,13 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueA
         const unsigned k = a.Mdiv.div((unsigned)j);
         key = ld_pad(a.nbrs, a.pad32, j);  // loaded together with the count (ignored for a padding slot)
         valid = (int)((unsigned)j - k * (unsigned)a.M) < a.cnt[k];
-        if (!valid) a.slot_of[q] = SLOT_EMPTY;  // padding slot: no sample here
+        if (!valid && FMT != FMT_DIRECT) a.slot_of[q] = SLOT_EMPTY;  // padding slot: no sample here
       } else {
         key = a.nbrs[q - nT];
       }
       if (valid && (key < 0 || key >= a.n)) {
         latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_ID_RANGE);
-        a.slot_of[q] = SLOT_BADID;  // a sample, but no key to number
+        if (FMT != FMT_DIRECT) a.slot_of[q] = SLOT_BADID;  // a sample, but no key to number
         valid = false;
       }
     }
@@ -138,6 +146,18 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueA
     const unsigned tmask = __ballot_sync(FULL_MASK, valid && is_target);
     if (valid && is_target && leader == lane && __popc(same & tmask) > 1)
       latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DUP_TARGET);
+    if (FMT == FMT_DIRECT) {  // no slots: the node's own word; targets check for an earlier target record
+      if (valid && leader == lane) {
+        if (is_target) {
+          const unsigned old = atomicMin(&dt[key], dword(tag, q));
+          if ((old >> DPOS_BITS) == tag && (int64_t)(old & DPOS_MASK) < nT)
+            latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DUP_TARGET);
+        } else {
+          atomicMin(&dt[key], dword(tag, q));
+        }
+      }
+      continue;
+    }
     long long slot = -1;
     if (valid && leader == lane) {
       if (COMPACT) {
@@ -160,14 +180,14 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueA
   }
 }
 
-template <bool COMPACT>
+template <int FMT>
 __device__ __forceinline__ int64_t min_pos_at(const UniqueArgs& a, int32_t slot) {
   if (slot < 0) return -1;
-  if (COMPACT) return chash_min_pos(a.ht, slot);
+  if (FMT == FMT_COMPACT) return chash_min_pos(a.ht, slot);
   return (int64_t)(a.ht.slots[slot].val & KEY_MASK);
 }
 
-template <bool PADDED, int UQ_ITEMS, bool COMPACT>
+template <bool PADDED, int UQ_ITEMS, int FMT>
 __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArgs a) {
   pdl_enter();
   // warp-striped: warp w of the tile covers 32 * UQ_ITEMS consecutive positions, lane l the
@@ -183,6 +203,9 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArg
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const unsigned lt = (1u << lane) - 1u;
 
+  const unsigned* const dt = FMT == FMT_DIRECT ? dtab_cur(a.dt, epoch) : nullptr;
+  const unsigned tag = FMT == FMT_DIRECT ? dtag(epoch) : 0u;
+  const int64_t pad_key = a.pad32 ? (int64_t)0xFFFFFFFFu : (int64_t)-1;  // direct: sampler's padding slots
   const int64_t tile_start = (int64_t)blockIdx.x * UQ_TILE;
   if (nE == 0) {
     if (blockIdx.x == 0 && tid == 0) {
@@ -204,16 +227,22 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArg
       const int64_t j = wbase + 32 * t;
       const bool in = j < nE;
       // every position's slot (the insert pass wrote SLOT_EMPTY for padding): no count read needed
-      slots[t] = in ? a.slot_of[nT + j] : SLOT_EMPTY;
+      if (FMT != FMT_DIRECT) slots[t] = in ? a.slot_of[nT + j] : SLOT_EMPTY;
       keys[t] = in ? (PADDED ? ld_pad(a.nbrs, a.pad32, j) : a.nbrs[j]) : -1;  // needed after the scan: issued now
     }
     unsigned long long wv = 0, wf = 0;
 #pragma unroll
     for (int t = 0; t < UQ_ITEMS; ++t) {
       const int64_t j = wbase + 32 * t;
-      const bool valid = j < nE && (!PADDED || slots[t] != SLOT_EMPTY);
+      bool valid;
+      if (FMT == FMT_DIRECT) {  // padding slots hold pad_key; the key's own word holds its first position
+        valid = j < nE && (!PADDED || keys[t] != pad_key);
+        mps[t] = (valid && keys[t] >= 0 && keys[t] < a.n) ? dtab_min_pos(dt, tag, keys[t]) : -1;
+      } else {
+        valid = j < nE && (!PADDED || slots[t] != SLOT_EMPTY);
+        mps[t] = min_pos_at<FMT>(a, slots[t]);  // independent L2 reads
+      }
       poss[t] = (PADDED && a.out_pos && valid) ? a.pos_pad[j] : 0;
-      mps[t] = min_pos_at<COMPACT>(a, slots[t]);  // independent L2 reads
       vm[t] = __ballot_sync(FULL_MASK, valid);
     }
 #pragma unroll
@@ -274,8 +303,10 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArg
       a.ctrl[CTRL_DONE_UNIQUE] = 0u;
       // the table is not read again in this call: advance its epoch (the compact table cycles
       // through 255 epochs and is cleared when a cycle restarts; the wide one has 2^23)
-      if (COMPACT)
-        a.ctrl[CTRL_EPOCH] = epoch + 1u >= CEPOCHS * 4096u ? (epoch + 1u) % CEPOCHS + CEPOCHS : epoch + 1u;
+      // (the counter wraps modulo 2 * CEPOCHS: compact_epoch and the direct table's parity continue)
+      if (FMT != FMT_WIDE)
+        a.ctrl[CTRL_EPOCH] =
+            epoch + 1u >= 2u * CEPOCHS * 2048u ? (epoch + 1u) % (2u * CEPOCHS) + 2u * CEPOCHS : epoch + 1u;
       else if (epoch + 1u >= EPOCH_MAX)
         latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_EPOCH);
       else
@@ -312,26 +343,29 @@ cudaError_t launch_hash_clear(wg_dsm* h, cudaStream_t st) {
                     reinterpret_cast<unsigned long long*>(h->ws.hslots), (int64_t)h->ws.hcap, (const unsigned*)h->ws.ctrl);
 }
 
-template <bool C>
+template <int FMT>
 static cudaError_t launch_insert_flag(wg_dsm* h, bool padded, int items, int64_t ib, unsigned fb, const UniqueArgs& a,
                                       cudaStream_t st) {
-  cudaError_t e = padded ? launch_pdl(unique_insert_kernel<true, C>, (unsigned)ib, UQ_THREADS, 0, st, a)
-                         : launch_pdl(unique_insert_kernel<false, C>, (unsigned)ib, UQ_THREADS, 0, st, a);
-  if (e != cudaSuccess) return e;
-  stage_mark(h, st);
+  // the fused hop with the direct table has no insert pass (its sampler inserted every key)
+  if (!(padded && FMT == FMT_DIRECT)) {
+    cudaError_t e = padded ? launch_pdl(unique_insert_kernel<true, FMT>, (unsigned)ib, UQ_THREADS, 0, st, a)
+                           : launch_pdl(unique_insert_kernel<false, FMT>, (unsigned)ib, UQ_THREADS, 0, st, a);
+    if (e != cudaSuccess) return e;
+    stage_mark(h, st);
+  }
   if (padded) {
     switch (items) {
-      case 8: return launch_pdl(unique_flag_kernel<true, 8, C>, fb, UQ_THREADS, 0, st, a);
-      case 4: return launch_pdl(unique_flag_kernel<true, 4, C>, fb, UQ_THREADS, 0, st, a);
-      case 2: return launch_pdl(unique_flag_kernel<true, 2, C>, fb, UQ_THREADS, 0, st, a);
-      default: return launch_pdl(unique_flag_kernel<true, 1, C>, fb, UQ_THREADS, 0, st, a);
+      case 8: return launch_pdl(unique_flag_kernel<true, 8, FMT>, fb, UQ_THREADS, 0, st, a);
+      case 4: return launch_pdl(unique_flag_kernel<true, 4, FMT>, fb, UQ_THREADS, 0, st, a);
+      case 2: return launch_pdl(unique_flag_kernel<true, 2, FMT>, fb, UQ_THREADS, 0, st, a);
+      default: return launch_pdl(unique_flag_kernel<true, 1, FMT>, fb, UQ_THREADS, 0, st, a);
     }
   }
   switch (items) {
-    case 8: return launch_pdl(unique_flag_kernel<false, 8, C>, fb, UQ_THREADS, 0, st, a);
-    case 4: return launch_pdl(unique_flag_kernel<false, 4, C>, fb, UQ_THREADS, 0, st, a);
-    case 2: return launch_pdl(unique_flag_kernel<false, 2, C>, fb, UQ_THREADS, 0, st, a);
-    default: return launch_pdl(unique_flag_kernel<false, 1, C>, fb, UQ_THREADS, 0, st, a);
+    case 8: return launch_pdl(unique_flag_kernel<false, 8, FMT>, fb, UQ_THREADS, 0, st, a);
+    case 4: return launch_pdl(unique_flag_kernel<false, 4, FMT>, fb, UQ_THREADS, 0, st, a);
+    case 2: return launch_pdl(unique_flag_kernel<false, 2, FMT>, fb, UQ_THREADS, 0, st, a);
+    default: return launch_pdl(unique_flag_kernel<false, 1, FMT>, fb, UQ_THREADS, 0, st, a);
   }
 }
 
@@ -345,6 +379,7 @@ static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, c
   // largest hop.  Slots outside the prefix, or left by earlier calls, carry older epochs and read as
   // empty.
   a.ht = HashTable{h->ws.hslots, (unsigned long long)table_prefix(h, a.capT + a.capE), h->ws.compact};
+  a.dt = DirectTable{{h->ws.dtab[0], h->ws.dtab[1]}, h->n};
   a.status = h->ws.status_unique;
   a.ctrl = h->ws.ctrl;
   a.n = h->n;
@@ -358,14 +393,16 @@ static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, c
   const int64_t tile = (int64_t)items * UQ_THREADS;
   const unsigned fb = (unsigned)(a.capE > 0 ? (a.capE + tile - 1) / tile : 1);
   cudaError_t e;
-  if (!padded && h->ws.compact) {
+  if (!padded && h->ws.compact && !h->ws.direct) {
     e = launch_hash_clear(h, st);
     if (e != cudaSuccess) return e;
   }
-  if (h->ws.compact)
-    e = launch_insert_flag<true>(h, padded, items, ib, fb, a, st);
+  if (h->ws.direct)
+    e = launch_insert_flag<FMT_DIRECT>(h, padded, items, ib, fb, a, st);
+  else if (h->ws.compact)
+    e = launch_insert_flag<FMT_COMPACT>(h, padded, items, ib, fb, a, st);
   else
-    e = launch_insert_flag<false>(h, padded, items, ib, fb, a, st);
+    e = launch_insert_flag<FMT_WIDE>(h, padded, items, ib, fb, a, st);
   if (e != cudaSuccess) return e;
   stage_mark(h, st);
   if (a.capE > 0) {
@@ -409,14 +446,15 @@ cudaError_t launch_append_unique(wg_dsm* h, const int64_t* T, int64_t capT, cons
 }
 
 cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap, const int64_t* d_n, int fanout,
-                                 uint64_t seed, const uint64_t* d_seed, int hop, bool want_pos, cudaStream_t st);
+                                 uint64_t seed, const uint64_t* d_seed, int hop, bool want_pos, cudaStream_t st,
+                                 int64_t* U, int32_t* dup);
 
 cudaError_t launch_hop(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t* d_nT, int fanout, uint64_t seed,
                        const uint64_t* d_seed, int hop, int64_t* out_row_ptr, int64_t* out_nbrs, int32_t* out_pos,
                        int64_t* d_num_edges, int64_t* U, int64_t* d_nU, int32_t* sub_col, int32_t* dup,
                        cudaStream_t st, cudaStream_t side) {
   h->stage_i = 0;
-  cudaError_t e = launch_sample_padded(h, T, capT, d_nT, fanout, seed, d_seed, hop, out_pos != nullptr, st);
+  cudaError_t e = launch_sample_padded(h, T, capT, d_nT, fanout, seed, d_seed, hop, out_pos != nullptr, st, U, dup);
   if (e != cudaSuccess) return e;
   stage_mark(h, st);
   UniqueArgs a{};

@@ -81,6 +81,11 @@ struct Workspace {
   HashSlot* hslots = nullptr;            // [hcap] append-unique hash table (hash.cuh)
   int64_t hcap = 0;                      // slots (a multiple of 8, < 2^31); each call uses a prefix
   int compact = 0;                       // 8 B slots {epoch8, key28, pos28} (hash.cuh), else 16 B slots
+  // direct table (hash.cuh, graphs small enough that a word per NODE beats a hashed slot per key): two
+  // uint32 arrays of num_nodes words {255 - compact_epoch, first position}, epoch e uses dtab[e & 1];
+  // the fused hop's sampler inserts into it, so a hop has no insert pass and no slot_of round trip
+  int direct = 0;
+  unsigned* dtab[2] = {nullptr, nullptr};
   int pad32 = 0;                         // padded sampler slots hold uint32 ids (num_nodes < 2^32)
   unsigned long long* status_sample = nullptr;  // decoupled look-back tile status
   unsigned long long* status_unique = nullptr;
@@ -100,6 +105,13 @@ constexpr unsigned EPOCH_MAX = (1u << 23) - 1;
 // compact hash table (8 B slots): epochs 1..255 cycle; the table is cleared when a cycle restarts
 constexpr unsigned CEPOCHS = 255;
 __host__ __device__ inline unsigned compact_epoch(unsigned e) { return e % CEPOCHS + 1u; }
+// Direct table eligibility: positions fit its 24-bit field and the two tables stay small (products:
+// 2 x 9.8 MB).  Above that (papers100M: 2 x 444 MB, whose 700k random words per hop would each cost a
+// line) the hashed formats touch fewer lines.  WG_DSM_HASHED forces the hashed formats.
+constexpr int DPOS_BITS = 24;
+#ifndef WG_DIRECT_MAX_NODES
+#define WG_DIRECT_MAX_NODES (int64_t(1) << 24)
+#endif
 constexpr int EXCL_RING = 4;
 // Hash-table sizing (measured on B200): a call uses a prefix of
 // HASH_FACTOR x its own key bound slots (at least HASH_MIN_SLOTS), so small hops touch few lines.

@@ -201,6 +201,13 @@ class DSM:
         arr = (ctypes.c_void_p * max(len(events), 1))(*[e.cuda_event for e in events])
         check(lib().wg_dsm_set_stage_events(self.h, arr, len(events)))
 
+    def unique_format(self):
+        """Append Unique key-table format of this handle's workspace (wg_dsm_unique_format):
+        WG_UNIQUE_WIDE / WG_UNIQUE_COMPACT / WG_UNIQUE_DIRECT."""
+        f = ctypes.c_int32(0)
+        check(lib().wg_dsm_unique_format(self.h, ctypes.byref(f)))
+        return f.value
+
     def debug_set_epoch(self, epoch):
         """Test hook: set the workspace's hash-table epoch (wg_dsm_debug_set_epoch)."""
         check(lib().wg_dsm_debug_set_epoch(self.h, int(epoch)))

@@ -53,3 +53,20 @@ def gpu_unique(dsm, T, nbrs, with_dup=True):
     torch.cuda.synchronize()
     u = int(nU.item())
     return U[:u].cpu().numpy(), sc[:len(nbrs)].cpu().numpy(), (dup[:u].cpu().numpy() if with_dup else None)
+
+
+def gpu_sample_hop(dsm, T, M, seed, hop):
+    """One fused hop (wg_sample_hop, no side stream): row_ptr, nbrs, pos, U, sub_col, dup."""
+    t = torch.from_numpy(np.asarray(T, dtype=np.int64)).cuda()
+    o = dsm.sample_hop(t, M, seed, hop, with_pos=True, with_dup=True)
+    torch.cuda.synchronize()
+    e, u = int(o["num_edges"].item()), int(o["num_unique"].item())
+    return (o["row_ptr"].cpu().numpy(), o["nbrs"][:e].cpu().numpy(), o["pos"][:e].cpu().numpy(),
+            o["unique"][:u].cpu().numpy(), o["sub_col"][:e].cpu().numpy(), o["dup"][:u].cpu().numpy())
+
+
+def oracle_sample_hop(row_ptr, col, T, M, seed, hop):
+    """The fused hop's definition: oracle sampling, then oracle append-unique of its neighbours."""
+    rp, nb, pos = oracle_hop(row_ptr, col, T, M, seed, hop)
+    U, sc, dup = oracle.append_unique(np.asarray(T, dtype=np.int64), nb)
+    return rp, nb, pos, U, sc, dup

@@ -19,7 +19,8 @@ from gpu_helpers import csr_from_rows
 pytestmark = pytest.mark.gpu
 
 FLAG_SETS = [0, pkg.WG_DSM_COL32, pkg.WG_DSM_WIDE_HASH, pkg.WG_DSM_PAD64 | pkg.WG_DSM_COL32,
-             pkg.WG_DSM_WHOLE_ROWS, pkg.WG_DSM_CSR_REPLICATED | pkg.WG_DSM_COL32, pkg.WG_DSM_CSR_REPLICATED]
+             pkg.WG_DSM_WHOLE_ROWS, pkg.WG_DSM_CSR_REPLICATED | pkg.WG_DSM_COL32, pkg.WG_DSM_CSR_REPLICATED,
+             pkg.WG_DSM_HASHED | pkg.WG_DSM_COL32, pkg.WG_DSM_HASHED | pkg.WG_DSM_PAD64]
 
 
 def _random_graph(rng, n):
@@ -124,7 +125,7 @@ def test_random_standalone_ops_bit_exact(case):
     M = int(rng.choice([1, 4, 5, 10, 16, 31, 32, 33, 64, 129]))
     nT = int(rng.integers(0, min(n, 300) + 1))
     T = rng.choice(n, nT, replace=False).astype(np.int64)
-    flags = [0, pkg.WG_DSM_COL32, pkg.WG_DSM_WIDE_HASH, pkg.WG_DSM_PAD64][case % 4]
+    flags = [0, pkg.WG_DSM_COL32, pkg.WG_DSM_WIDE_HASH, pkg.WG_DSM_PAD64, pkg.WG_DSM_HASHED][case % 5]
     dsms, feat = _make(rp, col, n, 12, "fp32", flags, 1, max(nT * (M + 1), 1))
     dsm = dsms[0]
     try:

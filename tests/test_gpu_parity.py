@@ -13,7 +13,7 @@ from paper_conf_sc_yanglql22_b200 import loader
 from synth import providers
 from synth import features, graph, presets, seeds
 
-from gpu_helpers import csr_from_rows, gpu_hop, gpu_unique, make_dsm, oracle_hop
+from gpu_helpers import csr_from_rows, gpu_hop, gpu_sample_hop, gpu_unique, make_dsm, oracle_hop, oracle_sample_hop
 
 pytestmark = pytest.mark.gpu
 
@@ -528,15 +528,20 @@ def test_epoch_exhaustion_and_reset():
     dsm.destroy()
 
 
-def test_compact_table_epoch_cycles(tiny):
-    """The compact 8 B hash table cycles through 255 epochs and is cleared when a cycle restarts
-    (by the fused hop's sampler, or before a standalone insert): 140 tiny batches (280 fused hops,
-    more than a whole cycle, starting just before a restart) and standalone append-unique calls
-    across a restart, all bit-exact against the oracle."""
+@pytest.mark.parametrize("fmt", ["direct", "compact"])
+def test_compact_table_epoch_cycles(tiny, fmt):
+    """The compact 8 B hash table and the direct tables cycle through 255 epochs and are cleared when
+    a cycle restarts (compact: by the fused hop's sampler, or before a standalone insert; direct: the
+    op at epoch e clears the idle table of epoch e+1): 140 tiny batches (280 fused hops, more than a
+    whole cycle, starting just before a restart) and standalone append-unique calls across a
+    restart, all bit-exact against the oracle."""
+    fl = 0 if fmt == "direct" else pkg.WG_DSM_HASHED
+    want = pkg.WG_UNIQUE_DIRECT if fmt == "direct" else pkg.WG_UNIQUE_COMPACT
     p, rp, col = tiny
     rows = providers.host_row_provider(p.graph(), rp, col)
     feats = providers.host_feat_provider(p)
-    dsm, _ = loader.build_dsm(p, on_device=False)
+    dsm, _ = loader.build_dsm(p, on_device=False, flags=fl)
+    assert dsm.unique_format() == want
     dsm.debug_set_epoch(250)
     pipe = pkg.MiniBatchPipeline(dsm, p.fanouts, p.seeds_per_batch, with_pos=True, with_dup=True)
     pipe.run(torch.from_numpy(seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 0)).cuda(), 5)
@@ -550,9 +555,12 @@ def test_compact_table_epoch_cycles(tiny):
     assert dsm.device_error() == 0
     dsm.destroy()
     rng = np.random.default_rng(3)
-    d2 = make_dsm(np.zeros(2001, np.int64), np.zeros(0, np.int64), max_keys=4096)
+    d2 = make_dsm(np.zeros(2001, np.int64), np.zeros(0, np.int64), max_keys=4096, flags=fl)
+    assert d2.unique_format() == want
     d2.debug_set_epoch(250)
     for i in range(300):
+        if i == 150 and fmt == "direct":   # fused hops and standalone calls share the epoch sequence
+            d2.debug_set_epoch(508)
         T = rng.choice(2000, 40, replace=False).astype(np.int64)
         nb = rng.integers(0, 2000, 600).astype(np.int64)
         U, sc, dup = gpu_unique(d2, T, nb)
@@ -587,7 +595,7 @@ def test_gather_occupancy_setting(tiny):
 
 
 @pytest.mark.parametrize("flags", ["WG_DSM_WIDE_HASH", "WG_DSM_PAD64", "WG_DSM_WIDE_HASH|WG_DSM_PAD64", "COL64",
-                                   "COL64|WG_DSM_PAD64"])
+                                   "COL64|WG_DSM_PAD64", "WG_DSM_HASHED", "WG_DSM_HASHED|WG_DSM_PAD64"])
 def test_table_and_slot_formats(tiny, flags):
     """The non-default hash-table / padded-slot / column formats (16 B wide slots claimed with one 128-bit
     CAS, int64 padded sampler slots, int64 col_idx instead of the loader's default uint32) stay bit-exact: 12 tiny batches through the fused
@@ -618,3 +626,41 @@ def test_table_and_slot_formats(tiny, flags):
         assert np.array_equal(U, Uo) and np.array_equal(sc, sco) and np.array_equal(dup, dupo), i
     assert d2.device_error() == 0
     d2.destroy()
+
+
+def test_unique_format_selection(tiny):
+    """wg_dsm_unique_format: the direct table for small graphs, the compact hash with WG_DSM_HASHED, the
+    wide hash with WG_DSM_WIDE_HASH; and a graph too large for the direct table (num_nodes > 2^24) is
+    hashed."""
+    p, rp, col = tiny
+    for fl, want in ((0, pkg.WG_UNIQUE_DIRECT), (pkg.WG_DSM_HASHED, pkg.WG_UNIQUE_COMPACT),
+                     (pkg.WG_DSM_WIDE_HASH, pkg.WG_UNIQUE_WIDE),
+                     (pkg.WG_DSM_WIDE_HASH | pkg.WG_DSM_HASHED, pkg.WG_UNIQUE_WIDE)):
+        dsm = make_dsm(np.zeros(101, np.int64), np.zeros(0, np.int64), max_keys=64, flags=fl)
+        assert dsm.unique_format() == want, fl
+        dsm.destroy()
+    big = make_dsm(np.zeros((1 << 24) + 2, np.int64), np.zeros(0, np.int64), max_keys=64)
+    assert big.unique_format() == pkg.WG_UNIQUE_COMPACT
+    big.destroy()
+
+
+@pytest.mark.parametrize("fl", [0, "WG_DSM_HASHED"])
+def test_direct_fused_hop_duplicate_and_bad_targets(fl):
+    """Fused hop (the direct table's sampler-side inserts): duplicate targets latch WG_DEVERR_DUP_TARGET
+    (A8), out-of-range targets and neighbours latch WG_DEVERR_ID_RANGE (B3), and a valid batch after
+    them is bit-exact again."""
+    flags = 0 if fl == 0 else getattr(pkg, fl)
+    n, (rp, col) = _edge_graph()
+    dsm = make_dsm(rp, col, max_keys=1 << 16, flags=flags)
+    T = np.array([5, 9, 5, 7], np.int64)
+    gpu_sample_hop(dsm, T, 4, 1, 0)
+    assert dsm.device_error() & 0x2               # (device_error clears the word)
+    gpu_sample_hop(dsm, np.array([5, n + 9, 7], np.int64), 4, 1, 0)
+    assert dsm.device_error() & 0x1
+    T = np.array([5, 9, 7, 11, 4999, 0, 1, 2], np.int64)
+    got = gpu_sample_hop(dsm, T, 4, 3, 2)
+    ref = oracle_sample_hop(rp, col, T, 4, 3, 2)
+    for g, r in zip(got, ref):
+        assert np.array_equal(g, r)
+    assert dsm.device_error() == 0
+    dsm.destroy()
