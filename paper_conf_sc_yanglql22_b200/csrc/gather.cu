@@ -133,10 +133,27 @@ __device__ __forceinline__ void st_out<u32x8>(u32x8* p, const u32x8& r) {
                : "memory");
 }
 
+// DENSE16 (V = u32x8 only): rows of R bytes with R % 32 == 16 (products: 400 B) written DENSELY (pitch R):
+// chunk c of a row is still the 32 B source piece [32c, 32c + 32) -- one 32 B load from the body, 16 B
+// for the last chunk -- but its destination row * R + 32c is only 16 B aligned, so it is stored as two
+// 16 B vectors (one for the last chunk).  Consecutive threads still cover consecutive output bytes, so
+// L2 merges the halves into whole sectors: no 16 B pitch padding reaches DRAM.
+template <typename V>
+__device__ __forceinline__ void st_out_dense16(uint8_t* p, const V& r, bool half);
+template <>
+__device__ __forceinline__ void st_out_dense16<u32x8>(uint8_t* p, const u32x8& r, bool half) {
+  asm volatile("st.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(r.v[0]), "r"(r.v[1]), "r"(r.v[2]), "r"(r.v[3])
+               : "memory");
+  if (!half)
+    asm volatile("st.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p + 16), "r"(r.v[4]), "r"(r.v[5]), "r"(r.v[6]),
+                 "r"(r.v[7])
+                 : "memory");
+}
+
 // MINB: resident blocks per SM the register allocation must allow -- GATHER_MINB for a gather that
 // fills the GPU alone; GATHER_LEAN_MINB (fewer registers, a few spills) for throughput-mode gathers
 // capped at a block or two per SM, whose register file the other streams' hop kernels then use.
-template <typename V, int GATHER_UNROLL, int MINB = GATHER_MINB>
+template <typename V, int GATHER_UNROLL, int MINB = GATHER_MINB, bool DENSE16 = false>
 __global__ void __launch_bounds__(GATHER_THREADS, MINB) gather_kernel(const GatherArgs a) {
   pdl_enter();
   KT_BEGIN(3);
@@ -155,7 +172,10 @@ __global__ void __launch_bounds__(GATHER_THREADS, MINB) gather_kernel(const Gath
   const unsigned cpr = a.cpr.d;
   const unsigned total = (unsigned)(n * cpr);  // < 2^31 (checked on the host)
   const unsigned stride = gridDim.x * GATHER_THREADS;
-  V* __restrict__ out = reinterpret_cast<V*>(a.out + begin * (int64_t)cpr * (int64_t)sizeof(V));
+  // DENSE16: rows of (cpr - 1) * 32 + 16 bytes
+  const int64_t out_row = DENSE16 ? (int64_t)cpr * (int64_t)sizeof(V) - 16 : (int64_t)cpr * (int64_t)sizeof(V);
+  V* __restrict__ out = reinterpret_cast<V*>(a.out + begin * out_row);
+  uint8_t* __restrict__ out8 = a.out + begin * out_row;
   const unsigned long long pol = l2_evict_last_policy();
   for (unsigned c0 = blockIdx.x * GATHER_THREADS + threadIdx.x; c0 < total; c0 += stride * GATHER_UNROLL) {
     V val[GATHER_UNROLL];
@@ -180,8 +200,17 @@ __global__ void __launch_bounds__(GATHER_THREADS, MINB) gather_kernel(const Gath
       }
     }
 #pragma unroll
-    for (int j = 0; j < GATHER_UNROLL; ++j)
-      if (dst[j] < total) st_out<V>(&out[dst[j]], val[j]);
+    for (int j = 0; j < GATHER_UNROLL; ++j) {
+      if (dst[j] < total) {
+        if (DENSE16) {
+          const unsigned row = a.cpr.div(dst[j]);
+          const unsigned colc = dst[j] - row * cpr;
+          st_out_dense16<V>(out8 + (int64_t)row * out_row + colc * 32u, val[j], colc == cpr - 1);
+        } else {
+          st_out<V>(&out[dst[j]], val[j]);
+        }
+      }
+    }
   }
   KT_END(3, "gather", n);
 }
@@ -193,6 +222,28 @@ cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int6
   // copy width per row: the row, or -- for a pitched output (out_pitch > row_bytes, <= the shard's
   // row pitch) -- the whole output pitch including padding, so 400 B rows can move as 13 x 32 B
   const int64_t cw = out_pitch > rb ? out_pitch : rb;
+  // dense rows of 32k + 16 bytes (k >= 1) whose stored body is whole 32 B pieces: 32 B loads, 16 B stores
+  const bool dense16 = cw == rb && rb % 32 == 16 && rb >= 48 && oa % 16 == 0 &&
+                       (h->tail_pitch == 0 || h->body_bytes % 32 == 0) && (h->feat_stride % 32 == 0) &&
+                       (h->tail_pitch == 0 || h->tail_pitch % 16 == 0);
+  if (dense16) {
+    GatherArgs a{h->view, ids, cap, d_n, d_begin, static_cast<uint8_t*>(out), h->ws.ctrl, FastDiv((unsigned)((rb + 16) / 32))};
+    static int occ16 = 0;
+    if (!occ16) {
+      int nb = 0;
+      cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, gather_kernel<u32x8, V32_UNROLL, GATHER_MINB, true>, GATHER_THREADS, 0);
+      occ16 = nb > 0 ? nb : 4;
+    }
+    const int want = h->gather_bps;
+    const int per_sm = (want > 0 && want < occ16) ? want : occ16;
+    const int64_t total = cap * ((rb + 16) / 32);
+    int64_t blocks = (total + GATHER_THREADS * V32_UNROLL - 1) / (GATHER_THREADS * V32_UNROLL);
+    const int64_t max_blocks = (int64_t)h->sm_count * per_sm;
+    blocks = blocks < 1 ? 1 : (blocks > max_blocks ? max_blocks : blocks);
+    if (per_sm <= 2)
+      return launch_pdl(gather_kernel<u32x8, LEAN_UNROLL, GATHER_LEAN_MINB, true>, (unsigned)blocks, GATHER_THREADS, 0, st, a);
+    return launch_pdl(gather_kernel<u32x8, V32_UNROLL, GATHER_MINB, true>, (unsigned)blocks, GATHER_THREADS, 0, st, a);
+  }
   const int vb = (cw % 32 == 0 && oa % 32 == 0)   ? 32
                  : (cw % 16 == 0 && oa % 16 == 0) ? 16
                  : (cw % 4 == 0 && oa % 4 == 0)   ? 4

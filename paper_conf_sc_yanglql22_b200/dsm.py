@@ -313,7 +313,9 @@ class DSM:
         self.gather_occupancy = int(blocks_per_sm)
 
     def out_pitch(self):
-        """Output row pitch that lets the gather move whole 32 B vectors (row bytes rounded up to 32)."""
+        """Output row pitch that lets the gather move whole 32 B vectors (row bytes rounded up to 32).  Dense
+        rows of 32k + 16 bytes also move as 32 B source pieces (stored as 16 B halves) and write 4 % fewer
+        bytes, but measured slower in the throughput pass (profiles/r02/ab_log.md), so buffers are pitched."""
         return (self.row_bytes + 31) // 32 * 32
 
     def gather(self, ids, n_ids=None, n_ids_dev=None, out=None, stream=None):

@@ -80,7 +80,7 @@ class MiniBatchPipeline:
                 dup=torch.zeros(max(T + E, 1), **i32) if with_dup else None))
         # X is pitched to a 32 B multiple (DSM.out_pitch) so every row moves as whole 32 B vectors; X_rows is
         # the [U, row_bytes] view of the feature bytes (self.X[:, :row_bytes]).  x_pitch: another output
-        # pitch (a multiple of 16 >= row_bytes, e.g. 400 = dense 400 B rows, 16 B vectors; A/B only)
+        # pitch (a multiple of 16 >= row_bytes, e.g. 400 = dense 400 B rows: 32 B loads, 16 B stores; A/B)
         pitch = dsm.out_pitch() if x_pitch is None else x_pitch
         self.X = torch.zeros((max(self.U_cap[-1], 1), pitch), dtype=torch.uint8, device=dev) \
             if dsm.row_bytes else None

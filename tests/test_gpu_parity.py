@@ -240,8 +240,9 @@ def test_gather_rows(dim, dtype):
             torch.cuda.synchronize()
             assert np.array_equal(Xp[:, :rb].cpu().numpy(), exp)
         if rb % 32 == 16 and len(ids) > 4:
-            # dense rows of R % 32 == 16 (the 16 B-vector path): whole lists and row ranges starting / ending
-            # on odd rows; bytes outside the range stay put
+            # dense rows of R % 32 == 16 (32 B source pieces stored as 16 B halves for R >= 48, else the
+            # 16 B-vector path): whole lists and row ranges starting / ending on odd rows; bytes outside the
+            # range stay put
             for b, e in ((0, len(ids)), (1, len(ids) - 1), (3, 4), (2, len(ids) - 3)):
                 Xd = torch.full((len(ids), rb), 0xCD, dtype=torch.uint8, device="cuda")
                 be = torch.tensor([b, e], dtype=torch.int64, device="cuda")
@@ -271,8 +272,8 @@ def test_feat_whole_rows_flag():
 
 
 def test_pipeline_dense_x_400b_rows():
-    """A pipeline with a dense X (pitch = the 400 B row, the 16 B-vector gather; incremental gathers start on
-    odd rows) is bit-exact."""
+    """A pipeline with a dense X (pitch = the 400 B row, 32 B source pieces stored as 16 B halves; incremental
+    gathers start on odd rows) is bit-exact, and so is the 32 B-pitched X (416 B)."""
     n, dim = 3000, 100
     rng = np.random.default_rng(5)
     rows = [np.unique(rng.integers(0, n, rng.integers(0, 40))) for _ in range(n)]
@@ -280,19 +281,21 @@ def test_pipeline_dense_x_400b_rows():
     g_rp, g_col = csr_from_rows(rows)
     feat = features.feature_bytes(presets.FEAT_SEED, np.arange(n), dim, "fp32")
     dsm = make_dsm(g_rp, g_col, feat, dim, "fp32", max_keys=1 << 16)
-    pipe = pkg.MiniBatchPipeline(dsm, [7, 4], 101, with_pos=True, with_dup=True, x_pitch=dim * 4)
+    assert dsm.out_pitch() == 416
     rowsf = providers.host_row_provider(None, g_rp, g_col)
 
     def feats(ids):
         u = np.unique(np.asarray(ids, dtype=np.int64))
         return u, features.feature_bytes(presets.FEAT_SEED, u, dim, "fp32")
-    for b in range(6):
-        S = np.random.default_rng(100 + b).choice(n, 101 - 2 * b, replace=False).astype(np.int64)
-        pipe.run(torch.from_numpy(S).cuda(), 77 + b)
-        torch.cuda.synchronize()
-        _check_batch(pipe, oracle.minibatch(rowsf, feats, S, [7, 4], 77 + b), [7, 4])
-        if b == 0:
-            pipe.capture()
+    for xp in (dim * 4, 416):
+        pipe = pkg.MiniBatchPipeline(dsm, [7, 4], 101, with_pos=True, with_dup=True, x_pitch=xp)
+        for b in range(6):
+            S = np.random.default_rng(100 + b).choice(n, 101 - 2 * b, replace=False).astype(np.int64)
+            pipe.run(torch.from_numpy(S).cuda(), 77 + b)
+            torch.cuda.synchronize()
+            _check_batch(pipe, oracle.minibatch(rowsf, feats, S, [7, 4], 77 + b), [7, 4])
+            if b == 0:
+                pipe.capture()
     assert dsm.device_error() == 0
     dsm.destroy()
 
