@@ -1,8 +1,9 @@
 #!/usr/bin/env python
-"""One products-shaped batch for ncu: 3 warm-up batches, then one batch whose 13 kernels
-(3 hops x sample/insert/flag/relabel + the whole gather) are the ones to capture:
+"""One products-shaped batch for ncu: 3 warm-up batches, then one batch whose kernels (3 hops x
+sample/flag/relabel with the direct key table, + insert with a hashed one; then the whole gather) are the
+ones to capture:
 
-    ncu --set full -k regex:'sample_kernel|unique_|gather_kernel' -s 39 -c 13 python profiles/ncu_step.py
+    ncu --set full -k regex:'sample_kernel|unique_|gather_kernel' -s 30 -c 10 python profiles/ncu_step.py
 """
 import os
 import sys
