@@ -70,10 +70,11 @@ __device__ __forceinline__ int64_t chash_min_pos(const HashTable& t, long long s
 
 // ---- direct table: one 32-bit word per node v, [31:24] 255 - compact_epoch(e) (1..255), [23:0] the first
 // position of v in the current call.  A newer epoch has a SMALLER tag, so one atomicMin of the whole word
-// both overrides a stale word and keeps the minimum position; 0xFFFFFFFF is empty.  Epoch e uses table
-// e & 1; the op running at epoch e clears table (e+1) & 1 (idle: its last use was epoch e-1, finished)
-// when compact_epoch(e+1) <= 2, i.e. when a 255-epoch cycle restarts there -- the tables are never
-// cleared per call.  No slot, no probe, no claim: a neighbour insert is a fire-and-forget RED.MIN.
+// both overrides a stale word and keeps the minimum position; 0xFFFFFFFF is empty.  Epochs come in cycles
+// of CEPOCHS; cycle c = e / CEPOCHS uses table c & 1 for all its epochs, so consecutive hops and batches of
+// a workspace keep hitting the same (L2-resident) lines.  The first op of cycle c clears table (c+1) & 1
+// -- idle: it served cycle c-1, whose ops have all finished -- so the next cycle starts on a clean table;
+// the tables are never cleared per call.  No slot, no probe, no claim: a neighbour insert is one RED.MIN.
 struct DirectTable {
   unsigned* t[2];
   int64_t n;  // words per table (num_nodes)
@@ -81,14 +82,14 @@ struct DirectTable {
 constexpr unsigned DPOS_MASK = (1u << DPOS_BITS) - 1u;
 __device__ __forceinline__ unsigned dtag(unsigned epoch) { return 255u - compact_epoch(epoch); }
 __device__ __forceinline__ unsigned dword(unsigned tag, int64_t q) { return (tag << DPOS_BITS) | (unsigned)q; }
-__device__ __forceinline__ unsigned* dtab_cur(const DirectTable& d, unsigned epoch) { return d.t[epoch & 1u]; }
+__device__ __forceinline__ unsigned* dtab_cur(const DirectTable& d, unsigned epoch) {
+  return ((epoch / CEPOCHS) & 1u) ? d.t[1] : d.t[0];
+}
 // First position recorded for v in this epoch, or -1 (not inserted in this epoch).
 __device__ __forceinline__ int64_t dtab_min_pos(const unsigned* t, unsigned tag, int64_t v) {
   const unsigned w = t[v];
   return (w >> DPOS_BITS) == tag ? (int64_t)(w & DPOS_MASK) : -1;
 }
-// Called by every thread of the FIRST kernel of an append-unique (the fused hop's sampler, or the
-// standalone insert pass): clear the table of epoch e+1 if a cycle restarts there (grid-strided).
 static __device__ __noinline__ void dtab_clear_words(unsigned* t, int64_t n) {
   uint4* w = reinterpret_cast<uint4*>(t);
   const int64_t n4 = (n + 3) / 4;  // tables are allocated in whole 16 B units
@@ -96,8 +97,10 @@ static __device__ __noinline__ void dtab_clear_words(unsigned* t, int64_t n) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n4; i += stride)
     w[i] = make_uint4(~0u, ~0u, ~0u, ~0u);
 }
+// Called by every thread of the FIRST kernel of an append-unique (the fused hop's sampler, or the
+// standalone insert pass): at the first epoch of a cycle, clear the other (idle) table (grid-strided).
 __device__ __forceinline__ void dtab_clear_ahead(const DirectTable& d, unsigned epoch) {
-  if (compact_epoch(epoch + 1u) <= 2u) dtab_clear_words(d.t[(epoch + 1u) & 1u], d.n);
+  if (compact_epoch(epoch) == 1u) dtab_clear_words(((epoch / CEPOCHS) & 1u) ? d.t[0] : d.t[1], d.n);
 }
 
 __device__ __forceinline__ unsigned long long stored_key(unsigned epoch, int64_t key) {

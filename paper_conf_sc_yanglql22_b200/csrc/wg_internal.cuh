@@ -82,7 +82,8 @@ struct Workspace {
   int64_t hcap = 0;                      // slots (a multiple of 8, < 2^31); each call uses a prefix
   int compact = 0;                       // 8 B slots {epoch8, key28, pos28} (hash.cuh), else 16 B slots
   // direct table (hash.cuh, graphs small enough that a word per NODE beats a hashed slot per key): two
-  // uint32 arrays of num_nodes words {255 - compact_epoch, first position}, epoch e uses dtab[e & 1];
+  // uint32 arrays of num_nodes words {255 - compact_epoch, first position}; the epochs of 255-epoch cycle c
+  // use dtab[c & 1] (hash.cuh);
   // the fused hop's sampler inserts into it, so a hop has no insert pass and no slot_of round trip
   int direct = 0;
   unsigned* dtab[2] = {nullptr, nullptr};

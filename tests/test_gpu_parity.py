@@ -562,8 +562,10 @@ def test_compact_table_epoch_cycles(tiny, fmt):
     assert d2.unique_format() == want
     d2.debug_set_epoch(250)
     for i in range(300):
-        if i == 150 and fmt == "direct":   # fused hops and standalone calls share the epoch sequence
+        if i == 150:   # the next cycle restart (direct: back to the first table)
             d2.debug_set_epoch(508)
+        if i == 200:   # the counter's wrap (modulo 2 x 255 epochs: cycle parity and tags continue)
+            d2.debug_set_epoch(2 * 255 * 2048 - 3)
         T = rng.choice(2000, 40, replace=False).astype(np.int64)
         nb = rng.integers(0, 2000, 600).astype(np.int64)
         U, sc, dup = gpu_unique(d2, T, nb)
