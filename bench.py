@@ -342,7 +342,7 @@ def measure_ceilings(dsm, reps=3):
 
 def hop_kernels(m, direct=False):
     """Kernel stages of one wg_sample_hop (the stage events the library records); with the direct key
-    table the sampler inserts every key and there is no insert pass."""
+    table (direct=True) the sampler inserts every key and there is no insert pass."""
     return ("sample", "flag", "relabel") if direct else ("sample", "insert", "flag", "relabel")
 
 
@@ -357,8 +357,7 @@ def stage_breakdown(pipe, seeds_dev, rngs, flush, ceil=None, nb=20):
     import torch
     st = torch.cuda.current_stream()
     H = len(pipe.fanouts)
-    from paper_conf_sc_yanglql22_b200 import WG_UNIQUE_DIRECT
-    direct = pipe.dsm.unique_format() == WG_UNIQUE_DIRECT
+    direct = not pipe.dsm.hop_insert_pass()   # the sampler inserts: no insert kernel
 
     def hop_kernels_(m):
         return hop_kernels(m, direct)
@@ -417,7 +416,7 @@ def stage_breakdown(pipe, seeds_dev, rngs, flush, ceil=None, nb=20):
         worst = min(((h, k, v) for h, d in fr.items() for k, v in d.items() if k in kinds), key=lambda x: x[2])
         fr["furthest_below"] = {"hop": worst[0], "kernel": worst[1], "frac": worst[2]}
     out["frac"] = fr
-    out["unique_format"] = "direct" if direct else "hashed"
+    out["unique_format"] = ["wide", "compact", "direct"][pipe.dsm.unique_format()]
     out["note"] = ("median ms per kernel of one batch (eager launches, an event after every kernel, L2 flushed per "
                    "batch; hop h = wg_sample_hop); frac = each kernel's operation rate over its measured ceiling "
                    "(ceilings)")

@@ -87,8 +87,10 @@ typedef enum { WG_F32 = 0, WG_F16 = 1, WG_BF16 = 2 } wg_dtype;
  * wg_dsm_unique_format).  DIRECT (num_nodes <= 2^24, max_batch_keys < 2^24, no WG_DSM_HASHED /
  * WG_DSM_WIDE_HASH): the "table" is indexed by the node id itself -- one 32-bit word per node holding
  * the key's first position, two such arrays per workspace (2 x 4 B x num_nodes); the fused hop's
- * sampler inserts every key (no insert pass).  COMPACT: 8 B hashed slots (ids and positions < 2^28).
- * WIDE: 16 B hashed slots.  Results never depend on the format. */
+ * sampler inserts every key (no insert pass).  COMPACT: 8 B hashed slots (ids and positions < 2^28),
+ * two tables alternating per 255-epoch cycle.  WIDE: 16 B hashed slots.  Both hashed formats run a
+ * separate insert pass.
+ * Results never depend on the format. */
 #define WG_UNIQUE_WIDE    0
 #define WG_UNIQUE_COMPACT 1
 #define WG_UNIQUE_DIRECT  2
@@ -224,8 +226,8 @@ wg_status wg_append_unique(wg_dsm_t h, const int64_t* d_targets, int64_t n_targe
  * pass of Append Unique reads them directly, and ONE single-pass scan both
  * compacts the sampler output into the CSR (row_ptr, neighbours, positions) and
  * numbers the first occurrences -- four kernels, no host sync (three with the
- * direct key table, wg_dsm_unique_format: the sampler inserts every key itself, a
- * RED.MIN of its position into the node's word, and there is no insert pass).  The relabel
+ * direct key table, wg_dsm_unique_format: the sampler inserts every key itself and
+ * there is no insert pass).  The relabel
  * (which fills d_out_sub_col / d_out_dup_count) is launched on side_stream when
  * it is non-NULL (forked from `stream` with an event); the caller must make its
  * consumers wait for side_stream, and must join it before issuing a fifth
@@ -338,13 +340,15 @@ wg_status wg_device_error(wg_dsm_t h, uint32_t* code, int32_t clear);
  * 8 B format cycles through 255 epochs and clears itself when a cycle restarts. */
 wg_status wg_dsm_reset_workspace(wg_dsm_t h, wg_stream_t stream);
 
-/* The Append Unique key-table format of h's workspace: WG_UNIQUE_WIDE / _COMPACT / _DIRECT.
- * Errors: WG_ERR_INVALID_ARG for NULL arguments. */
-wg_status wg_dsm_unique_format(wg_dsm_t h, int32_t* format);
+/* The Append Unique key-table format of h's workspace: WG_UNIQUE_WIDE / _COMPACT / _DIRECT; and
+ * (hop_insert_pass, nullable) 1 if wg_sample_hop runs a separate insert pass (the hashed formats), 0 if
+ * its sampler inserts the keys (the direct format).  Errors: WG_ERR_INVALID_ARG if h or format is
+ * NULL. */
+wg_status wg_dsm_unique_format(wg_dsm_t h, int32_t* format, int32_t* hop_insert_pass);
 
 /* Diagnostics (per-kernel device times): while set, wg_sample_hop records events[0..n)
  * in order after its kernels -- sampler, insert, flag scan, relabel (the relabel's on the side stream
- * when one is given; with the direct format there is no insert pass: sampler, flag scan, relabel) --
+ * when one is given; without an insert pass (wg_dsm_unique_format): sampler, flag scan, relabel) --
  * and wg_append_unique after insert, flag scan, relabel.  events are cudaEvent_t
  * handles owned by the caller; n = 0 clears.  Use with eager launches (not inside a graph capture).
  * Errors: WG_ERR_INVALID_ARG if n is outside [0, 8] or events is NULL with n > 0. */

@@ -75,7 +75,7 @@ def lib():
     L.wg_dsm_set_gather_occupancy.argtypes = [P, I32]
     L.wg_dsm_debug_set_epoch.argtypes = [P, ctypes.c_uint32]
     L.wg_dsm_set_stage_events.argtypes = [P, P, I32]
-    L.wg_dsm_unique_format.argtypes = [P, P]
+    L.wg_dsm_unique_format.argtypes = [P, P, P]
     L.wg_micro_random_read.argtypes = [P, I64, I32, I32, I32, P, P, P]
     L.wg_micro_atomics.argtypes = [P, I64, I32, I32, I32, P, P, P]
     for f in ("wg_dsm_create", "wg_dsm_fork", "wg_dsm_local_view", "wg_dsm_shard_info", "wg_dsm_feat_layout",

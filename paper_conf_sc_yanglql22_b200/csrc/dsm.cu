@@ -88,6 +88,7 @@ static wg_status barrier(wg_dsm* h) {
 static void free_workspace(wg_dsm* h) {
   Workspace& w = h->ws;
   cudaFree(w.hslots);
+  cudaFree(w.hslots2);
   cudaFree(w.dtab[0]);
   cudaFree(w.dtab[1]);
   cudaFree(w.status_sample);
@@ -145,7 +146,14 @@ static wg_status alloc_workspace(wg_dsm* h, int64_t max_keys) {
   }
   w.pad32 = !(h->flags & WG_DSM_PAD64) && h->n < (int64_t(1) << 32) ? 1 : 0;
   if (w.compact) {
-    WG_CUDA_TRY(cudaMemset(w.hslots, 0, cap * sizeof(HashSlot)));  // every word stale (epoch 0)
+    // two tables of 8 B words, alternating per 255-epoch cycle (hash.cuh); every word stale (epoch 0)
+    if (cudaMalloc(&w.hslots2, cap * 8) != cudaSuccess) {
+      cudaGetLastError();
+      free_workspace(h);
+      return fail(WG_ERR_OOM, "workspace allocation failed (hash table)");
+    }
+    WG_CUDA_TRY(cudaMemset(w.hslots, 0, cap * sizeof(HashSlot)));
+    WG_CUDA_TRY(cudaMemset(w.hslots2, 0, cap * 8));
   } else {
     WG_CUDA_TRY(cudaMemset(w.hslots, 0xff, cap * sizeof(HashSlot)));                   // val = all ones
     WG_CUDA_TRY(cudaMemset2D(w.hslots, sizeof(HashSlot), 0, sizeof(unsigned long long), cap));  // key = 0 (empty)
@@ -560,6 +568,7 @@ wg_status wg_dsm_reset_workspace(wg_dsm_t h, wg_stream_t stream) {
   }
   if (h->ws.compact) {
     WG_CUDA_TRY(cudaMemsetAsync(h->ws.hslots, 0, h->ws.hcap * sizeof(HashSlot), st));
+    WG_CUDA_TRY(cudaMemsetAsync(h->ws.hslots2, 0, h->ws.hcap * 8, st));
   } else {
     WG_CUDA_TRY(cudaMemsetAsync(h->ws.hslots, 0xff, h->ws.hcap * sizeof(HashSlot), st));
     WG_CUDA_TRY(cudaMemset2DAsync(h->ws.hslots, sizeof(HashSlot), 0, sizeof(unsigned long long), h->ws.hcap, st));
@@ -586,12 +595,17 @@ wg_status wg_dsm_debug_set_epoch(wg_dsm_t h, uint32_t epoch) {
   // clean, hash.cuh)
   if (h->ws.direct)
     for (int t = 0; t < 2; ++t) WG_CUDA_TRY(cudaMemset(h->ws.dtab[t], 0xff, (size_t)((h->n + 3) / 4) * 16));
+  if (h->ws.compact) {  // likewise the compact tables (the next cycle's table must be clean)
+    WG_CUDA_TRY(cudaMemset(h->ws.hslots, 0, h->ws.hcap * 8));
+    WG_CUDA_TRY(cudaMemset(h->ws.hslots2, 0, h->ws.hcap * 8));
+  }
   return WG_OK;
 }
 
-wg_status wg_dsm_unique_format(wg_dsm_t h, int32_t* format) {
+wg_status wg_dsm_unique_format(wg_dsm_t h, int32_t* format, int32_t* hop_insert_pass) {
   if (!h || !format) return fail(WG_ERR_INVALID_ARG, "null argument");
   *format = h->ws.direct ? WG_UNIQUE_DIRECT : h->ws.compact ? WG_UNIQUE_COMPACT : WG_UNIQUE_WIDE;
+  if (hop_insert_pass) *hop_insert_pass = wg::hop_inserts_in_sampler(h) ? 0 : 1;
   return WG_OK;
 }
 

@@ -20,28 +20,56 @@ struct HashTable {
   HashSlot* slots;
   unsigned long long size;  // slots in use (any size: slot = high half of hash * size)
   int compact;              // 8 B slots (below) instead of 16 B HashSlots
+  HashSlot* slots2;         // compact: the table of odd 255-epoch cycles (slots serves the even ones)
 };
+// The table an op at this epoch uses: the compact format alternates between two tables per 255-epoch
+// cycle like the direct one (below); the wide format has one table and 2^23 epochs.
+__device__ __forceinline__ HashTable ht_for_epoch(HashTable t, unsigned epoch) {
+  if (t.compact && ((epoch / CEPOCHS) & 1u)) t.slots = t.slots2;
+  return t;
+}
+// Compact format, called by every thread of the FIRST kernel of an append-unique: at the first epoch of
+// a cycle, zero the other (idle) table's `words` words (grid-strided) -- it served the previous cycle,
+// whose ops have all finished, and serves the next one.
+static __device__ __noinline__ void chash_clear_words(unsigned long long* w, int64_t words) {
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < words; i += stride) w[i] = 0ull;
+}
+__device__ __forceinline__ void chash_clear_ahead(const HashTable& t, int64_t words, unsigned epoch) {
+  if (t.compact && compact_epoch(epoch) == 1u)
+    chash_clear_words(reinterpret_cast<unsigned long long*>(((epoch / CEPOCHS) & 1u) ? t.slots : t.slots2), words);
+}
 
 // ---- compact table: one 64-bit word per slot, [63:56] epoch (1..255), [55:28] node id, [27:0]
 // first position (nodes and positions < 2^28).  Claimed with one 64-bit CAS of the whole word;
 // later occurrences of the key lower it with a 64-bit atomicMin (epoch and id bits are equal,
 // so the minimum is taken over the position).  Stale words (another epoch, or 0 after a clear)
-// read as empty; the table is cleared when the 255-epoch cycle restarts (sample_kernel /
-// hash_clear_kernel), so it never needs a per-call memset.
+// read as empty; two tables alternate per 255-epoch cycle and the idle one is zeroed at a cycle's
+// first op (chash_clear_ahead), so neither needs a per-call memset.
 constexpr unsigned long long CPOS_MASK = (1ull << 28) - 1;
 __device__ __forceinline__ unsigned long long cword(unsigned ce, int64_t key, int64_t q) {
   return ((unsigned long long)ce << 56) | ((unsigned long long)key << 28) | (unsigned long long)q;
 }
-// Returns the slot of `key` (claimed with position q if new), or -1 if full; *old = the word seen
-// (0 if this call claimed the slot).  Applies the atomicMin (with return if want_old).
-__device__ __forceinline__ long long chash_insert(const HashTable& t, int64_t key, int64_t q, unsigned ce,
-                                                  bool want_old, unsigned long long* old) {
+// Home slot of `key` in a table of t.size slots.
+__device__ __forceinline__ unsigned long long chash_home(const HashTable& t, int64_t key) {
+  return __umul64hi(fmix64((unsigned long long)key), t.size);
+}
+__device__ __forceinline__ unsigned long long chash_load(const HashTable& t, unsigned long long slot) {
+  unsigned long long cur;
+  asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(cur) : "l"(&reinterpret_cast<unsigned long long*>(t.slots)[slot]));
+  return cur;
+}
+// Insert continuing from slot `slot` whose word was read as `cur` (chash_home / chash_load: callers with
+// several keys issue all their first loads before resolving any).  Returns the slot of `key` (claimed
+// with position q if new), or -1 if full; *old = the word seen (0 if this call claimed the slot).
+// Applies the atomicMin (with return if want_old; else only when the word holds a larger position).
+__device__ __forceinline__ long long chash_insert_from(const HashTable& t, int64_t key, int64_t q, unsigned ce,
+                                                       bool want_old, unsigned long long* old, unsigned long long slot,
+                                                       unsigned long long cur) {
   unsigned long long* w = reinterpret_cast<unsigned long long*>(t.slots);
   const unsigned long long mine = cword(ce, key, q);
-  unsigned long long slot = __umul64hi(fmix64((unsigned long long)key), t.size);
   for (unsigned long long probe = 0; probe < t.size; ++probe) {
-    unsigned long long cur;
-    asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(cur) : "l"(&w[slot]));
+    if (probe) cur = chash_load(t, slot);
     for (;;) {
       if ((cur >> 28) == (mine >> 28)) {  // our key, this epoch
         if (want_old) {
@@ -63,6 +91,11 @@ __device__ __forceinline__ long long chash_insert(const HashTable& t, int64_t ke
     slot = slot + 1 == t.size ? 0 : slot + 1;
   }
   return -1;
+}
+__device__ __forceinline__ long long chash_insert(const HashTable& t, int64_t key, int64_t q, unsigned ce,
+                                                  bool want_old, unsigned long long* old) {
+  const unsigned long long slot = chash_home(t, key);
+  return chash_insert_from(t, key, q, ce, want_old, old, slot, chash_load(t, slot));
 }
 __device__ __forceinline__ int64_t chash_min_pos(const HashTable& t, long long slot) {
   return (int64_t)(reinterpret_cast<const unsigned long long*>(t.slots)[slot] & CPOS_MASK);

@@ -52,9 +52,9 @@ struct SampleArgs {
   int32_t* pos_pad;   // [nT * M]
   int32_t* cnt;       // [nT]
   unsigned* ctrl;
-  unsigned long long* hclear;  // fused hop, compact hash table: zeroed here when its epoch cycle restarts
+  HashTable ht;                // fused hop, compact hash table (prefix size of this hop's key bound)
+  int64_t hwords;              // its full capacity (the idle table is zeroed at a cycle's first op)
   int pad32;                   // padded neighbour slots hold uint32 ids (num_nodes < 2^32)
-  int64_t hwords;
   // MODE_DIRECT (fused hop with the direct table): the Append Unique insert happens here -- targets
   // first (U[k] = T[k], their own position k, duplicate-target check), every sampled id a RED.MIN of
   // its padded position nT + k*M + i (same order as the dense positions); padding slots get PAD_ID
@@ -62,8 +62,9 @@ struct SampleArgs {
   int64_t* U;
   int32_t* dup;
 };
-// sampler modes: plain, plain + compact-table clear (fused hop, compact hash), fused hop with the
-// direct table (inserts here; the hop then has no insert pass)
+// sampler modes: plain; plain + the compact table's clear-ahead (fused hop with the compact hash: the
+// insert pass follows); fused hop with the direct table, inserting here (the hop then has no insert pass).
+// (Inserting into the compact hash table here measured slower: profiles/r02/ab_log.md.)
 enum { MODE_PLAIN = 0, MODE_CLEAR = 1, MODE_DIRECT = 2 };
 
 // Padded slot without a sample (direct mode: the flag pass reads no per-target count)
@@ -84,48 +85,49 @@ __device__ __forceinline__ unsigned direct_insert_target(const SampleArgs& a, un
 __device__ __forceinline__ void direct_target_check(const SampleArgs& a, unsigned tag, int64_t nT, unsigned old) {
   if ((old >> DPOS_BITS) == tag && (int64_t)(old & DPOS_MASK) < nT) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DUP_TARGET);
 }
-// Sampled id nb at padded position q: fire-and-forget atomicMin (compiles to RED.E.MIN).  lead = false:
-// a lower lane of the warp round holds the same id at a smaller position (no atomic needed).
-#ifndef WG_DIRECT_FILTER
-#define WG_DIRECT_FILTER 1  // read the word first and skip the RED when it already holds a smaller position
-#endif
-#ifndef WG_DIRECT_DEDUP
-#define WG_DIRECT_DEDUP 0  // warp-round __match_any_sync before the REDs (A/B: no gain)
-#endif
+// Sampled id nb at padded position q: RED.MIN of its word, issued only when a plain load of the word shows
+// a larger position (the filter: hubs meet their own target's or an earlier sample's smaller position and
+// issue no atomic; unfiltered REDs serialise on hub words, profiles/r02/ab_log.md).  Batched over a lane's
+// UNR rounds: every round's load is issued before any is resolved.
+template <int UNR>
+__device__ __forceinline__ void direct_insert_nbrs(const SampleArgs& a, unsigned* t, unsigned tag, int64_t nT, int M,
+                                                   int i, const int64_t* nb, const int64_t* kk, const bool* ok) {
+  unsigned cur[UNR];
+  bool in[UNR];
+#pragma unroll
+  for (int u = 0; u < UNR; ++u) {
+    in[u] = ok[u] && nb[u] >= 0 && nb[u] < a.s.n;
+    if (ok[u] && !in[u]) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_ID_RANGE);
+    cur[u] = 0u;
+    if (in[u]) asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(cur[u]) : "l"(&t[nb[u]]));
+  }
+#pragma unroll
+  for (int u = 0; u < UNR; ++u) {
+    const unsigned mine = dword(tag, nT + kk[u] * M + i);
+    if (in[u] && cur[u] > mine) atomicMin(&t[nb[u]], mine);
+  }
+}
+// Single-key form (block sampler).
 __device__ __forceinline__ void direct_insert_nbr(const SampleArgs& a, unsigned* t, unsigned tag, int64_t q,
-                                                  int64_t nb, bool lead = true) {
+                                                  int64_t nb) {
   if (nb < 0 || nb >= a.s.n) {
     latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_ID_RANGE);
     return;
   }
-  if (!lead) return;
   const unsigned mine = dword(tag, q);
-  if (WG_DIRECT_FILTER) {
-    unsigned cur;
-    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(cur) : "l"(&t[nb]));
-    if (cur <= mine) return;
-  }
-  atomicMin(&t[nb], mine);
-}
-
-// The insert pass that follows this sampler (same hop) needs a zeroed compact table when the epoch
-// cycle restarts (hash.cuh); every block clears a grid-strided share before sampling.
-__device__ __noinline__ void clear_table_if_cycle_restarts(unsigned long long* w, int64_t words, const unsigned* ctrl) {
-  if (compact_epoch(ctrl[CTRL_EPOCH]) != 1u) return;
-  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
-  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < words; i += stride) w[i] = 0ull;
+  unsigned cur;
+  asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(cur) : "l"(&t[nb]));
+  if (cur > mine) atomicMin(&t[nb], mine);
 }
 
 template <int SAMPLE_UNR, int MODE, bool COL32>
 __global__ void __launch_bounds__(SAMPLE_THREADS, SAMPLE_MINB) sample_kernel(const SampleArgs a) {
   pdl_enter();
   KT_BEGIN(0);
-  if (MODE == MODE_CLEAR) clear_table_if_cycle_restarts(a.hclear, a.hwords, a.ctrl);
   unsigned epoch = 0;
-  if (MODE == MODE_DIRECT) {
-    epoch = a.ctrl[CTRL_EPOCH];
-    dtab_clear_ahead(a.dt, epoch);
-  }
+  if (MODE != MODE_PLAIN) epoch = a.ctrl[CTRL_EPOCH];
+  if (MODE == MODE_CLEAR) chash_clear_ahead(a.ht, a.hwords, epoch);
+  if (MODE == MODE_DIRECT) dtab_clear_ahead(a.dt, epoch);
   __shared__ unsigned sm_chain[SAMPLE_THREADS / 32][32];
   const int tid = threadIdx.x, warp = tid >> 5;
   int64_t nT = a.cap;
@@ -144,24 +146,27 @@ __global__ void __launch_bounds__(SAMPLE_THREADS, SAMPLE_MINB) sample_kernel(con
   // padded slots k*M + i of the workspace (the scan pass that follows compacts them)
   unsigned* const dt = MODE == MODE_DIRECT ? dtab_cur(a.dt, epoch) : nullptr;
   const unsigned tag = MODE == MODE_DIRECT ? dtag(epoch) : 0u;
-  sample_warp<SAMPLE_UNR, COL32, MODE == MODE_DIRECT && WG_DIRECT_DEDUP>(
+  sample_warp<SAMPLE_UNR, COL32>(
       a.s, a.targets, nT, M, a.hop, key, warp_base, sm_chain[warp], &a.ctrl[CTRL_ERR],
       [&](int64_t k, int64_t v) -> unsigned {
         return MODE == MODE_DIRECT ? direct_insert_target(a, dt, tag, k, v) : 0u;
       },
-      [&](int64_t k, unsigned old) {
-        if (MODE == MODE_DIRECT) direct_target_check(a, tag, nT, old);
+      [&](int64_t k, unsigned tok) {
+        if (MODE == MODE_DIRECT) direct_target_check(a, tag, nT, tok);
       },
       [&](int64_t k, int c) {
         if (MODE != MODE_DIRECT) a.cnt[k] = c;
       },
-      [&](int64_t k, int i, int64_t nb, unsigned pos, bool lead) {
+      [&](int64_t k, int i, int64_t nb, unsigned pos) {
         st_pad(a.nbrs_pad, a.pad32, k * M + i, nb);
         if (a.pos_pad) a.pos_pad[k * M + i] = (int32_t)pos;
-        if (MODE == MODE_DIRECT) direct_insert_nbr(a, dt, tag, nT + k * M + i, nb, lead);
       },
       [&](int64_t k, int i) {
         if (MODE == MODE_DIRECT) st_pad(a.nbrs_pad, a.pad32, k * M + i, pad_id(a.pad32));
+      },
+      [&](const int64_t* nb, const int64_t* kk, const bool* ok) {
+        const int i = (threadIdx.x & 31) - ((threadIdx.x & 31) / sample_group(M)) * sample_group(M);
+        if (MODE == MODE_DIRECT) direct_insert_nbrs<SAMPLE_UNR>(a, dt, tag, nT, M, i, nb, kk, ok);
       });
   KT_END(0, "sample", nT);
 }
@@ -175,12 +180,10 @@ __global__ void __launch_bounds__(SAMPLE_THREADS, SAMPLE_MINB) sample_kernel(con
 template <int BT, int MODE, bool COL32>
 __global__ void __launch_bounds__(BT) sample_block_kernel(const SampleArgs a) {
   pdl_enter();
-  if (MODE == MODE_CLEAR) clear_table_if_cycle_restarts(a.hclear, a.hwords, a.ctrl);
   unsigned epoch = 0;
-  if (MODE == MODE_DIRECT) {
-    epoch = a.ctrl[CTRL_EPOCH];
-    dtab_clear_ahead(a.dt, epoch);
-  }
+  if (MODE != MODE_PLAIN) epoch = a.ctrl[CTRL_EPOCH];
+  if (MODE == MODE_CLEAR) chash_clear_ahead(a.ht, a.hwords, epoch);
+  if (MODE == MODE_DIRECT) dtab_clear_ahead(a.dt, epoch);
   unsigned* const dt = MODE == MODE_DIRECT ? dtab_cur(a.dt, epoch) : nullptr;
   const unsigned tag = MODE == MODE_DIRECT ? dtag(epoch) : 0u;
   __shared__ unsigned long long s_key[BT];
@@ -412,13 +415,15 @@ cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap,
   a.pos_pad = want_pos ? h->ws.pos_pad : nullptr;
   a.cnt = h->ws.cnt;
   a.ctrl = h->ws.ctrl;
-  a.hclear = h->ws.compact ? reinterpret_cast<unsigned long long*>(h->ws.hslots) : nullptr;
+  a.ht = HashTable{h->ws.hslots, (unsigned long long)table_prefix(h, cap + cap * fanout), h->ws.compact,
+                   reinterpret_cast<HashSlot*>(h->ws.hslots2)};
   a.hwords = h->ws.hcap;
   a.dt = DirectTable{{h->ws.dtab[0], h->ws.dtab[1]}, h->n};
   a.U = U;
   a.dup = dup;
-  // U != NULL: the fused hop (wg_sample_hop); with the direct table its inserts happen here
-  const int mode = (U && h->ws.direct) ? MODE_DIRECT : (a.hclear ? MODE_CLEAR : MODE_PLAIN);
+  // U != NULL: the fused hop (wg_sample_hop); with the direct key table its inserts happen here
+  // (launch_hop skips the insert pass, hop_inserts_in_sampler)
+  const int mode = !U ? MODE_PLAIN : h->ws.direct ? MODE_DIRECT : h->ws.compact ? MODE_CLEAR : MODE_PLAIN;
   const bool block = fanout > 32;  // block per target (Algorithm 1 with a block sort)
   int unr = 1;
   unsigned blocks = (unsigned)(cap > 0 ? cap : 1);
@@ -435,6 +440,9 @@ cudaError_t launch_sample_padded(wg_dsm* h, const int64_t* targets, int64_t cap,
   if (mode == MODE_CLEAR) return launch_sampler_mode<MODE_CLEAR>(block, c32, fanout, unr, blocks, a, st);
   return launch_sampler_mode<MODE_PLAIN>(block, c32, fanout, unr, blocks, a, st);
 }
+
+// Whether the fused hop's sampler inserts the keys itself (no insert pass), for launch_hop.
+bool hop_inserts_in_sampler(const wg_dsm* h) { return h->ws.direct != 0; }
 
 cudaError_t launch_sample(wg_dsm* h, const int64_t* targets, int64_t cap, const int64_t* d_n, int fanout,
                           uint64_t seed, const uint64_t* d_seed, int hop, int64_t* out_row_ptr,

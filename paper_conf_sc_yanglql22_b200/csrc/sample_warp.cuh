@@ -23,19 +23,19 @@ __host__ __device__ inline int sample_group(int M) { return M > SAMPLE_UNR_MAX ?
 
 // One warp samples the targets k = warp_base + u * TPW + g (u < UNR, g < TPW, k < nT) of targets[].
 // on_target(k, v) is called once per target k < nT with its id as loaded (before the range check),
-// right after the load; it returns a token handed to on_target_end(k, token) after every other callback
+// right after its row_ptr loads are issued; it returns a token handed to on_target_end(k, token) after every other callback
 // of the warp (the direct table issues the target's atomic early and checks its result late); emit_cnt(k, c) once per target k < nT (c = min(M, deg), 0
-// for an invalid id); emit(k, i, nb, pos, lead) for every sampled slot i < c (draw order, A5), lead =
-// no lower lane of this warp round sampled the same id (DEDUP; always true without); emit_pad(k, i)
-// for the slots c <= i < M.
+// for an invalid id); emit(k, i, nb, pos) for every sampled slot i < c (draw order, A5); emit_pad(k, i)
+// for the slots c <= i < M; then insert_all(nb, kk, ok) once with this lane's UNR rounds (sampled id,
+// target, valid), so a key-table insert can issue all its first loads before resolving any.
 // chain: this warp's 32 words of shared memory.
 // All 32 lanes must call it (warp-collective); warps past nT return at once.
-template <int UNR, bool COL32, bool DEDUP, typename OnTarget, typename OnTargetEnd, typename EmitCnt, typename Emit,
-          typename EmitPad>
+template <int UNR, bool COL32, typename OnTarget, typename OnTargetEnd, typename EmitCnt, typename Emit,
+          typename EmitPad, typename InsertAll>
 __device__ __forceinline__ void sample_warp(const ShardView& s, const int64_t* targets, int64_t nT, int M, int hop,
                                             uint2 key, int64_t warp_base, unsigned* chain, unsigned* ctrl_err,
                                             OnTarget on_target, OnTargetEnd on_target_end, EmitCnt emit_cnt, Emit emit,
-                                            EmitPad emit_pad) {
+                                            EmitPad emit_pad, InsertAll insert_all) {
   if (warp_base >= nT) return;  // warp-uniform
   const int lane = threadIdx.x & 31;
   const int G = sample_group(M);
@@ -50,7 +50,8 @@ __device__ __forceinline__ void sample_warp(const ShardView& s, const int64_t* t
     const int64_t k = warp_base + (int64_t)i * TPW + g;
     if (k < nT) {
       my_v = targets[k];
-      my_tok = on_target(k, my_v);
+      const int64_t raw = my_v;
+      int64_t r1 = 0;
       if (my_v < 0 || my_v >= s.n) {
         latch_error(ctrl_err, WG_DEVERR_ID_RANGE);
         my_v = -1;
@@ -60,7 +61,11 @@ __device__ __forceinline__ void sample_warp(const ShardView& s, const int64_t* t
         csr_owner_local(s, my_v, o, l);
         const int64_t* rp = s.row_ptr[o] + l;
         my_start = rp[0];
-        const int64_t d = rp[1] - my_start;
+        r1 = rp[1];
+      }
+      my_tok = on_target(k, raw);  // after the row_ptr loads are issued: their latency hides its work
+      if (my_v >= 0) {
+        const int64_t d = r1 - my_start;
         if (d >= (int64_t(1) << 32) || d < 0)
           latch_error(ctrl_err, WG_DEVERR_DEGREE);
         else
@@ -124,15 +129,10 @@ __device__ __forceinline__ void sample_warp(const ShardView& s, const int64_t* t
   for (int u = 0; u < UNR; ++u) nb[u] = ok[u] ? ld_col<COL32>(s, osrc[u], src[u]) : -1;
 #pragma unroll
   for (int u = 0; u < UNR; ++u) {
-    bool lead = true;
-    if (DEDUP) {  // lanes are in position order within a round: the lowest lane holds the first position
-      const unsigned same =
-          __match_any_sync(FULL_MASK, ok[u] ? (unsigned long long)nb[u] : (0x8000000000000000ull | (unsigned)lane));
-      lead = (same & ((1u << lane) - 1u)) == 0u;
-    }
-    if (ok[u]) emit(kk[u], i, nb[u], pos[u], lead);
+    if (ok[u]) emit(kk[u], i, nb[u], pos[u]);
     else if (pad[u]) emit_pad(kk[u], i);
   }
+  insert_all(nb, kk, ok);
   if (i < UNR && g < TPW) {
     const int64_t k = warp_base + (int64_t)i * TPW + g;
     if (k < nT) on_target_end(k, my_tok);

@@ -105,7 +105,8 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueA
   load_counts<PADDED>(a, nT, nE);
   const unsigned epoch = a.ctrl[CTRL_EPOCH];
   constexpr bool COMPACT = FMT == FMT_COMPACT;
-  if (FMT == FMT_DIRECT) dtab_clear_ahead(a.dt, epoch);  // table e+1 is idle (standalone first kernel)
+  if (FMT == FMT_DIRECT) dtab_clear_ahead(a.dt, epoch);  // the idle table (standalone: the op's first kernel)
+  const HashTable ht = ht_for_epoch(a.ht, epoch);
   unsigned* const dt = FMT == FMT_DIRECT ? dtab_cur(a.dt, epoch) : nullptr;
   const unsigned tag = FMT == FMT_DIRECT ? dtag(epoch) : 0u;
   const int64_t total = nT + nE;
@@ -162,16 +163,16 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueA
     if (valid && leader == lane) {
       if (COMPACT) {
         unsigned long long old;
-        slot = chash_insert(a.ht, key, q, compact_epoch(epoch), is_target, &old);
+        slot = chash_insert(ht, key, q, compact_epoch(epoch), is_target, &old);
         // a target meeting an earlier TARGET record of its key: duplicate target (A8)
         if (is_target && slot >= 0 && old != 0 && (int64_t)(old & CPOS_MASK) < nT)
           latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DUP_TARGET);
       } else if (is_target) {
         bool dup = false;
-        slot = hash_insert_target(a.ht, key, q, nT, epoch, &dup);
+        slot = hash_insert_target(ht, key, q, nT, epoch, &dup);
         if (dup) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_DUP_TARGET);
       } else {
-        slot = hash_insert_min(a.ht, key, q, epoch);
+        slot = hash_insert_min(ht, key, q, epoch);
       }
       if (slot < 0) latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_CAPACITY);
     }
@@ -181,10 +182,10 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_insert_kernel(const UniqueA
 }
 
 template <int FMT>
-__device__ __forceinline__ int64_t min_pos_at(const UniqueArgs& a, int32_t slot) {
+__device__ __forceinline__ int64_t min_pos_at(const HashTable& ht, int32_t slot) {
   if (slot < 0) return -1;
-  if (FMT == FMT_COMPACT) return chash_min_pos(a.ht, slot);
-  return (int64_t)(a.ht.slots[slot].val & KEY_MASK);
+  if (FMT == FMT_COMPACT) return chash_min_pos(ht, slot);
+  return (int64_t)(ht.slots[slot].val & KEY_MASK);
 }
 
 template <bool PADDED, int UQ_ITEMS, int FMT>
@@ -205,6 +206,7 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArg
 
   const unsigned* const dt = FMT == FMT_DIRECT ? dtab_cur(a.dt, epoch) : nullptr;
   const unsigned tag = FMT == FMT_DIRECT ? dtag(epoch) : 0u;
+  const HashTable ht = ht_for_epoch(a.ht, epoch);
   const int64_t pad_key = a.pad32 ? (int64_t)0xFFFFFFFFu : (int64_t)-1;  // direct: sampler's padding slots
   const int64_t tile_start = (int64_t)blockIdx.x * UQ_TILE;
   if (nE == 0) {
@@ -240,7 +242,7 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_flag_kernel(const UniqueArg
         mps[t] = (valid && keys[t] >= 0 && keys[t] < a.n) ? dtab_min_pos(dt, tag, keys[t]) : -1;
       } else {
         valid = j < nE && (!PADDED || slots[t] != SLOT_EMPTY);
-        mps[t] = min_pos_at<FMT>(a, slots[t]);  // independent L2 reads
+        mps[t] = min_pos_at<FMT>(ht, slots[t]);  // independent L2 reads
       }
       poss[t] = (PADDED && a.out_pos && valid) ? a.pos_pad[j] : 0;
       vm[t] = __ballot_sync(FULL_MASK, valid);
@@ -330,24 +332,24 @@ __global__ void __launch_bounds__(UQ_THREADS) unique_relabel_kernel(const Unique
   }
 }
 
-// Compact table: zero it when the epoch cycle restarts (compact_epoch == 1).  Launched before the
+// Compact tables: at the first epoch of a cycle zero the idle one (chash_clear_ahead).  Launched before the
 // insert pass of a standalone append-unique; the fused hop does the same inside its sampler.
-__global__ void __launch_bounds__(256) hash_clear_kernel(unsigned long long* w, int64_t words, const unsigned* ctrl) {
+__global__ void __launch_bounds__(256) hash_clear_kernel(const HashTable t, int64_t words, const unsigned* ctrl) {
   pdl_enter();
-  if (compact_epoch(ctrl[CTRL_EPOCH]) != 1u) return;
-  for (int64_t i = (int64_t)blockIdx.x * 256 + threadIdx.x; i < words; i += (int64_t)gridDim.x * 256) w[i] = 0ull;
+  chash_clear_ahead(t, words, ctrl[CTRL_EPOCH]);
 }
 
 cudaError_t launch_hash_clear(wg_dsm* h, cudaStream_t st) {
-  return launch_pdl(hash_clear_kernel, (unsigned)h->sm_count * 4, 256, 0, st,
-                    reinterpret_cast<unsigned long long*>(h->ws.hslots), (int64_t)h->ws.hcap, (const unsigned*)h->ws.ctrl);
+  const HashTable t{h->ws.hslots, 0ull, h->ws.compact, reinterpret_cast<HashSlot*>(h->ws.hslots2)};
+  return launch_pdl(hash_clear_kernel, (unsigned)h->sm_count * 4, 256, 0, st, t, (int64_t)h->ws.hcap,
+                    (const unsigned*)h->ws.ctrl);
 }
 
 template <int FMT>
 static cudaError_t launch_insert_flag(wg_dsm* h, bool padded, int items, int64_t ib, unsigned fb, const UniqueArgs& a,
                                       cudaStream_t st) {
-  // the fused hop with the direct table has no insert pass (its sampler inserted every key)
-  if (!(padded && FMT == FMT_DIRECT)) {
+  // the fused hop with the direct or the compact table has no insert pass (its sampler inserted every key)
+  if (!(padded && hop_inserts_in_sampler(h))) {
     cudaError_t e = padded ? launch_pdl(unique_insert_kernel<true, FMT>, (unsigned)ib, UQ_THREADS, 0, st, a)
                            : launch_pdl(unique_insert_kernel<false, FMT>, (unsigned)ib, UQ_THREADS, 0, st, a);
     if (e != cudaSuccess) return e;
@@ -378,7 +380,8 @@ static cudaError_t launch_unique_passes(wg_dsm* h, UniqueArgs& a, bool padded, c
   // about as many lines as it has keys instead of random lines all over the table sized for the
   // largest hop.  Slots outside the prefix, or left by earlier calls, carry older epochs and read as
   // empty.
-  a.ht = HashTable{h->ws.hslots, (unsigned long long)table_prefix(h, a.capT + a.capE), h->ws.compact};
+  a.ht = HashTable{h->ws.hslots, (unsigned long long)table_prefix(h, a.capT + a.capE), h->ws.compact,
+                   reinterpret_cast<HashSlot*>(h->ws.hslots2)};
   a.dt = DirectTable{{h->ws.dtab[0], h->ws.dtab[1]}, h->n};
   a.status = h->ws.status_unique;
   a.ctrl = h->ws.ctrl;

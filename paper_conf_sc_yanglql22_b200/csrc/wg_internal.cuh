@@ -79,6 +79,7 @@ struct __align__(16) HashSlot {
 };
 struct Workspace {
   HashSlot* hslots = nullptr;            // [hcap] append-unique hash table (hash.cuh)
+  unsigned long long* hslots2 = nullptr;  // compact format: [hcap] 8 B words, the odd epoch cycles' table
   int64_t hcap = 0;                      // slots (a multiple of 8, < 2^31); each call uses a prefix
   int compact = 0;                       // 8 B slots {epoch8, key28, pos28} (hash.cuh), else 16 B slots
   // direct table (hash.cuh, graphs small enough that a word per NODE beats a hashed slot per key): two
@@ -200,6 +201,9 @@ __device__ __forceinline__ void st_pad(int64_t* p, int pad32, int64_t i, int64_t
 __device__ __forceinline__ int64_t ld_pad(const int64_t* p, int pad32, int64_t i) {
   return pad32 ? (int64_t)reinterpret_cast<const uint32_t*>(p)[i] : p[i];
 }
+
+// Whether the fused hop's sampler inserts the keys itself (the direct key table: no insert pass).
+bool hop_inserts_in_sampler(const wg_dsm* h);
 
 // launchers (stream-ordered); arguments already validated by the ABI layer
 cudaError_t launch_sample(wg_dsm* h, const int64_t* targets, int64_t cap, const int64_t* d_n, int fanout,

@@ -205,8 +205,15 @@ class DSM:
         """Append Unique key-table format of this handle's workspace (wg_dsm_unique_format):
         WG_UNIQUE_WIDE / WG_UNIQUE_COMPACT / WG_UNIQUE_DIRECT."""
         f = ctypes.c_int32(0)
-        check(lib().wg_dsm_unique_format(self.h, ctypes.byref(f)))
+        check(lib().wg_dsm_unique_format(self.h, ctypes.byref(f), None))
         return f.value
+
+    def hop_insert_pass(self):
+        """True if wg_sample_hop runs a separate insert pass (wide key table); False if its sampler
+        inserts the keys (wg_dsm_unique_format)."""
+        f, ip = ctypes.c_int32(0), ctypes.c_int32(0)
+        check(lib().wg_dsm_unique_format(self.h, ctypes.byref(f), ctypes.byref(ip)))
+        return bool(ip.value)
 
     def debug_set_epoch(self, epoch):
         """Test hook: set the workspace's hash-table epoch (wg_dsm_debug_set_epoch)."""

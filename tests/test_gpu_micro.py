@@ -70,14 +70,18 @@ def test_micro_ceilings_plausible():
     assert lib().wg_micro_atomics(P(table), table.numel(), 3, 8, 8, P(sink), None, st) != 0
 
 
-@pytest.mark.parametrize("fanout,hashed,stages", [(10, False, 3), (40, False, 3), (10, True, 4), (40, True, 4)])
-def test_stage_events_split_a_hop(fanout, hashed, stages):
+@pytest.mark.parametrize("fanout,flags", [(10, 0), (40, 0), (10, "WG_DSM_HASHED"), (40, "WG_DSM_HASHED"),
+                                          (10, "WG_DSM_WIDE_HASH"), (40, "WG_DSM_WIDE_HASH")])
+def test_stage_events_split_a_hop(fanout, flags):
     """wg_dsm_set_stage_events: the events recorded after the sampler, insert (hashed key tables only),
     flag scan and relabel of a hop (warp sampler and block sampler) are ordered and together cover the hop."""
     p = presets.get("tiny")
     dsm, _ = loader.build_dsm(p, on_device=False, extra_keys=p.seeds_per_batch * (1 + fanout),
-                              flags=pkg.WG_DSM_HASHED if hashed else 0)
-    assert dsm.unique_format() == (pkg.WG_UNIQUE_COMPACT if hashed else pkg.WG_UNIQUE_DIRECT)
+                              flags=getattr(pkg, flags) if flags else 0)
+    fmt = {0: pkg.WG_UNIQUE_DIRECT, "WG_DSM_HASHED": pkg.WG_UNIQUE_COMPACT, "WG_DSM_WIDE_HASH": pkg.WG_UNIQUE_WIDE}
+    assert dsm.unique_format() == fmt[flags]
+    stages = 4 if dsm.hop_insert_pass() else 3
+    assert dsm.hop_insert_pass() == (flags != 0)
     S = torch.from_numpy(seeds.seed_nodes(p.n, p.seeds_per_batch, presets.SEED_BASE, 1)).cuda()
     evs = [torch.cuda.Event(enable_timing=True) for _ in range(stages + 1)]
     for e in evs:
