@@ -114,8 +114,7 @@ static wg_status alloc_workspace(wg_dsm* h, int64_t max_keys) {
   w.hcap = cap;
   w.max_keys = max_keys;
   w.status_cap = max_keys / 32 + 2;  // sampler tiles hold >= 32 targets, flag tiles 1024 positions
-  if (cudaMalloc(&w.hslots, cap * sizeof(HashSlot)) != cudaSuccess ||
-      cudaMalloc(&w.status_sample, w.status_cap * 8) != cudaSuccess ||
+  if (cudaMalloc(&w.status_sample, w.status_cap * 8) != cudaSuccess ||
       cudaMalloc(&w.status_unique, w.status_cap * 8) != cudaSuccess ||
       cudaMalloc(&w.excl[0], max_keys * 4) != cudaSuccess || cudaMalloc(&w.excl[1], max_keys * 4) != cudaSuccess ||
       cudaMalloc(&w.excl[2], max_keys * 4) != cudaSuccess || cudaMalloc(&w.excl[3], max_keys * 4) != cudaSuccess ||
@@ -133,7 +132,8 @@ static wg_status alloc_workspace(wg_dsm* h, int64_t max_keys) {
                      max_keys < (int64_t(1) << DPOS_BITS)
                  ? 1
                  : 0;
-  if (w.direct) {
+  if (w.direct) {  // no hash table at all: every append-unique of this workspace keys the direct tables
+    w.hcap = 0;
     const size_t db = (size_t)((h->n + 3) / 4) * 16;  // whole 16 B units (dtab_clear_ahead)
     for (int t = 0; t < 2; ++t) {
       if (cudaMalloc(&w.dtab[t], db) != cudaSuccess) {
@@ -145,16 +145,22 @@ static wg_status alloc_workspace(wg_dsm* h, int64_t max_keys) {
     }
   }
   w.pad32 = !(h->flags & WG_DSM_PAD64) && h->n < (int64_t(1) << 32) ? 1 : 0;
-  if (w.compact) {
+  if (w.direct) {
+  } else if (w.compact) {
     // two tables of 8 B words, alternating per 255-epoch cycle (hash.cuh); every word stale (epoch 0)
-    if (cudaMalloc(&w.hslots2, cap * 8) != cudaSuccess) {
+    if (cudaMalloc(&w.hslots, cap * 8) != cudaSuccess || cudaMalloc(&w.hslots2, cap * 8) != cudaSuccess) {
       cudaGetLastError();
       free_workspace(h);
       return fail(WG_ERR_OOM, "workspace allocation failed (hash table)");
     }
-    WG_CUDA_TRY(cudaMemset(w.hslots, 0, cap * sizeof(HashSlot)));
+    WG_CUDA_TRY(cudaMemset(w.hslots, 0, cap * 8));
     WG_CUDA_TRY(cudaMemset(w.hslots2, 0, cap * 8));
   } else {
+    if (cudaMalloc(&w.hslots, cap * sizeof(HashSlot)) != cudaSuccess) {
+      cudaGetLastError();
+      free_workspace(h);
+      return fail(WG_ERR_OOM, "workspace allocation failed (hash table)");
+    }
     WG_CUDA_TRY(cudaMemset(w.hslots, 0xff, cap * sizeof(HashSlot)));                   // val = all ones
     WG_CUDA_TRY(cudaMemset2D(w.hslots, sizeof(HashSlot), 0, sizeof(unsigned long long), cap));  // key = 0 (empty)
   }
@@ -566,8 +572,9 @@ wg_status wg_dsm_reset_workspace(wg_dsm_t h, wg_stream_t stream) {
   if (h->ws.direct) {
     for (int t = 0; t < 2; ++t) WG_CUDA_TRY(cudaMemsetAsync(h->ws.dtab[t], 0xff, (size_t)((h->n + 3) / 4) * 16, st));
   }
-  if (h->ws.compact) {
-    WG_CUDA_TRY(cudaMemsetAsync(h->ws.hslots, 0, h->ws.hcap * sizeof(HashSlot), st));
+  if (h->ws.direct) {
+  } else if (h->ws.compact) {
+    WG_CUDA_TRY(cudaMemsetAsync(h->ws.hslots, 0, h->ws.hcap * 8, st));
     WG_CUDA_TRY(cudaMemsetAsync(h->ws.hslots2, 0, h->ws.hcap * 8, st));
   } else {
     WG_CUDA_TRY(cudaMemsetAsync(h->ws.hslots, 0xff, h->ws.hcap * sizeof(HashSlot), st));
@@ -595,7 +602,7 @@ wg_status wg_dsm_debug_set_epoch(wg_dsm_t h, uint32_t epoch) {
   // clean, hash.cuh)
   if (h->ws.direct)
     for (int t = 0; t < 2; ++t) WG_CUDA_TRY(cudaMemset(h->ws.dtab[t], 0xff, (size_t)((h->n + 3) / 4) * 16));
-  if (h->ws.compact) {  // likewise the compact tables (the next cycle's table must be clean)
+  if (h->ws.compact && !h->ws.direct) {  // likewise the compact tables (the next cycle's table must be clean)
     WG_CUDA_TRY(cudaMemset(h->ws.hslots, 0, h->ws.hcap * 8));
     WG_CUDA_TRY(cudaMemset(h->ws.hslots2, 0, h->ws.hcap * 8));
   }
