@@ -669,3 +669,40 @@ def test_direct_fused_hop_duplicate_and_bad_targets(fl):
         assert np.array_equal(g, r)
     assert dsm.device_error() == 0
     dsm.destroy()
+
+
+@pytest.mark.parametrize("dim", [4, 100, 132, 260])
+def test_spmm_mean_row_lengths_and_widths(dim):
+    """g-SpMM forward / backward on a hand-made CSR whose rows have 0, 1, 5, 31, 32, 33, 40 and 300 edges
+    (the forward's lane-held ids cover 32 edges, the rest come from a loop) and feature widths of 1 to 65
+    float4 slices (more than one slice per lane), with repeated columns and invalid ids, against the fp64
+    oracle (fp32 tolerance)."""
+    from paper_conf_sc_yanglql22_b200 import layers
+    rng = np.random.default_rng(dim)
+    lens = [0, 1, 5, 31, 32, 33, 40, 300, 7, 0, 64]
+    n_x = 500
+    rows = [rng.integers(0, n_x, k) for k in lens]
+    rp, col = csr_from_rows(rows)
+    X = rng.uniform(-1, 1, (n_x, dim)).astype(np.float32)
+    dY = rng.uniform(-1, 1, (len(lens), dim)).astype(np.float32)
+    rp_t, col_t = torch.from_numpy(rp).cuda(), torch.from_numpy(col.astype(np.int32)).cuda()
+    Y = layers.spmm_mean_forward(rp_t, col_t, torch.from_numpy(X).cuda())
+    assert np.allclose(Y.cpu().numpy(), oracle.spmm_mean_forward(rp, col, X.astype(np.float64)), rtol=0, atol=2e-5)
+    dup = np.bincount(col, minlength=n_x).astype(np.int32)
+    dX = layers.spmm_mean_backward(rp_t, col_t, torch.from_numpy(dup).cuda(), torch.from_numpy(dY).cuda(), n_x)
+    assert np.allclose(dX.cpu().numpy(), oracle.spmm_mean_backward(rp, col, dY.astype(np.float64), n_x),
+                       rtol=1e-5, atol=2e-5)
+    bad = col_t.clone()
+    bad[3] = -1
+    bad[50] = n_x + 7
+    Yb = layers.spmm_mean_forward(rp_t, bad, torch.from_numpy(X).cuda())
+    keep = np.ones(len(col), bool)
+    keep[[3, 50]] = False
+    # skipped edges still count in the mean's denominator (the row's degree)
+    ref = np.zeros((len(lens), dim))
+    for t in range(len(lens)):
+        b, e = rp[t], rp[t + 1]
+        idx = [k for k in range(b, e) if keep[k]]
+        if e > b:
+            ref[t] = X[col[idx]].astype(np.float64).sum(0) / (e - b)
+    assert np.allclose(Yb.cpu().numpy(), ref, rtol=0, atol=2e-5)
