@@ -749,6 +749,7 @@ def bench_wg(args):
     n_single = args.warmup + args.steps
     n_conc = args.warmup + args.steps * P
     wl = Workload(args, p, d, P, args.placement, n_single, n_conc)
+    kph = 4 if wl.dsm.hop_insert_pass() else 3   # kernels per hop (wg_dsm_unique_format)
     clocks = ClockSampler(d.local)
     if d.rank == 0:
         clocks.start()
@@ -843,9 +844,9 @@ def bench_wg(args):
                     "note": f"public API (MiniBatchLoader, {P} batches in flight): per batch pinned-host seeds "
                             "+ (n_seeds, rng_seed) H2D, batch graph, per-hop counts D2H, host-timed from first "
                             "submit to last batch handed out"},
-            # our kernels per batch: 4 per hop (sample, insert, flag-scan, relabel) + one gather (pass A) or
-            # one gather_rows per hop (the shipped incremental graph: passes A' and B)
-            "gpu_launches": args.steps * (4 * len(p.fanouts) + 1) + args.steps * (1 + P) * 5 * len(p.fanouts),
+            # our kernels per batch: 3 per hop (sample, flag-scan, relabel; + insert with a hashed key table)
+            # + one gather (pass A) or one gather_rows per hop (the shipped incremental graph: passes A' and B)
+            "gpu_launches": args.steps * (kph * len(p.fanouts) + 1) + args.steps * (1 + P) * (kph + 1) * len(p.fanouts),
             "clocks": clk,
             "wall_s_timed_region": wall,
             "workload_stats": {**wdesc, "edges_per_hop_mean": hc[:, :, 0].mean(0).tolist(),
