@@ -60,7 +60,9 @@ typedef enum {
 typedef enum { WG_F32 = 0, WG_F16 = 1, WG_BF16 = 2 } wg_dtype;
 
 /* Bits of the latched device error word (wg_device_error). */
-#define WG_DEVERR_ID_RANGE   0x1u  /* a node id outside [0, num_nodes): treated as degree 0 / skipped */
+#define WG_DEVERR_ID_RANGE   0x1u  /* a node id outside [0, num_nodes): treated as degree 0 / skipped
+                                       (a col_idx entry of 0xFFFFFFFF in a uint32 shard with the direct key
+                                       table reads as "no sample"; the error is latched either way) */
 #define WG_DEVERR_DUP_TARGET 0x2u  /* wg_append_unique: duplicate target (A8) */
 #define WG_DEVERR_CAPACITY   0x4u  /* a device count exceeded its host capacity, or the hash table filled */
 #define WG_DEVERR_DEGREE     0x8u  /* a degree >= 2^32 (A3 requires N < 2^32) */
