@@ -30,7 +30,7 @@ import numpy as np  # noqa: E402
 def parse():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=50)
+    ap.add_argument("--steps", type=int, default=200)
     ap.add_argument("--warmup", type=int, default=5)
     ap.add_argument("--config", default="products", choices=["tiny", "products", "papers100m", "mag240m"])
     ap.add_argument("--impl", default="wg", choices=["wg", "reference"])
