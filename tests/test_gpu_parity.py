@@ -647,6 +647,21 @@ def test_unique_format_selection(tiny):
     big = make_dsm(np.zeros((1 << 24) + 2, np.int64), np.zeros(0, np.int64), max_keys=64)
     assert big.unique_format() == pkg.WG_UNIQUE_COMPACT
     big.destroy()
+    # at the boundary (2^24 nodes) the direct table is used; ids near the top of the range round-trip
+    n = 1 << 24
+    rp = np.zeros(n + 1, np.int64)
+    hub = n - 1
+    rp[hub + 1:] = 40  # node n-1 has 40 neighbours, all near the top of the id range (and itself excluded)
+    col = (n - 2 - np.arange(40, dtype=np.int64) * 7919 % (n - 1))
+    edge = make_dsm(rp, col, max_keys=1 << 12)
+    assert edge.unique_format() == pkg.WG_UNIQUE_DIRECT
+    T = np.array([hub, 5, n - 2], np.int64)
+    got = gpu_sample_hop(edge, T, 10, 99, 1)
+    ref = oracle_sample_hop(rp, col, T, 10, 99, 1)
+    for g, r in zip(got, ref):
+        assert np.array_equal(g, r)
+    assert edge.device_error() == 0
+    edge.destroy()
 
 
 @pytest.mark.parametrize("fl", [0, "WG_DSM_HASHED"])
