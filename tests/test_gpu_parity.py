@@ -721,3 +721,26 @@ def test_spmm_mean_row_lengths_and_widths(dim):
         if e > b:
             ref[t] = X[col[idx]].astype(np.float64).sum(0) / (e - b)
     assert np.allclose(Yb.cpu().numpy(), ref, rtol=0, atol=2e-5)
+
+
+@pytest.mark.parametrize("fl", [0, "WG_DSM_HASHED", "WG_DSM_WIDE_HASH"])
+def test_fused_hop_invalid_neighbour_ids(fl):
+    """A col_idx entry outside [0, n) (a corrupt graph, reading B3) through the fused hop of every key-table
+    format: WG_DEVERR_ID_RANGE is latched, the sample stays in the CSR with the invalid id, is never
+    numbered (sub_col -1, not in U), and every valid neighbour is numbered exactly as the oracle numbers the
+    neighbour list without it."""
+    flags = 0 if fl == 0 else getattr(pkg, fl)
+    n = 50
+    rows = [np.array([(v + 1) % n, (v + 7) % n], np.int64) for v in range(n)]
+    rows[3] = np.array([4, n + 11, 9], np.int64)      # one invalid entry (int64 col storage)
+    rp, col = csr_from_rows(rows)
+    dsm = make_dsm(rp, col, max_keys=1 << 10, flags=flags)
+    T = np.array([3, 10, 20], np.int64)
+    rp_g, nb, pos, U, sc, dup = gpu_sample_hop(dsm, T, 8, 5, 0)   # fanout >= degree: whole rows, CSR order
+    assert dsm.device_error() & 0x1
+    assert list(rp_g) == [0, 3, 5, 7] and list(nb[:3]) == [4, n + 11, 9]
+    assert sc[1] == -1 and (n + 11) not in set(U.tolist())
+    keep = np.array([k for k in range(len(nb)) if k != 1])
+    Uo, sco, dupo = oracle.append_unique(T, nb[keep])
+    assert np.array_equal(U, Uo) and np.array_equal(sc[keep], sco)
+    dsm.destroy()
