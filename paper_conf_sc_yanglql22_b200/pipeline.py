@@ -8,9 +8,28 @@ is enqueued without a host sync and can be captured once as a CUDA graph and
 replayed with new seeds / rng_seed written into device buffers.
 """
 
+import contextlib
+import os
+
 import torch
 
 from .dsm import DSM
+
+# NVTX ranges (host-side enqueue of every hop / gather, loader submit / collect) for nsys-style timelines;
+# off unless WG_NVTX=1 in the environment at import (the ranges cost host time on the e2e path).
+_NVTX = os.environ.get("WG_NVTX", "0") == "1"
+
+
+@contextlib.contextmanager
+def nvtx_range(name):
+    if not _NVTX:
+        yield
+        return
+    torch.cuda.nvtx.range_push(name)
+    try:
+        yield
+    finally:
+        torch.cuda.nvtx.range_pop()
 
 
 def capacities(n, fanouts, max_seeds):
@@ -118,8 +137,9 @@ class MiniBatchPipeline:
                 # hop h reuses hop h-EXCL_RING's buffer, so that relabel must be done (include/wg.h)
                 main.wait_stream(self.side)
             if self.fused:
-                d.sample_hop(tgt, m, 0, h, n_targets_dev=tn, seed_dev=self.rng_seed, out=b, cap=tcap, stream=main,
-                             side_stream=self.side)
+                with nvtx_range(f"wg.sample_hop h{h}"):
+                    d.sample_hop(tgt, m, 0, h, n_targets_dev=tn, seed_dev=self.rng_seed, out=b, cap=tcap,
+                                 stream=main, side_stream=self.side)
             else:
                 d.sample_neighbors(tgt, m, 0, h, n_targets_dev=tn, seed_dev=self.rng_seed, out_row_ptr=b["row_ptr"],
                                    out_nbrs=b["nbrs"], out_pos=b["pos"], out_num_edges=b["num_edges"], cap=tcap,
@@ -129,7 +149,8 @@ class MiniBatchPipeline:
                                 out_sub_col=b["sub_col"], out_dup=b["dup"], stream=main)
             if incr:  # rows [|U_{h-1}|, |U_h|) of X are final now
                 self.gside.wait_stream(main)
-                d.gather_rows(b["unique"], self.U_cap[h], prev_nu, b["num_unique"], self.X, stream=self.gside)
+                with nvtx_range(f"wg.gather_rows h{h}"):
+                    d.gather_rows(b["unique"], self.U_cap[h], prev_nu, b["num_unique"], self.X, stream=self.gside)
                 prev_nu = b["num_unique"]
             tgt, tcap, tn = b["unique"], self.U_cap[h], b["num_unique"]
         if gather and self.X is not None and not incr:
@@ -289,6 +310,10 @@ class MiniBatchLoader:
 
     def submit(self, seeds, rng_seed):
         """Enqueue one batch on the next slot; returns the slot index (stream-ordered, no sync)."""
+        with nvtx_range("wg.loader.submit"):
+            return self._submit(seeds, rng_seed)
+
+    def _submit(self, seeds, rng_seed):
         j = self.next_slot
         self.next_slot = (j + 1) % self.depth
         pl, st = self.pipes[j], self.streams[j]
@@ -320,7 +345,8 @@ class MiniBatchLoader:
     def collect(self, j, index=0):
         """Wait (host) for slot j's batch and hand it out (call release(j) when the consumer's
         work on it has been enqueued)."""
-        self.done[j].synchronize()
+        with nvtx_range("wg.loader.collect"):
+            self.done[j].synchronize()
         counts = [(int(e), int(u)) for e, u in self.counts[j].tolist()]
         return PreparedBatch(index, self.pipes[j], counts, self.n_seeds[j])
 

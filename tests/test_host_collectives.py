@@ -116,3 +116,10 @@ def test_bench_reference_arm_nonzero_rank_exits_quietly():
                         "--steps", "1", "--warmup", "0"], cwd=ROOT, capture_output=True, text=True, timeout=300,
                        env=dict(os.environ, RANK="1", WORLD_SIZE="2"))
     assert r.returncode == 0 and not r.stdout.strip()
+
+
+def test_nvtx_range_helper_is_a_noop_without_env():
+    """pipeline.nvtx_range: a no-op context manager unless WG_NVTX=1 (no CUDA needed)."""
+    from paper_conf_sc_yanglql22_b200 import pipeline
+    with pipeline.nvtx_range("x"):
+        pass
