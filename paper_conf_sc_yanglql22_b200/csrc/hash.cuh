@@ -59,8 +59,8 @@ __device__ __forceinline__ unsigned long long chash_load(const HashTable& t, uns
   asm volatile("ld.volatile.global.u64 %0, [%1];" : "=l"(cur) : "l"(&reinterpret_cast<unsigned long long*>(t.slots)[slot]));
   return cur;
 }
-// Insert continuing from slot `slot` whose word was read as `cur` (chash_home / chash_load: callers with
-// several keys issue all their first loads before resolving any).  Returns the slot of `key` (claimed
+// Insert continuing from slot `slot` whose word was read as `cur` (chash_home / chash_load; issuing several
+// keys' first loads before resolving any measured slower, profiles/r02/ab_log.md).  Returns the slot of `key` (claimed
 // with position q if new), or -1 if full; *old = the word seen (0 if this call claimed the slot).
 // Applies the atomicMin (with return if want_old; else only when the word holds a larger position).
 __device__ __forceinline__ long long chash_insert_from(const HashTable& t, int64_t key, int64_t q, unsigned ce,
