@@ -251,19 +251,6 @@ wg_status wg_sample_hop(wg_dsm_t h, const int64_t* d_targets, int64_t n_targets,
 wg_status wg_gather(wg_dsm_t h, const int64_t* d_ids, int64_t n_ids, const int64_t* d_n_ids,
                     void* d_out, wg_stream_t stream);
 
-/* Joint gather of n_batches (<= 16) batches prepared concurrently -- beyond the paper (L176, L182 define
- * the per-batch gather; the results are those of n_batches wg_gather_rows calls): for b < n_batches and
- * i < *d_n_ids[b] (clamped to cap), row i of d_out[b] (pitch out_pitch: a 32 B multiple in [row_bytes,
- * row_bytes rounded up to 32], i.e. DSM.out_pitch; bytes past the row unspecified) = the feature row of
- * d_ids[b][i].  A row held by several batches (power-law hubs are in every batch) is read from the shard
- * ONCE and stored into each: per-node linked lists built with one atomicExch per row (a per-handle table
- * of num_nodes words, allocated at the first call), then one load per distinct row and 32 B piece.
- * Invalid ids give zero rows and latch WG_DEVERR_ID_RANGE.  Requires n_batches * cap < 2^24; not CUDA-graph
- * capturable (a host-side per-call tag); stream-ordered.  The pointer arrays are host arrays of device
- * pointers.  Errors: WG_ERR_INVALID_ARG, WG_ERR_UNSUPPORTED (pitch / size), WG_ERR_CUDA. */
-wg_status wg_gather_joint(wg_dsm_t h, int32_t n_batches, const int64_t* const* d_ids, int64_t cap,
-                          const int64_t* const* d_n_ids, void* const* d_out, int64_t out_pitch, wg_stream_t stream);
-
 /* ---- Distributed-memory global gather: the comparison baseline (PAPER.md L178-180,
  * Fig. 4 left, Fig. 10).  The caller drives the five steps with NCCL all-to-alls:
  *   1 wg_bucket_by_owner  2 all-to-all counts + ids  3 wg_gather on the received ids

@@ -76,7 +76,6 @@ def lib():
     L.wg_dsm_debug_set_epoch.argtypes = [P, ctypes.c_uint32]
     L.wg_dsm_set_stage_events.argtypes = [P, P, I32]
     L.wg_dsm_unique_format.argtypes = [P, P, P]
-    L.wg_gather_joint.argtypes = [P, I32, P, I64, P, P, I64, P]
     L.wg_micro_random_read.argtypes = [P, I64, I32, I32, I32, P, P, P]
     L.wg_micro_atomics.argtypes = [P, I64, I32, I32, I32, P, P, P]
     for f in ("wg_dsm_create", "wg_dsm_fork", "wg_dsm_local_view", "wg_dsm_shard_info", "wg_dsm_feat_layout",
@@ -84,7 +83,7 @@ def lib():
               "wg_dsm_chase", "wg_spmm_mean_forward", "wg_spmm_mean_backward", "wg_bucket_by_owner", "wg_rows_permute",
               "wg_device_error", "wg_dsm_reset_workspace", "wg_dsm_set_gather_occupancy",
               "wg_dsm_debug_set_epoch", "wg_micro_random_read", "wg_micro_atomics", "wg_dsm_set_stage_events",
-              "wg_dsm_unique_format", "wg_gather_joint"):
+              "wg_dsm_unique_format"):
         getattr(L, f).restype = ctypes.c_int
     L.wg_last_error.restype = ctypes.c_char_p
     L.wg_last_error.argtypes = []
@@ -102,4 +101,4 @@ def check(status):
 EXPORTS = ["wg_dsm_create", "wg_dsm_fork", "wg_dsm_local_view", "wg_dsm_shard_info", "wg_dsm_feat_layout", "wg_dsm_destroy", "wg_sample_neighbors",
            "wg_append_unique", "wg_sample_hop", "wg_gather", "wg_gather_rows", "wg_dsm_chase", "wg_spmm_mean_forward",
            "wg_spmm_mean_backward", "wg_bucket_by_owner", "wg_rows_permute", "wg_device_error", "wg_dsm_reset_workspace", "wg_dsm_set_gather_occupancy",
-           "wg_dsm_debug_set_epoch", "wg_micro_random_read", "wg_micro_atomics", "wg_dsm_set_stage_events", "wg_dsm_unique_format", "wg_gather_joint", "wg_last_error", "wg_version"]
+           "wg_dsm_debug_set_epoch", "wg_micro_random_read", "wg_micro_atomics", "wg_dsm_set_stage_events", "wg_dsm_unique_format", "wg_last_error", "wg_version"]

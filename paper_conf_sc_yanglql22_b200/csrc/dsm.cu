@@ -99,10 +99,6 @@ static void free_workspace(wg_dsm* h) {
   cudaFree(w.pos_pad);
   cudaFree(w.cnt);
   cudaFree(w.ctrl);
-  cudaFree(w.jhead);
-  cudaFree(w.jnext);
-  cudaFree(w.jtails);
-  cudaFree(w.jcnt);
   w = Workspace{};
 }
 
@@ -558,26 +554,6 @@ wg_status wg_gather_rows(wg_dsm_t h, const int64_t* d_ids, int64_t n_ids, const 
 wg_status wg_gather(wg_dsm_t h, const int64_t* d_ids, int64_t n_ids, const int64_t* d_n_ids, void* d_out,
                     wg_stream_t stream) {
   return wg_gather_rows(h, d_ids, n_ids, nullptr, d_n_ids, d_out, 0, stream);
-}
-
-wg_status wg_gather_joint(wg_dsm_t h, int32_t n_batches, const int64_t* const* d_ids, int64_t cap,
-                          const int64_t* const* d_n_ids, void* const* d_out, int64_t out_pitch, wg_stream_t stream) {
-  if (!h) return fail(WG_ERR_INVALID_ARG, "handle is NULL");
-  if (n_batches < 1 || n_batches > JOINT_MAX || cap < 0 || !d_ids || !d_n_ids || !d_out)
-    return fail(WG_ERR_INVALID_ARG, "bad arguments (1 <= n_batches <= 16, pointer arrays required)");
-  for (int b = 0; b < n_batches; ++b)
-    if (cap > 0 && (!d_ids[b] || !d_n_ids[b] || !d_out[b])) return fail(WG_ERR_INVALID_ARG, "null batch pointer");
-  if (h->row_bytes == 0) return fail(WG_ERR_INVALID_ARG, "DSM has no feature table");
-  if (out_pitch % 32 != 0 || out_pitch < h->row_bytes || out_pitch > round_up(h->row_bytes, 32) ||
-      (h->tail_pitch == 0 && out_pitch > h->feat_stride) || (h->tail_pitch != 0 && h->body_bytes % 32 != 0) ||
-      h->feat_stride % 32 != 0)
-    return fail(WG_ERR_UNSUPPORTED, "joint gather needs a 32 B-multiple output pitch (DSM.out_pitch) and 32 B rows pieces");
-  if ((int64_t)n_batches * cap >= (int64_t(1) << 24)) return fail(WG_ERR_UNSUPPORTED, "n_batches * cap must be < 2^24");
-  cudaSetDevice(h->device);
-  if (cap == 0) return WG_OK;
-  cudaError_t e = launch_gather_joint(h, n_batches, d_ids, cap, d_n_ids, d_out, out_pitch, (cudaStream_t)stream);
-  if (e != cudaSuccess) return fail(WG_ERR_CUDA, std::string("joint gather: ") + cudaGetErrorString(e));
-  return WG_OK;
 }
 
 wg_status wg_device_error(wg_dsm_t h, uint32_t* code, int32_t clear) {

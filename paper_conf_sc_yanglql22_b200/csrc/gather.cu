@@ -215,168 +215,6 @@ __global__ void __launch_bounds__(GATHER_THREADS, MINB) gather_kernel(const Gath
   KT_END(3, "gather", n);
 }
 
-// ---------------------------------------------------------------- joint gather
-// G batches prepared concurrently share rows (power-law hubs are in every batch: on products-shaped
-// batches 8 unique lists of 610k ids hold only ~2.1M distinct ids).  The joint gather reads every
-// distinct row ONCE and stores it into every batch that holds it.  Triple t = b * cap + p stands for row
-// p of batch b.
-//   link   each valid triple pushes itself on its node's list: old = atomicExch(head[v], tag | t),
-//          next[t] = old (or -1 when old is of another call: t is the list's tail, appended to `tails`
-//          by a warp-aggregated atomic).  Invalid ids: the row is zeroed, WG_DEVERR_ID_RANGE latched.
-//   copy   per (tail, 32 B chunk): one load of the chunk from the owner's shard, then the walk head ->
-//          ... -> tail stores it into each output row holding v (one per batch for unique lists).
-// The heads carry an 8-bit per-call tag (host counter; the table is reset to "empty" when it wraps), so
-// nothing is cleared per call.
-struct JointArgs {
-  ShardView s;
-  const int64_t* ids[JOINT_MAX];
-  const int64_t* d_n[JOINT_MAX];
-  uint8_t* out[JOINT_MAX];
-  int G;
-  int64_t cap;
-  FastDiv capdiv;
-  int64_t pitch;
-  FastDiv cpr;
-  unsigned tag;
-  unsigned* head;
-  int32_t* next;
-  int32_t* tails;
-  unsigned* cnt;
-  unsigned* ctrl;
-};
-
-__global__ void __launch_bounds__(256) joint_link_kernel(const JointArgs a) {
-  pdl_enter();
-  __shared__ int64_t sn[JOINT_MAX];
-  if (threadIdx.x < a.G) {
-    int64_t v = *a.d_n[threadIdx.x];
-    sn[threadIdx.x] = v < 0 ? 0 : (v > a.cap ? a.cap : v);
-  }
-  __syncthreads();
-  const int64_t total = (int64_t)a.G * a.cap;  // < 2^24
-  const int lane = threadIdx.x & 31;
-  const unsigned stride = gridDim.x * blockDim.x;
-  for (unsigned t0 = blockIdx.x * blockDim.x; t0 < total; t0 += stride) {  // warp-uniform trip count
-    const unsigned t = t0 + threadIdx.x;
-    bool tail = false;
-    if (t < total) {
-      const unsigned b = a.capdiv.div(t);
-      const unsigned p = t - b * (unsigned)a.cap;
-      if (p < sn[b]) {
-        const int64_t v = a.ids[b][p];
-        if (v < 0 || v >= a.s.n) {
-          latch_error(&a.ctrl[CTRL_ERR], WG_DEVERR_ID_RANGE);
-          u32x8 z{};
-          for (unsigned c = 0; c < a.cpr.d; ++c) st_out<u32x8>(reinterpret_cast<u32x8*>(a.out[b] + p * a.pitch) + c, z);
-        } else {
-          const unsigned old = atomicExch(&a.head[v], (a.tag << 24) | t);
-          tail = (old >> 24) != a.tag;
-          a.next[t] = tail ? -1 : (int32_t)(old & 0xFFFFFFu);
-        }
-      }
-    }
-    const unsigned m = __ballot_sync(FULL_MASK, tail);
-    if (m) {
-      unsigned base = 0;
-      if (lane == 0) base = atomicAdd(a.cnt, (unsigned)__popc(m));
-      base = __shfl_sync(FULL_MASK, base, 0);
-      if (tail) a.tails[base + __popc(m & ((1u << lane) - 1u))] = (int32_t)t;
-    }
-  }
-}
-
-template <int MINB>
-__global__ void __launch_bounds__(GATHER_THREADS, MINB) joint_copy_kernel(const JointArgs a) {
-  pdl_enter();
-  const unsigned ntails = *a.cnt;
-  const unsigned cpr = a.cpr.d;
-  const unsigned total = ntails * cpr;  // < 2^24 * 128 (checked on the host)
-  const unsigned stride = gridDim.x * GATHER_THREADS;
-  const unsigned long long pol = l2_evict_last_policy();
-  for (unsigned c = blockIdx.x * GATHER_THREADS + threadIdx.x; c < total; c += stride) {
-    const unsigned i = a.cpr.div(c);
-    const unsigned k = c - i * cpr;
-    const unsigned tt = (unsigned)a.tails[i];
-    const unsigned tb = a.capdiv.div(tt);
-    const int64_t v = a.ids[tb][tt - tb * (unsigned)a.cap];
-    int o;
-    int64_t l;
-    owner_local(a.s, v, o, l);
-    const u32x8 val = ld_row_chunk<u32x8>(a.s, o, l, k * 32u, pol);
-    unsigned t = a.head[v] & 0xFFFFFFu;
-    for (;;) {  // head -> ... -> this tail: every row of every batch that holds v (repeats included)
-      const unsigned b = a.capdiv.div(t);
-      const unsigned p = t - b * (unsigned)a.cap;
-      st_out<u32x8>(reinterpret_cast<u32x8*>(a.out[b] + p * a.pitch) + k, val);
-      if (t == tt) break;
-      t = (unsigned)a.next[t];
-    }
-  }
-}
-
-cudaError_t launch_gather_joint(wg_dsm* h, int G, const int64_t* const* ids, int64_t cap, const int64_t* const* d_n,
-                                void* const* out, int64_t out_pitch, cudaStream_t st) {
-  Workspace& w = h->ws;
-  const int64_t need = (int64_t)G * cap;
-  if (!w.jhead) {
-    const size_t hb = (size_t)h->n * 4;
-    if (cudaMalloc(&w.jhead, hb > 0 ? hb : 4) != cudaSuccess || cudaMalloc(&w.jcnt, 4) != cudaSuccess) return cudaErrorMemoryAllocation;
-    cudaError_t e = cudaMemsetAsync(w.jhead, 0xff, hb, st);  // tag 255: never a call's tag
-    if (e != cudaSuccess) return e;
-  }
-  if (w.jcap < need) {
-    cudaFree(w.jnext);
-    cudaFree(w.jtails);
-    w.jnext = nullptr;
-    w.jtails = nullptr;
-    if (cudaMalloc(&w.jnext, need * 4) != cudaSuccess || cudaMalloc(&w.jtails, need * 4) != cudaSuccess) {
-      w.jcap = 0;
-      return cudaErrorMemoryAllocation;
-    }
-    w.jcap = need;
-  }
-  // per-call tag 1..254; the heads are reset when the counter wraps
-  w.jepoch = w.jepoch >= 254 ? 0 : w.jepoch;
-  if (w.jepoch == 0) {
-    cudaError_t e = cudaMemsetAsync(w.jhead, 0xff, (size_t)h->n * 4, st);
-    if (e != cudaSuccess) return e;
-  }
-  w.jepoch += 1;
-  JointArgs a{};
-  a.s = h->view;
-  for (int b = 0; b < G; ++b) {
-    a.ids[b] = ids[b];
-    a.d_n[b] = d_n[b];
-    a.out[b] = static_cast<uint8_t*>(out[b]);
-  }
-  a.G = G;
-  a.cap = cap;
-  a.capdiv = FastDiv((unsigned)cap);
-  a.pitch = out_pitch;
-  a.cpr = FastDiv((unsigned)(out_pitch / 32));
-  a.tag = w.jepoch;
-  a.head = w.jhead;
-  a.next = w.jnext;
-  a.tails = w.jtails;
-  a.cnt = w.jcnt;
-  a.ctrl = w.ctrl;
-  cudaError_t e = cudaMemsetAsync(w.jcnt, 0, 4, st);
-  if (e != cudaSuccess) return e;
-  int64_t lb = (need + 255) / 256;
-  const int64_t lmax = (int64_t)h->sm_count * 8;
-  lb = lb < 1 ? 1 : (lb > lmax ? lmax : lb);
-  e = launch_pdl(joint_link_kernel, (unsigned)lb, 256, 0, st, a);
-  if (e != cudaSuccess) return e;
-  static int occ = 0;
-  if (!occ) {
-    int nb = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, joint_copy_kernel<GATHER_MINB>, GATHER_THREADS, 0);
-    occ = nb > 0 ? nb : 4;
-  }
-  const int per_sm = (h->gather_bps > 0 && h->gather_bps < occ) ? h->gather_bps : occ;
-  return launch_pdl(joint_copy_kernel<GATHER_MINB>, (unsigned)(h->sm_count * per_sm), GATHER_THREADS, 0, st, a);
-}
-
 cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int64_t* d_n, const int64_t* d_begin,
                           void* out, int64_t out_pitch, cudaStream_t st) {
   const int64_t rb = h->row_bytes;

@@ -100,14 +100,6 @@ struct Workspace {
   int32_t* pos_pad = nullptr;            // [max_keys] adjacency positions of the padded slots
   int32_t* cnt = nullptr;                // [max_keys] per-target sample counts min(M, deg)
   unsigned* ctrl = nullptr;              // [16] control words (see CTRL_*)
-  // joint gather (wg_gather_joint), allocated at its first call: per-node list heads {tag8, triple24},
-  // per-triple next links, the list tails (one per distinct node) and their count
-  unsigned* jhead = nullptr;
-  int32_t* jnext = nullptr;
-  int32_t* jtails = nullptr;
-  unsigned* jcnt = nullptr;
-  int64_t jcap = 0;                      // triples the link arrays hold
-  unsigned jepoch = 0;                   // host-side tag of the last call (1..254)
   int64_t max_keys = 0;
 };
 enum { CTRL_ERR = 0, CTRL_EPOCH = 1, CTRL_DONE_SAMPLE = 2, CTRL_DONE_UNIQUE = 3, CTRL_WORDS = 16 };
@@ -226,7 +218,4 @@ cudaError_t launch_hop(wg_dsm* h, const int64_t* T, int64_t capT, const int64_t*
                        cudaStream_t st, cudaStream_t side);
 cudaError_t launch_gather(wg_dsm* h, const int64_t* ids, int64_t cap, const int64_t* d_n, const int64_t* d_begin,
                           void* out, int64_t out_pitch, cudaStream_t st);
-constexpr int JOINT_MAX = 16;  // batches per joint gather
-cudaError_t launch_gather_joint(wg_dsm* h, int G, const int64_t* const* ids, int64_t cap, const int64_t* const* d_n,
-                                void* const* out, int64_t out_pitch, cudaStream_t st);
 }  // namespace wg

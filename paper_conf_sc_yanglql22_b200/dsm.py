@@ -313,17 +313,6 @@ class DSM:
                                    _stream(stream)))
         return out
 
-    def gather_joint(self, ids_list, cap, n_list, outs, stream=None):
-        """Joint gather of several batches (wg_gather_joint): outs[b][i] = row of ids_list[b][i] for i <
-        n_list[b] (device int64 counts); a row shared by several batches is read once.  outs: uint8
-        [*, pitch] tensors with pitch = DSM.out_pitch()."""
-        G = len(ids_list)
-        P = ctypes.c_void_p * G
-        ids = P(*[t.data_ptr() for t in ids_list])
-        ns = P(*[t.data_ptr() for t in n_list])
-        os_ = P(*[t.data_ptr() for t in outs])
-        check(lib().wg_gather_joint(self.h, G, ids, int(cap), ns, os_, outs[0].stride(0), _stream(stream)))
-
     def set_gather_occupancy(self, blocks_per_sm):
         """Resident gather blocks per SM for this handle's gathers (0 = occupancy maximum);
         read at enqueue / capture time (wg_dsm_set_gather_occupancy)."""

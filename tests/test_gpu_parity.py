@@ -744,47 +744,3 @@ def test_fused_hop_invalid_neighbour_ids(fl):
     Uo, sco, dupo = oracle.append_unique(T, nb[keep])
     assert np.array_equal(U, Uo) and np.array_equal(sc[keep], sco)
     dsm.destroy()
-
-
-@pytest.mark.parametrize("G,dim,dtype,flags", [(8, 100, "fp32", 0), (3, 128, "fp32", 0), (1, 100, "fp32", 0),
-                                               (16, 36, "fp32", 0), (5, 200, "fp16", "WG_DSM_WHOLE_ROWS")])
-def test_gather_joint_vs_per_batch(G, dim, dtype, flags):
-    """wg_gather_joint (rows shared by several batches read once, per-node lists) gives every batch exactly
-    the rows wg_gather gives it: power-law-overlapping unique lists, a list with repeats, an empty batch,
-    counts below the capacity, invalid ids (zero rows + WG_DEVERR_ID_RANGE), and repeated calls (tags)."""
-    fl = getattr(pkg, flags) if flags else 0
-    n = 5000
-    rp = np.zeros(n + 1, dtype=np.int64)
-    feat = features.feature_bytes(presets.FEAT_SEED, np.arange(n), dim, dtype)
-    dsm = make_dsm(rp, np.zeros(0, np.int64), feat, dim, dtype, flags=fl)
-    rb, pitch = dsm.row_bytes, dsm.out_pitch()
-    rng = np.random.default_rng(G * 100 + dim)
-    cap = 3000
-    for call in range(3):
-        lists = []
-        for b in range(G):
-            k = int(rng.integers(0, cap + 1)) if b != 1 else 0
-            ids = np.unique(np.minimum((rng.random(3 * k + 1) ** 2.5 * n).astype(np.int64), n - 1))[:k]
-            rng.shuffle(ids)
-            if b == 2 and len(ids) > 10:
-                ids[5] = ids[3]            # a repeat inside one batch
-            lists.append(ids)
-        ids_t = [torch.from_numpy(np.concatenate([l, np.zeros(cap - len(l), np.int64)])).cuda() for l in lists]
-        n_t = [torch.tensor([len(l)], dtype=torch.int64, device="cuda") for l in lists]
-        outs = [torch.full((cap, pitch), 0xAB, dtype=torch.uint8, device="cuda") for _ in range(G)]
-        dsm.gather_joint(ids_t, cap, n_t, outs)
-        torch.cuda.synchronize()
-        for b, l in enumerate(lists):
-            got = outs[b][:len(l), :rb].cpu().numpy()
-            assert np.array_equal(got, oracle.gather(feat, np.arange(n), l)), (call, b)
-            assert (outs[b][len(l):].cpu().numpy() == 0xAB).all()
-    assert dsm.device_error() == 0
-    bad = [torch.tensor([3, n + 4, -1, 7], dtype=torch.int64, device="cuda")]
-    out = [torch.full((4, pitch), 0xAB, dtype=torch.uint8, device="cuda")]
-    dsm.gather_joint(bad, 4, [torch.tensor([4], dtype=torch.int64, device="cuda")], out)
-    torch.cuda.synchronize()
-    o = out[0][:, :rb].cpu().numpy()
-    assert dsm.device_error() & 0x1
-    assert (o[1] == 0).all() and (o[2] == 0).all()
-    assert np.array_equal(o[[0, 3]], oracle.gather(feat, np.arange(n), np.array([3, 7])))
-    dsm.destroy()
